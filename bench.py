@@ -1,0 +1,476 @@
+#!/usr/bin/env python
+"""Benchmark of the breadth-first D&C hot path on B200 (one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl dc|reference]
+                    [--workload sort_u32|sort_kv|sort_u32_small|maxsub] [--dist uniform]
+
+A step is one pass of the whole hot path over one batch of synthetic input:
+for the sort workloads, NK1 (fused bottom levels) + every global merge level
+(NK2 + NK3) of a stable mergesort of n keys; for max-subarray, NK4 + NK5.
+
+Default workload (N=1): BASELINE configs[2], mergesort of 2^28 uniform uint32
+keys on one B200 -- the configuration the metric "sorted keys/sec (32-bit,
+2^28-2^30)" is quoted on.  N>1: configs[4], 2^30 keys sharded over N GPUs with
+the cross-GPU top-level merge (see paper_conf_ipps_lopez_ortizss13_b200/dist.py).
+
+Timing: inputs resident in HBM; before every step (untimed) the keys are
+restored from a pristine device copy and L2 is flushed by writing a 512 MiB
+buffer; each step is bracketed by CUDA events on the launching stream; W
+warm-up steps, then exactly K timed steps between barrier + synchronize.
+Per-kernel device times come from the library's own event instrumentation
+(dc_plan_kernel_time) over the same timed steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (description, n, kind)
+    "sort_u32": ("mergesort of 2^28 uint32 keys on 1 B200 (BASELINE configs[2])", 1 << 28, "sort"),
+    "sort_kv": ("stable mergesort of 2^28 uint32 key + uint32 value pairs (configs[3])", 1 << 28,
+                "sort_kv"),
+    "sort_u32_small": ("mergesort of 2^20 uniform uint32 keys (configs[0])", 1 << 20, "sort"),
+    "maxsub": ("max-subarray-sum D&C on 2^24 int32 values (configs[1])", 1 << 24, "maxsub"),
+    "sort_u32_2p30": ("mergesort of 2^30 uint32 keys sharded over N B200 (configs[4])", 1 << 30,
+                      "sort"),
+}
+METRIC = "sorted keys/sec (32-bit, 2^28-2^30) at 1/2/4/8 B200; per-pass HBM GB/s vs peak"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["dc", "reference"], default="dc")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS), default=None)
+    ap.add_argument("--dist", default="uniform")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- helpers
+
+def peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(path))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def ncu_traffic(kernel: str, workload: str):
+    """dram bytes per launch of `kernel` from the committed ncu --set full summary."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(path))
+        return d[workload][kernel]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.p is not None:
+            self.p.terminate()
+            try:
+                self.p.wait(timeout=5)
+            except Exception:
+                self.p.kill()
+
+    def summary(self):
+        self.f.flush()
+        rows = []
+        for line in open(self.f.name):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append(parts)
+            except ValueError:
+                pass
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def cpu_info():
+    model = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return model, os.cpu_count()
+
+
+# --------------------------------------------------------- oracle timings
+
+def oracle_sort_sample(n_total: int, dist: str, kv: bool, budget_s: float = 12.0,
+                       sample_n: int = 1 << 24):
+    """The oracle (Alg 6, 1 thread) on prefixes of the workload, as it stands."""
+    import numpy as np
+
+    import dcgen
+    import oracle
+
+    sample_n = min(sample_n, n_total)
+    keys = dcgen.sort_keys(n_total, dist, seed=3, start=0, count=sample_n).numpy().view(np.uint32)
+    vals = np.arange(sample_n, dtype=np.uint32) if kv else None
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        oracle.mergesort(keys, vals)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el > budget_s or reps >= 20:
+            break
+    return reps * sample_n / el, reps, sample_n, el
+
+
+def oracle_maxsub_sample(n_total: int, dist: str, budget_s: float = 12.0):
+    import dcgen
+    import oracle
+
+    x = dcgen.maxsub_input(n_total, dist, seed=2).numpy()
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        oracle.maxsub(x)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el > budget_s or reps >= 50:
+            break
+    return reps * x.size / el, reps, x.size, el
+
+
+# ------------------------------------------------------------ reference arm
+
+def run_reference(args, wl):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    desc, n, kind = WORKLOADS[wl]
+    model, cores = cpu_info()
+    step_times = []
+    if kind == "maxsub":
+        import dcgen
+        import oracle
+
+        x = dcgen.maxsub_input(n, args.dist, seed=2).numpy()
+        sample_n = n
+        for i in range(args.warmup + args.steps):
+            t0 = time.perf_counter()
+            oracle.maxsub(x)
+            if i >= args.warmup:
+                step_times.append(time.perf_counter() - t0)
+        unit = "elements/s"
+        sample = f"oracle recursive D&C max-subarray of the full 2^24 input, 1 thread, per step"
+    else:
+        import numpy as np
+
+        import dcgen
+        import oracle
+
+        sample_n = 1 << 22
+        keys = dcgen.sort_keys(n, args.dist, seed=3, count=sample_n).numpy().view(np.uint32)
+        vals = np.arange(sample_n, dtype=np.uint32) if kind == "sort_kv" else None
+        for i in range(args.warmup + args.steps):
+            t0 = time.perf_counter()
+            oracle.mergesort(keys, vals)
+            if i >= args.warmup:
+                step_times.append(time.perf_counter() - t0)
+        unit = "keys/s"
+        sample = (f"oracle Alg 6 recursive mergesort (1 thread) of the first 2^22 keys of the "
+                  f"{desc} workload, per step")
+    t = statistics.mean(step_times)
+    v = sample_n / t
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": unit, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
+        "higher_is_better": True, "scaling": "strong" if args.gpus > 1 else "weak",
+        "vs_baseline": None, "dtype": "u32" if kind != "maxsub" else "i32",
+        "data": "synthetic (counter-based splitmix64)",
+        "config": {"workload": wl, "description": desc, "n": n, "dist": args.dist,
+                   "sample_n": sample_n},
+        "cpu_baseline": {"value": v, "unit": unit, "cores": 1, "kind": "oracle",
+                         "sample": sample, "cpu": model, "host_cores": cores},
+        "e2e": {"value": v, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+# ------------------------------------------------------------------ our arm
+
+def run_dc(args, wl):
+    import torch
+
+    import dcgen
+    import paper_conf_ipps_lopez_ortizss13_b200 as dc
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        from paper_conf_ipps_lopez_ortizss13_b200 import dist as dcdist
+
+        return dcdist.bench_main(args, wl, WORKLOADS, METRIC)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    desc, n, kind = WORKLOADS[wl]
+    if kind == "maxsub":
+        return run_dc_maxsub(args, wl, desc, n)
+
+    kv = kind == "sort_kv"
+    pristine_k = dcgen.sort_keys(n, args.dist, seed=3, device=dev)
+    keys = torch.empty_like(pristine_k)
+    vals = torch.empty_like(pristine_k) if kv else None
+    pristine_v = dcgen.sort_vals(n, device=dev) if kv else None
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    plan = dc.Plan(n)
+    stream = torch.cuda.current_stream(dev)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.warmup + args.steps)]
+
+    def prep():
+        keys.copy_(pristine_k)
+        if kv:
+            vals.copy_(pristine_v)
+        flush.zero_()
+
+    for i in range(args.warmup):
+        prep()
+        ev[i][0].record(stream)
+        plan.sort_(keys, vals, key_type="u32")
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    plan.enable_timing(True)
+    launches0 = plan.launch_count()
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        for i in range(args.warmup, args.warmup + args.steps):
+            prep()
+            ev[i][0].record(stream)
+            plan.sort_(keys, vals, key_type="u32")
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    launches = plan.launch_count() - launches0
+    kt = plan.kernel_times()
+    plan.enable_timing(False)
+    step_ms = [ev[i][0].elapsed_time(ev[i][1]) for i in range(args.warmup, args.warmup + args.steps)]
+    ms = statistics.mean(step_ms)
+    value = n / (ms / 1e3)
+
+    # correctness spot-check of the last timed output (cheap invariant, untimed)
+    k64 = keys.to(torch.int64) & 0xFFFFFFFF
+    sorted_ok = bool((k64[1:] >= k64[:-1]).all())
+    del k64
+
+    sched = plan.schedule()
+    peak, peak_src = peaks()
+    bytes_per_key = 16 if kv else 8
+    nk3_ms, nk3_n = kt["nk3_merge"]
+    nk1_ms, nk1_n = kt["nk1_blocksort"]
+    nk2_ms, nk2_n = kt["nk2_partition"]
+    nk3_avg = nk3_ms / max(nk3_n, 1)
+    achieved = bytes_per_key * n / (nk3_avg / 1e3) / 1e9 if nk3_n else None
+    nk1_avg = nk1_ms / max(nk1_n, 1)
+    roofline = {
+        "kernel": "nk3_merge (one global merge level)",
+        "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+        "frac": achieved / peak if achieved else None,
+        "traffic": ncu_traffic("nk3_merge", wl),
+        "algorithmic_bytes_per_launch": bytes_per_key * n,
+        "avg_launch_ms": nk3_avg, "peak_source": peak_src,
+        "share_of_step": nk3_ms / args.steps / ms if ms else None,
+    }
+    kernels = {
+        "nk1_blocksort": {"avg_ms": nk1_avg, "launches_per_step": nk1_n / args.steps,
+                          "hbm_gbs": bytes_per_key * n / (nk1_avg / 1e3) / 1e9 if nk1_n else None,
+                          "share_of_step": nk1_ms / args.steps / ms},
+        "nk2_partition": {"avg_ms": nk2_ms / max(nk2_n, 1), "launches_per_step": nk2_n / args.steps,
+                          "share_of_step": nk2_ms / args.steps / ms},
+        "nk3_merge": {"avg_ms": nk3_avg, "launches_per_step": nk3_n / args.steps,
+                      "hbm_gbs": achieved, "share_of_step": nk3_ms / args.steps / ms},
+    }
+
+    e2e = None
+    if not args.no_e2e:
+        e2e = e2e_sort(args, plan, n, kv, pristine_k, pristine_v)
+
+    cpu = None
+    if not args.no_cpu_baseline:
+        v, reps, sn, el = oracle_sort_sample(n, args.dist, kv)
+        model, cores = cpu_info()
+        cpu = {"value": v, "unit": "keys/s", "cores": 1, "kind": "oracle",
+               "sample": f"oracle Alg 6 recursive mergesort, 1 thread, {reps} x the first {sn} "
+                         f"keys of this workload ({el:.1f} s)",
+               "cpu": model, "host_cores": cores}
+
+    print(json.dumps({
+        "metric": METRIC, "value": value, "unit": "keys/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic (counter-based splitmix64)",
+        "config": {"workload": wl, "description": desc, "n": n, "dist": args.dist,
+                   "key_type": "u32", "values": kv, "tile": sched["tile"],
+                   "fused_levels": sched["fused_levels"], "global_passes": sched["global_passes"],
+                   "l2": "flushed before every step (512 MiB write); input 1 GiB > L2",
+                   "step_ms_min": min(step_ms), "step_ms_max": max(step_ms),
+                   "sorted_check": sorted_ok},
+        "roofline": roofline, "kernels": kernels, "gpu_launches": launches,
+        "clocks": clk.summary(), "e2e": e2e, "cpu_baseline": cpu,
+    }), flush=True)
+
+
+def e2e_sort(args, plan, n, kv, pristine_k, pristine_v):
+    """Same metric through the C ABI with pinned HOST buffers: H2D + sort + D2H."""
+    import torch
+
+    hk0 = pristine_k.cpu()
+    hk = torch.empty_like(hk0).pin_memory()
+    hv0 = pristine_v.cpu() if kv else None
+    hv = torch.empty_like(hv0).pin_memory() if kv else None
+    stream = torch.cuda.current_stream()
+    times = []
+    for i in range(args.warmup + args.steps):
+        hk.copy_(hk0)
+        if kv:
+            hv.copy_(hv0)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        plan.sort_host_(hk, hv, key_type="u32")
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if i >= args.warmup:
+            times.append(e0.elapsed_time(e1))
+    ms = statistics.mean(times)
+    return {"value": n / (ms / 1e3), "unit": "keys/s", "ms_per_step": ms,
+            "h2d_bytes_per_step": n * 4 * (2 if kv else 1),
+            "d2h_bytes_per_step": n * 4 * (2 if kv else 1)}
+
+
+def run_dc_maxsub(args, wl, desc, n):
+    import torch
+
+    import dcgen
+    import paper_conf_ipps_lopez_ortizss13_b200 as dc
+
+    dev = torch.device("cuda", torch.cuda.current_device())
+    x = dcgen.maxsub_input(n, args.dist if args.dist != "uniform" else "uniform", seed=2,
+                           device=dev)
+    out = torch.empty(3, dtype=torch.int64, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    plan = dc.Plan(n)
+    stream = torch.cuda.current_stream(dev)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.warmup + args.steps)]
+    for i in range(args.warmup):
+        flush.zero_()
+        ev[i][0].record(stream)
+        plan.max_subarray_async(x, out)
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    plan.enable_timing(True)
+    l0 = plan.launch_count()
+    with ClockSampler(dev.index) as clk:
+        for i in range(args.warmup, args.warmup + args.steps):
+            flush.zero_()
+            ev[i][0].record(stream)
+            plan.max_subarray_async(x, out)
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+    launches = plan.launch_count() - l0
+    kt = plan.kernel_times()
+    plan.enable_timing(False)
+    step_ms = [ev[i][0].elapsed_time(ev[i][1]) for i in range(args.warmup, args.warmup + args.steps)]
+    ms = statistics.mean(step_ms)
+    k_ms, k_n = kt["nk4_maxsub"]
+    avg = k_ms / max(k_n, 1)
+    peak, src = peaks()
+    ach = 4 * n / (avg / 1e3) / 1e9
+    # e2e through the C ABI with a pinned host buffer
+    hx = x.cpu().pin_memory()
+    times = []
+    for i in range(args.warmup + args.steps):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        plan.max_subarray_host(hx)
+        if i >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    e2e_ms = statistics.mean(times) * 1e3
+    cpu = None
+    if not args.no_cpu_baseline:
+        v, reps, sn, el = oracle_maxsub_sample(n, "uniform")
+        model, cores = cpu_info()
+        cpu = {"value": v, "unit": "elements/s", "cores": 1, "kind": "oracle",
+               "sample": f"oracle recursive D&C max-subarray, 1 thread, {reps} x the full input "
+                         f"({el:.1f} s)", "cpu": model, "host_cores": cores}
+    print(json.dumps({
+        "metric": "max-subarray elements/sec (2^24 int32)", "value": n / (ms / 1e3),
+        "unit": "elements/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "i32->i64", "data": "synthetic (counter-based splitmix64)",
+        "config": {"workload": wl, "description": desc, "n": n, "dist": args.dist,
+                   "l2": "flushed before every step (512 MiB write)"},
+        "roofline": {"kernel": "nk4_maxsub (tiles + last-CTA top combine)", "bound": "hbm",
+                     "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                     "traffic": ncu_traffic("nk4_maxsub", wl), "avg_launch_ms": avg,
+                     "algorithmic_bytes_per_launch": 4 * n, "peak_source": src},
+        "gpu_launches": launches, "clocks": clk.summary(),
+        "e2e": {"value": n / (e2e_ms / 1e3), "unit": "elements/s", "ms_per_step": e2e_ms,
+                "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 24},
+        "cpu_baseline": cpu,
+    }), flush=True)
+
+
+def main():
+    args = parse()
+    wl = args.workload or ("sort_u32" if args.gpus == 1 else "sort_u32_2p30")
+    if args.impl == "reference":
+        return run_reference(args, wl)
+    return run_dc(args, wl)
+
+
+if __name__ == "__main__":
+    main()

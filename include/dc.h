@@ -1,0 +1,186 @@
+/*
+ * dc.h -- C ABI of the B200-native breadth-first divide-and-conquer library.
+ *
+ * The operation: the breadth-first, level-by-level execution of a recursive
+ * divide-and-conquer T(n) = aT(n/b) + f(n) (Sec. 4, P:L229-306;
+ * Alg 2): all a^i subproblems of size n/b^i at level i run in one
+ * data-parallel step, base cases first, then one combine pass per level,
+ * bottom-up.  Two instances:
+ *   - mergesort, a = b = 2, linear stable merge combine (Alg 6 P:L623-630,
+ *     Alg 7);
+ *   - maximum-subarray-sum with an O(1) combine (north star; the O(1)-combine
+ *     pattern of Alg 4/5).
+ * "P:Lx-y" = lines of PAPER.md (the paper text).
+ *
+ * Conventions (all entry points)
+ *   - No exception crosses the ABI; every call returns a dc_status.
+ *   - Validation failures return before any device work; inputs untouched.
+ *   - Device pointers are plain CUDA device pointers on the device that was
+ *     current when the plan first ran (the "plan device"); 4-byte elements,
+ *     16-byte aligned (misalignment -> DC_ERR_INVALID_ARG).  Host pointers
+ *     are ordinary host memory (pinned or pageable).
+ *   - Ownership: the caller owns every buffer passed in.  The plan owns its
+ *     scratch (allocated lazily on first run unless dc_plan_set_scratch gave
+ *     one), its partition arrays and its CUDA graphs; dc_free releases them.
+ *   - Asynchrony: dc_run_mergesort and the *_async calls only enqueue work on
+ *     the plan stream (default: the legacy default stream) and return.  Calls
+ *     that return a result through a host pointer synchronise the stream.
+ *     An asynchronous CUDA fault surfaces as DC_ERR_CUDA on a later call; the
+ *     plan is then in DC_ERR_BAD_STATE and must be freed.
+ *   - A plan is used by one host thread at a time.
+ *   - dc_last_error() returns a thread-local human-readable detail string for
+ *     the last non-OK status returned on this thread.
+ */
+#ifndef DC_H
+#define DC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    DC_OK = 0,
+    DC_ERR_INVALID_ARG = 1,   /* bad size, NULL, misaligned pointer, ...     */
+    DC_ERR_UNSUPPORTED = 2,   /* valid request this build cannot run (a!=2) */
+    DC_ERR_OUT_OF_MEMORY = 3, /* scratch allocation failed                    */
+    DC_ERR_CUDA = 4,          /* a CUDA runtime call or kernel failed        */
+    DC_ERR_NCCL = 5,          /* reserved: collectives run in torch.distributed */
+    DC_ERR_BAD_STATE = 6      /* plan poisoned by an earlier CUDA error       */
+} dc_status;
+
+typedef enum {
+    DC_KEY_U32 = 0, /* uint32 keys                                           */
+    DC_KEY_I32 = 1, /* int32 keys                                            */
+    DC_KEY_F32 = 2  /* float32 keys compared with '<' only: +0.0 == -0.0 keep
+                       input order; NaN is a precondition violation.         */
+} dc_key_type;
+
+typedef struct dc_plan_s *dc_plan_t; /* opaque */
+
+/* Result of the max-subarray instance: the non-empty subarray x[start..end]
+ * (inclusive, 0-based, global indices) of maximum int64 sum; among several
+ * maxima the lexicographically smallest (start, end) (R9-R10). */
+typedef struct {
+    int64_t sum;
+    int64_t start;
+    int64_t end;
+} dc_maxsub_result;
+
+/* The O(1)-combine summary of a contiguous segment [l, r]:
+ * tot = sum; pre = max prefix sum (ends at pe, smallest end on ties);
+ * suf = max suffix sum (starts at ss, smallest start); best = max subarray
+ * (bs..be, lexicographically smallest).  Indices are global.  Used to combine
+ * per-rank results of a sharded max-subarray in rank order. */
+typedef struct {
+    int64_t tot, pre, suf, best;
+    int64_t pe, ss, bs, be;
+} dc_maxsub_tuple;
+
+/* ------------------------------------------------------------------ plans */
+
+/* dc_plan: describe the recursion T(n) = aT(n/b) + f(n) for an input
+ * of n elements whose recursion stops at subproblems of size <= base_size.
+ * Host-only (no device work).  n >= 1, 2 <= a,b <= 1024, 1 <= base_size <= n,
+ * n <= 2^31-1.  Runs need a == b == 2 (mergesort and max-subarray);
+ * other (a, b) only serve level-table queries (DC_ERR_UNSUPPORTED at run).
+ * base_size changes only the level table, never a result. */
+dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t *out);
+
+/* Level table of the plan: level i (0 = root) has nodes[i] = a^i
+ * subproblems of size sizes[i] = ceil(n / b^i); the last level L is the first
+ * whose size is <= base_size.  Writes *num_levels = L + 1 and, if the arrays
+ * are non-NULL, min(L+1, capacity) entries of each. */
+dc_status dc_plan_levels(dc_plan_t plan, int32_t *num_levels, int64_t *nodes,
+                         int64_t *sizes, int32_t capacity);
+
+/* Execution schedule of the a=b=2 runs: the fused bottom kernel sorts tiles
+ * of `tile` keys (the leaves plus fused_levels = log2(tile) combine levels,
+ * entirely on chip), then global_passes = ceil(log2(ceil(n/tile))) merge
+ * passes each combine one level of the tree over HBM. */
+dc_status dc_plan_schedule(dc_plan_t plan, int32_t *tile, int32_t *fused_levels,
+                           int32_t *global_passes);
+
+/* Stream all device work of this plan is enqueued on (a cudaStream_t). */
+dc_status dc_plan_set_stream(dc_plan_t plan, void *cuda_stream);
+
+/* Scratch the sort needs: n*4 bytes for keys (+ n*4 for values) ping-pong
+ * (the paper's 2n working space) plus the partition array. */
+dc_status dc_plan_scratch_bytes(dc_plan_t plan, int32_t with_vals, size_t *bytes);
+
+/* Optional caller-owned scratch (device, 16-byte aligned, >= the size above).
+ * Without it the plan allocates its own on first use. */
+dc_status dc_plan_set_scratch(dc_plan_t plan, void *d_scratch, size_t bytes);
+
+/* Frees the plan and everything it owns.  Accepts NULL. */
+dc_status dc_free(dc_plan_t plan);
+
+/* ------------------------------------------------------------- mergesort */
+
+/* In-place stable sort of d_keys[0..n) (device), permuting d_vals[0..n)
+ * (device, nullable) with the keys.  Alg 7 executed bottom-up: fused bottom
+ * levels, then one merge-path pass per remaining level.  Enqueues only. */
+dc_status dc_run_mergesort(dc_plan_t plan, dc_key_type key_type, void *d_keys,
+                           uint32_t *d_vals);
+
+/* Same, host buffers: copies h_keys (+h_vals) to device memory owned by the
+ * plan, sorts, copies back, synchronises.  End-to-end entry point. */
+dc_status dc_run_mergesort_host(dc_plan_t plan, dc_key_type key_type, void *h_keys,
+                                uint32_t *h_vals);
+
+/* ----------------------------------------------------------- max-subarray */
+
+/* Max subarray of d_x[0..n) (device int32).  Synchronises; writes *h_out. */
+dc_status dc_run_maxsubarray(dc_plan_t plan, const int32_t *d_x, dc_maxsub_result *h_out);
+
+/* Enqueue-only variant: writes the result (dc_maxsub_result, device memory)
+ * to d_out; index_offset is added to every index (a shard's global start). */
+dc_status dc_run_maxsubarray_async(dc_plan_t plan, const int32_t *d_x, int64_t index_offset,
+                                   dc_maxsub_result *d_out);
+
+/* Enqueue-only: the segment summary tuple of d_x[0..n) with indices offset by
+ * index_offset, written to d_tuple (device). */
+dc_status dc_run_maxsubarray_tuple_async(dc_plan_t plan, const int32_t *d_x,
+                                         int64_t index_offset, dc_maxsub_tuple *d_tuple);
+
+/* Enqueue-only: ordered combine of count tuples (device; tuple r covers the
+ * segment left of tuple r+1) into one result (device). */
+dc_status dc_maxsub_combine_async(dc_plan_t plan, const dc_maxsub_tuple *d_tuples,
+                                  int32_t count, dc_maxsub_result *d_out);
+
+/* Host buffers end to end: copy h_x to the device, run, return the result. */
+dc_status dc_run_maxsubarray_host(dc_plan_t plan, const int32_t *h_x, dc_maxsub_result *h_out);
+
+/* ------------------------------------------------------ instrumentation */
+
+/* Kernel classes for dc_plan_kernel_time. */
+#define DC_KERNEL_NK1_BLOCKSORT 0 /* fused bottom levels              */
+#define DC_KERNEL_NK2_PARTITION 1 /* merge-path co-ranks of one level */
+#define DC_KERNEL_NK3_MERGE 2     /* one global merge level           */
+#define DC_KERNEL_NK4_MAXSUB 3    /* max-subarray tiles + top combine */
+#define DC_KERNEL_COUNT 4
+
+/* Turn per-launch CUDA-event timing on (1) or off (0); resets the totals.
+ * When on, every kernel launch is bracketed by two events on the plan stream. */
+dc_status dc_plan_enable_timing(dc_plan_t plan, int32_t enable);
+
+/* Total device time (ms) and number of timed launches of one kernel class
+ * since timing was enabled.  Waits for the pending events. */
+dc_status dc_plan_kernel_time(dc_plan_t plan, int32_t kernel, double *total_ms,
+                              int64_t *launches);
+
+/* ------------------------------------------------------------- misc */
+
+const char *dc_status_string(dc_status s);
+const char *dc_last_error(void);
+/* Number of kernels this plan launched since creation (instrumentation). */
+int64_t dc_plan_launch_count(dc_plan_t plan);
+/* Library version string. */
+const char *dc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DC_H */

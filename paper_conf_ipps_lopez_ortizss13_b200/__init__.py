@@ -1,0 +1,276 @@
+"""B200-native breadth-first divide-and-conquer (Lopez-Ortiz, Salinger, Suderman).
+
+Thin Python binding over the C ABI in ``include/dc.h`` (``libdcb200.so``,
+built by :mod:`.build`).  This module only marshals arguments: every step of
+the hot path runs in the library's sm_100a kernels.  There is no CPU fallback:
+if the library is missing or no CUDA device is present, calls raise.
+
+    import paper_conf_ipps_lopez_ortizss13_b200 as dc
+    dc.sort_(keys, vals=None)            # in-place stable sort on the GPU
+    dc.max_subarray(x) -> (sum, start, end)
+    dc.Plan(n)                            # explicit plan: level table, schedule, runs
+
+Multi-GPU (one process per GPU, torch.distributed/NCCL): see :mod:`.dist`.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+from . import build as _build
+
+__all__ = [
+    "DcError", "Plan", "sort_", "max_subarray", "lib", "KEY_U32", "KEY_I32", "KEY_F32",
+    "MaxsubResult", "MaxsubTuple",
+]
+
+KEY_U32, KEY_I32, KEY_F32 = 0, 1, 2
+_KEY_NAMES = {"u32": KEY_U32, "i32": KEY_I32, "f32": KEY_F32}
+_STATUS = {0: "DC_OK", 1: "DC_ERR_INVALID_ARG", 2: "DC_ERR_UNSUPPORTED",
+           3: "DC_ERR_OUT_OF_MEMORY", 4: "DC_ERR_CUDA", 5: "DC_ERR_NCCL",
+           6: "DC_ERR_BAD_STATE"}
+
+
+class DcError(RuntimeError):
+    def __init__(self, status: int, detail: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {detail}")
+        self.status = status
+
+
+class MaxsubResult(ctypes.Structure):
+    _fields_ = [("sum", ctypes.c_int64), ("start", ctypes.c_int64), ("end", ctypes.c_int64)]
+
+
+class MaxsubTuple(ctypes.Structure):
+    _fields_ = [(f, ctypes.c_int64) for f in ("tot", "pre", "suf", "best", "pe", "ss", "bs", "be")]
+
+
+_lib = None
+_P = ctypes.c_void_p
+_I64 = ctypes.c_int64
+_I32 = ctypes.c_int32
+_SIGS = {
+    "dc_plan": ([_I64, _I32, _I32, _I64, ctypes.POINTER(_P)], ctypes.c_int),
+    "dc_plan_levels": ([_P, ctypes.POINTER(_I32), _P, _P, _I32], ctypes.c_int),
+    "dc_plan_schedule": ([_P, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
+                          ctypes.POINTER(_I32)], ctypes.c_int),
+    "dc_plan_set_stream": ([_P, _P], ctypes.c_int),
+    "dc_plan_scratch_bytes": ([_P, _I32, ctypes.POINTER(ctypes.c_size_t)], ctypes.c_int),
+    "dc_plan_set_scratch": ([_P, _P, ctypes.c_size_t], ctypes.c_int),
+    "dc_free": ([_P], ctypes.c_int),
+    "dc_run_mergesort": ([_P, ctypes.c_int, _P, _P], ctypes.c_int),
+    "dc_run_mergesort_host": ([_P, ctypes.c_int, _P, _P], ctypes.c_int),
+    "dc_run_maxsubarray": ([_P, _P, ctypes.POINTER(MaxsubResult)], ctypes.c_int),
+    "dc_run_maxsubarray_async": ([_P, _P, _I64, _P], ctypes.c_int),
+    "dc_run_maxsubarray_tuple_async": ([_P, _P, _I64, _P], ctypes.c_int),
+    "dc_maxsub_combine_async": ([_P, _P, _I32, _P], ctypes.c_int),
+    "dc_run_maxsubarray_host": ([_P, _P, ctypes.POINTER(MaxsubResult)], ctypes.c_int),
+    "dc_status_string": ([ctypes.c_int], ctypes.c_char_p),
+    "dc_last_error": ([], ctypes.c_char_p),
+    "dc_plan_launch_count": ([_P], _I64),
+    "dc_version": ([], ctypes.c_char_p),
+    "dc_plan_enable_timing": ([_P, _I32], ctypes.c_int),
+    "dc_plan_kernel_time": ([_P, _I32, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_I64)],
+                            ctypes.c_int),
+}
+
+#: kernel classes of dc_plan_kernel_time
+KERNELS = {"nk1_blocksort": 0, "nk2_partition": 1, "nk3_merge": 2, "nk4_maxsub": 3}
+
+
+def lib() -> ctypes.CDLL:
+    """Load (building first if stale and nvcc is available) libdcb200.so."""
+    global _lib
+    if _lib is None:
+        path = _build.LIB
+        try:
+            path = _build.build()
+        except (OSError, FileNotFoundError):
+            if not os.path.exists(path):
+                raise
+        handle = ctypes.CDLL(path)
+        for name, (args, res) in _SIGS.items():
+            fn = getattr(handle, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = handle
+    return _lib
+
+
+def _check(status: int) -> None:
+    if status != 0:
+        raise DcError(status, lib().dc_last_error().decode())
+
+
+def _key_type(t: torch.Tensor, key_type: str | None) -> int:
+    if key_type is not None:
+        return _KEY_NAMES[key_type]
+    if t.dtype == torch.uint32:
+        return KEY_U32
+    if t.dtype == torch.int32:
+        return KEY_I32
+    if t.dtype == torch.float32:
+        return KEY_F32
+    raise TypeError(f"unsupported key dtype {t.dtype}")
+
+
+def _require_cuda(t: torch.Tensor, what: str) -> None:
+    if not t.is_cuda:
+        raise ValueError(f"{what} must be a CUDA tensor (no CPU fallback)")
+    if not t.is_contiguous():
+        raise ValueError(f"{what} must be contiguous")
+    if t.element_size() != 4:
+        raise ValueError(f"{what} must have 4-byte elements")
+
+
+class Plan:
+    """A ``dc_plan`` handle: T(n) = aT(n/b) + f(n) recursion for n elements."""
+
+    def __init__(self, n: int, a: int = 2, b: int = 2, base_size: int = 1):
+        h = _P()
+        _check(lib().dc_plan(n, a, b, base_size, ctypes.byref(h)))
+        self._h = h
+        self.n, self.a, self.b, self.base_size = n, a, b, base_size
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and _lib is not None:
+            _lib.dc_free(h)
+            self._h = None
+
+    def levels(self) -> list[tuple[int, int]]:
+        """[(nodes a^i, size ceil(n/b^i)) for each level i]."""
+        cnt = _I32()
+        _check(lib().dc_plan_levels(self._h, ctypes.byref(cnt), None, None, 0))
+        nodes = (_I64 * cnt.value)()
+        sizes = (_I64 * cnt.value)()
+        _check(lib().dc_plan_levels(self._h, ctypes.byref(cnt), nodes, sizes, cnt.value))
+        return list(zip(nodes, sizes))
+
+    def schedule(self) -> dict:
+        t, f, p = _I32(), _I32(), _I32()
+        _check(lib().dc_plan_schedule(self._h, ctypes.byref(t), ctypes.byref(f), ctypes.byref(p)))
+        return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value}
+
+    def scratch_bytes(self, with_vals: bool = False) -> int:
+        b = ctypes.c_size_t()
+        _check(lib().dc_plan_scratch_bytes(self._h, int(with_vals), ctypes.byref(b)))
+        return b.value
+
+    def set_scratch(self, buf: torch.Tensor) -> None:
+        _check(lib().dc_plan_set_scratch(self._h, buf.data_ptr(), buf.numel() * buf.element_size()))
+        self._scratch_ref = buf
+
+    def launch_count(self) -> int:
+        return int(lib().dc_plan_launch_count(self._h))
+
+    def enable_timing(self, on: bool = True) -> None:
+        """Bracket every launch with CUDA events on the plan stream (resets totals)."""
+        _check(lib().dc_plan_enable_timing(self._h, int(on)))
+
+    def kernel_times(self) -> dict:
+        """{kernel: (total_ms, launches)} since enable_timing (waits for the events)."""
+        out = {}
+        for name, k in KERNELS.items():
+            ms, cnt = ctypes.c_double(), _I64()
+            _check(lib().dc_plan_kernel_time(self._h, k, ctypes.byref(ms), ctypes.byref(cnt)))
+            out[name] = (ms.value, cnt.value)
+        return out
+
+    def _bind_stream(self, t: torch.Tensor) -> None:
+        _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream(t.device).cuda_stream))
+
+    def sort_(self, keys: torch.Tensor, vals: torch.Tensor | None = None,
+              key_type: str | None = None) -> torch.Tensor:
+        """In-place stable sort of keys (and vals alongside) on the GPU."""
+        _require_cuda(keys, "keys")
+        if keys.numel() != self.n:
+            raise ValueError("keys length != plan n")
+        if vals is not None:
+            _require_cuda(vals, "vals")
+            if vals.numel() != self.n:
+                raise ValueError("vals length != plan n")
+        kt = _key_type(keys, key_type)
+        self._bind_stream(keys)
+        _check(lib().dc_run_mergesort(self._h, kt, keys.data_ptr(),
+                                      None if vals is None else vals.data_ptr()))
+        return keys
+
+    def sort_host_(self, keys: torch.Tensor, vals: torch.Tensor | None = None,
+                   key_type: str | None = None) -> torch.Tensor:
+        """End-to-end sort of HOST tensors (pinned for full speed): H2D, sort, D2H."""
+        if keys.is_cuda or (vals is not None and vals.is_cuda):
+            raise ValueError("sort_host_ takes host tensors")
+        kt = _key_type(keys, key_type)
+        _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
+        _check(lib().dc_run_mergesort_host(self._h, kt, keys.data_ptr(),
+                                           None if vals is None else vals.data_ptr()))
+        return keys
+
+    def max_subarray(self, x: torch.Tensor) -> tuple[int, int, int]:
+        _require_cuda(x, "x")
+        if x.numel() != self.n:
+            raise ValueError("x length != plan n")
+        self._bind_stream(x)
+        r = MaxsubResult()
+        _check(lib().dc_run_maxsubarray(self._h, x.data_ptr(), ctypes.byref(r)))
+        return (r.sum, r.start, r.end)
+
+    def max_subarray_async(self, x: torch.Tensor, out: torch.Tensor, index_offset: int = 0):
+        """Enqueue only; ``out`` is a CUDA int64 tensor of 3 elements (sum, start, end)."""
+        _require_cuda(x, "x")
+        self._bind_stream(x)
+        _check(lib().dc_run_maxsubarray_async(self._h, x.data_ptr(), index_offset, out.data_ptr()))
+        return out
+
+    def max_subarray_tuple_async(self, x: torch.Tensor, out: torch.Tensor, index_offset: int = 0):
+        """Enqueue only; ``out`` is a CUDA int64 tensor of 8 elements (segment summary)."""
+        _require_cuda(x, "x")
+        self._bind_stream(x)
+        _check(lib().dc_run_maxsubarray_tuple_async(self._h, x.data_ptr(), index_offset,
+                                                    out.data_ptr()))
+        return out
+
+    def maxsub_combine_async(self, tuples: torch.Tensor, out: torch.Tensor):
+        """Ordered combine of a (count, 8) int64 CUDA tensor of summaries into out[3]."""
+        self._bind_stream(tuples)
+        _check(lib().dc_maxsub_combine_async(self._h, tuples.data_ptr(), tuples.shape[0],
+                                             out.data_ptr()))
+        return out
+
+    def max_subarray_host(self, x: torch.Tensor) -> tuple[int, int, int]:
+        """End-to-end max subarray of a HOST int32 tensor."""
+        if x.is_cuda:
+            raise ValueError("max_subarray_host takes a host tensor")
+        _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
+        r = MaxsubResult()
+        _check(lib().dc_run_maxsubarray_host(self._h, x.data_ptr(), ctypes.byref(r)))
+        return (r.sum, r.start, r.end)
+
+
+_plans: dict = {}
+
+
+def _plan_for(n: int, device) -> Plan:
+    key = (n, str(device))
+    p = _plans.get(key)
+    if p is None:
+        p = _plans[key] = Plan(n)
+    return p
+
+
+def sort_(keys: torch.Tensor, vals: torch.Tensor | None = None,
+          key_type: str | None = None) -> torch.Tensor:
+    """In-place stable GPU mergesort of ``keys`` (uint32/int32/float32 CUDA tensor).
+
+    ``key_type`` overrides the dtype-derived key type ("u32", "i32", "f32"),
+    e.g. to sort int32-stored bit patterns as unsigned.
+    """
+    return _plan_for(keys.numel(), keys.device).sort_(keys, vals, key_type)
+
+
+def max_subarray(x: torch.Tensor) -> tuple[int, int, int]:
+    """(sum, start, end) of the maximum non-empty subarray of an int32 CUDA tensor."""
+    return _plan_for(x.numel(), x.device).max_subarray(x)

@@ -1,0 +1,544 @@
+// dc_api.cu -- the C ABI (include/dc.h): plans, the level driver and launches.
+//
+// Layer a0 (plan): the level table of T(n) = aT(n/b) + f(n) (P:L236,
+// P:L425-439) and the execution schedule (fused bottom levels + global merge
+// passes).  Layer a4 (level driver): Alg 7's recursion unrolled bottom-up
+// (Alg 2): NK1 once, then for every remaining level NK2 + NK3 with
+// src/dst ping-pong over the paper's 2n working space, the
+// parity chosen so that the last pass lands in the caller's buffer.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "dc.h"
+#include "maxsub_kernels.cuh"
+#include "sort_kernels.cuh"
+
+namespace {
+
+// ---------------------------------------------------------------- config
+constexpr int kNK1Threads = 512;
+constexpr int kNK1Items = 16;
+constexpr int kTile = kNK1Threads * kNK1Items;     // 8192 keys, 13 fused levels
+constexpr int kNK3Threads = 256;
+constexpr int kNK3Items = 16;
+constexpr int kTout = kNK3Threads * kNK3Items;      // 4096 outputs per merge CTA
+static_assert((2 * kTile) % kTout == 0, "merge tiles must not straddle pairs");
+constexpr int kNK4Threads = 256;
+constexpr int kNK4Chunk = 32;
+constexpr int kMsTile = kNK4Threads * kNK4Chunk;   // 8192 values per CTA
+
+constexpr int64_t kMaxN = 2147483647LL;
+
+thread_local std::string g_last_error;
+
+dc_status fail(dc_status s, const std::string& msg) {
+    g_last_error = msg;
+    return s;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+int nk1_smem_bytes(bool vals) {
+    const int padded = kTile + kTile / 32 + 1;
+    return (vals ? 2 * padded + kTile : padded) * 4;
+}
+int nk3_smem_bytes(bool vals) {
+    const int padded = kTout + kTout / 32 + 1;
+    return (vals ? 2 * padded : padded) * 4;
+}
+
+}  // namespace
+
+struct dc_plan_s {
+    int64_t n = 0;
+    int32_t a = 2, b = 2;
+    int64_t base_size = 1;
+    std::vector<int64_t> nodes, sizes;
+    cudaStream_t stream = nullptr;
+    bool bad = false;
+    int64_t launches = 0;
+    // scratch (keys ping-pong, values ping-pong, partition array)
+    void* scratch = nullptr;
+    size_t scratch_bytes = 0;
+    bool own_scratch = false;
+    // max-subarray state
+    dc_maxsub_tuple* ms_tiles = nullptr;
+    unsigned int* ms_ticket = nullptr;
+    dc_maxsub_result* ms_res = nullptr;
+    // host-buffer (end-to-end) staging
+    void* d_stage = nullptr;
+    size_t d_stage_bytes = 0;
+    // per-kernel CUDA-event timing (instrumentation, off by default)
+    bool timing = false;
+    struct Timed { int kind; cudaEvent_t e0, e1; };
+    std::vector<Timed> pending;
+    std::vector<cudaEvent_t> event_pool;
+    double acc_ms[DC_KERNEL_COUNT] = {0};
+    int64_t acc_n[DC_KERNEL_COUNT] = {0};
+};
+
+namespace {
+
+int64_t num_tiles(int64_t n, int64_t t) { return (n + t - 1) / t; }
+
+int global_passes(int64_t n) {
+    int p = 0;
+    for (int64_t w = kTile; w < n; w *= 2) ++p;
+    return p;
+}
+
+size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kTout) + 1; }
+
+size_t scratch_needed(int64_t n, bool vals) {
+    size_t kb = align_up((size_t)n * 4, 256);
+    return kb + (vals ? kb : 0) + align_up(split_entries(n) * 4, 256);
+}
+
+dc_status check_plan(dc_plan_t p) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (p->bad) return fail(DC_ERR_BAD_STATE, "plan poisoned by an earlier CUDA error");
+    return DC_OK;
+}
+
+dc_status cuda_fail(dc_plan_t p, cudaError_t e, const char* what) {
+    if (p) p->bad = true;
+    return fail(DC_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define DC_CUDA(p, call)                                          \
+    do {                                                          \
+        cudaError_t e_ = (call);                                  \
+        if (e_ != cudaSuccess) return cuda_fail((p), e_, #call);  \
+    } while (0)
+
+#define DC_LAUNCHED(p)                                                     \
+    do {                                                                   \
+        cudaError_t e_ = cudaGetLastError();                               \
+        if (e_ != cudaSuccess) return cuda_fail((p), e_, "kernel launch"); \
+        (p)->launches++;                                                   \
+    } while (0)
+
+cudaEvent_t take_event(dc_plan_t p) {
+    if (!p->event_pool.empty()) {
+        cudaEvent_t e = p->event_pool.back();
+        p->event_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+
+// Brackets one kernel launch with events on the plan stream when timing is on.
+struct TimedScope {
+    dc_plan_t p;
+    int kind;
+    cudaEvent_t e0 = nullptr;
+    TimedScope(dc_plan_t p_, int kind_) : p(p_), kind(kind_) {
+        if (p->timing) {
+            e0 = take_event(p);
+            cudaEventRecord(e0, p->stream);
+        }
+    }
+    ~TimedScope() {
+        if (e0) {
+            cudaEvent_t e1 = take_event(p);
+            cudaEventRecord(e1, p->stream);
+            p->pending.push_back({kind, e0, e1});
+        }
+    }
+};
+
+bool aligned16(const void* ptr) { return ((uintptr_t)ptr & 15u) == 0; }
+
+dc_status ensure_scratch(dc_plan_t p, bool vals) {
+    size_t need = scratch_needed(p->n, vals);
+    if (p->scratch && p->scratch_bytes >= need) return DC_OK;
+    if (p->scratch && !p->own_scratch)
+        return fail(DC_ERR_INVALID_ARG, "caller scratch too small for this run");
+    if (p->scratch) {
+        cudaFree(p->scratch);
+        p->scratch = nullptr;
+    }
+    void* ptr = nullptr;
+    cudaError_t e = cudaMalloc(&ptr, need);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DC_ERR_OUT_OF_MEMORY, "scratch cudaMalloc failed");
+    }
+    p->scratch = ptr;
+    p->scratch_bytes = need;
+    p->own_scratch = true;
+    return DC_OK;
+}
+
+template <class K, bool V>
+dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
+    const int64_t n = p->n;
+    const bool hv = V;
+    dc_status st = ensure_scratch(p, hv);
+    if (st != DC_OK) return st;
+    size_t kb = align_up((size_t)n * 4, 256);
+    uint32_t* sk = (uint32_t*)p->scratch;
+    uint32_t* sv = hv ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
+    int* split = (int*)((char*)p->scratch + kb + (hv ? kb : 0));
+
+    static bool attr_done = false;   // per key/value instantiation
+    if (!attr_done) {
+        DC_CUDA(p, cudaFuncSetAttribute(dc::nk1_blocksort<kNK1Threads, kNK1Items, K, V>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        nk1_smem_bytes(hv)));
+        DC_CUDA(p, cudaFuncSetAttribute(dc::nk3_merge<kNK3Threads, kNK3Items, K, V>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        nk3_smem_bytes(hv)));
+        attr_done = true;
+    }
+
+    const int P = global_passes(n);
+    // Ping-pong parity: pass P-1 must write the caller's buffer, so NK1
+    // writes the caller's buffer iff P is even.
+    uint32_t* cur_k = (P % 2 == 0) ? keys : sk;
+    uint32_t* cur_v = (P % 2 == 0) ? vals : sv;
+    uint32_t* oth_k = (P % 2 == 0) ? sk : keys;
+    uint32_t* oth_v = (P % 2 == 0) ? sv : vals;
+
+    // NK1: base cases + fused bottom levels (reads the caller's buffer).
+    {
+    TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT);
+    dc::nk1_blocksort<kNK1Threads, kNK1Items, K, V>
+        <<<(unsigned)num_tiles(n, kTile), kNK1Threads, nk1_smem_bytes(hv), p->stream>>>(
+            keys, vals, cur_k, cur_v, n);
+    DC_LAUNCHED(p);
+    }
+
+    const int tiles = (int)num_tiles(n, kTout);
+    for (int64_t w = kTile; w < n; w *= 2) {
+        {
+        TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
+        dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(cur_k, n, w, kTout,
+                                                                        tiles, split);
+        DC_LAUNCHED(p);
+        }
+        {
+        TimedScope ts(p, DC_KERNEL_NK3_MERGE);
+        dc::nk3_merge<kNK3Threads, kNK3Items, K, V>
+            <<<tiles, kNK3Threads, nk3_smem_bytes(hv), p->stream>>>(cur_k, cur_v, oth_k, oth_v,
+                                                                    split, n, w);
+        DC_LAUNCHED(p);
+        }
+        std::swap(cur_k, oth_k);
+        std::swap(cur_v, oth_v);
+    }
+    return DC_OK;
+}
+
+dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
+    const bool v = vals != nullptr;
+    switch (kt) {
+        case DC_KEY_U32:
+            return v ? sort_typed<dc::KeyU32, true>(p, keys, vals)
+                     : sort_typed<dc::KeyU32, false>(p, keys, nullptr);
+        case DC_KEY_I32:
+            return v ? sort_typed<dc::KeyI32, true>(p, keys, vals)
+                     : sort_typed<dc::KeyI32, false>(p, keys, nullptr);
+        case DC_KEY_F32:
+            return v ? sort_typed<dc::KeyF32, true>(p, keys, vals)
+                     : sort_typed<dc::KeyF32, false>(p, keys, nullptr);
+    }
+    return fail(DC_ERR_INVALID_ARG, "unknown key type");
+}
+
+dc_status ensure_ms_state(dc_plan_t p) {
+    if (p->ms_tiles) return DC_OK;
+    size_t tiles = (size_t)num_tiles(p->n, kMsTile);
+    void* ptr = nullptr;
+    size_t bytes = align_up(tiles * sizeof(dc_maxsub_tuple), 256) + 256 + 256;
+    if (cudaMalloc(&ptr, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DC_ERR_OUT_OF_MEMORY, "max-subarray state cudaMalloc failed");
+    }
+    DC_CUDA(p, cudaMemsetAsync(ptr, 0, bytes, p->stream));
+    p->ms_tiles = (dc_maxsub_tuple*)ptr;
+    p->ms_ticket = (unsigned int*)((char*)ptr + align_up(tiles * sizeof(dc_maxsub_tuple), 256));
+    p->ms_res = (dc_maxsub_result*)((char*)p->ms_ticket + 256);
+    return DC_OK;
+}
+
+dc_status maxsub_launch(dc_plan_t p, const int32_t* d_x, int64_t off, int mode,
+                        dc_maxsub_result* out_res, dc_maxsub_tuple* out_tup) {
+    dc_status st = ensure_ms_state(p);
+    if (st != DC_OK) return st;
+    const int64_t tiles = num_tiles(p->n, kMsTile);
+    TimedScope ts(p, DC_KERNEL_NK4_MAXSUB);
+    dc::nk4_maxsub<kNK4Threads, kNK4Chunk><<<(unsigned)tiles, kNK4Threads, 0, p->stream>>>(
+        d_x, p->n, p->ms_tiles, p->ms_ticket, off, mode, out_res, out_tup);
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+dc_status ensure_stage(dc_plan_t p, size_t bytes) {
+    if (p->d_stage && p->d_stage_bytes >= bytes) return DC_OK;
+    if (p->d_stage) cudaFree(p->d_stage);
+    p->d_stage = nullptr;
+    if (cudaMalloc(&p->d_stage, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        p->d_stage = nullptr;
+        return fail(DC_ERR_OUT_OF_MEMORY, "staging cudaMalloc failed");
+    }
+    p->d_stage_bytes = bytes;
+    return DC_OK;
+}
+
+}  // namespace
+
+// =================================================================== ABI
+
+extern "C" {
+
+const char* dc_version(void) { return "dc-b200 0.1 (sm_100a)"; }
+
+const char* dc_status_string(dc_status s) {
+    switch (s) {
+        case DC_OK: return "DC_OK";
+        case DC_ERR_INVALID_ARG: return "DC_ERR_INVALID_ARG";
+        case DC_ERR_UNSUPPORTED: return "DC_ERR_UNSUPPORTED";
+        case DC_ERR_OUT_OF_MEMORY: return "DC_ERR_OUT_OF_MEMORY";
+        case DC_ERR_CUDA: return "DC_ERR_CUDA";
+        case DC_ERR_NCCL: return "DC_ERR_NCCL";
+        case DC_ERR_BAD_STATE: return "DC_ERR_BAD_STATE";
+    }
+    return "DC_ERR_UNKNOWN";
+}
+
+const char* dc_last_error(void) { return g_last_error.c_str(); }
+
+dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t* out) {
+    if (!out) return fail(DC_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (n < 1 || n > kMaxN) return fail(DC_ERR_INVALID_ARG, "n must be in [1, 2^31-1]");
+    if (a < 2 || b < 2 || a > 1024 || b > 1024)
+        return fail(DC_ERR_INVALID_ARG, "a and b must be in [2, 1024]");
+    if (base_size < 1 || base_size > n)
+        return fail(DC_ERR_INVALID_ARG, "base_size must be in [1, n]");
+    dc_plan_s* p = new (std::nothrow) dc_plan_s();
+    if (!p) return fail(DC_ERR_OUT_OF_MEMORY, "plan allocation failed");
+    p->n = n;
+    p->a = a;
+    p->b = b;
+    p->base_size = base_size;
+    // Level i: a^i nodes of size ceil(n / b^i); stop at the first level whose
+    // size is <= base_size (leaves at level log_b n for base 1).
+    int64_t nodes = 1, size = n, bpow = 1;
+    for (;;) {
+        p->nodes.push_back(nodes);
+        p->sizes.push_back(size);
+        if (size <= base_size) break;
+        if (nodes > INT64_MAX / a) {
+            delete p;
+            return fail(DC_ERR_INVALID_ARG, "a^L overflows int64");
+        }
+        nodes *= a;
+        bpow = (bpow > INT64_MAX / b) ? INT64_MAX : bpow * b;
+        size = (n + bpow - 1) / bpow;
+    }
+    *out = p;
+    return DC_OK;
+}
+
+dc_status dc_plan_levels(dc_plan_t p, int32_t* num_levels, int64_t* nodes, int64_t* sizes,
+                         int32_t capacity) {
+    if (!p || !num_levels) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    *num_levels = (int32_t)p->nodes.size();
+    int32_t m = capacity < *num_levels ? capacity : *num_levels;
+    for (int32_t i = 0; i < m; ++i) {
+        if (nodes) nodes[i] = p->nodes[i];
+        if (sizes) sizes[i] = p->sizes[i];
+    }
+    return DC_OK;
+}
+
+dc_status dc_plan_schedule(dc_plan_t p, int32_t* tile, int32_t* fused_levels,
+                           int32_t* passes) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (tile) *tile = kTile;
+    int f = 0;
+    while ((1 << f) < kTile) ++f;
+    if (fused_levels) *fused_levels = f;
+    if (passes) *passes = global_passes(p->n);
+    return DC_OK;
+}
+
+dc_status dc_plan_set_stream(dc_plan_t p, void* stream) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    p->stream = (cudaStream_t)stream;
+    return DC_OK;
+}
+
+dc_status dc_plan_scratch_bytes(dc_plan_t p, int32_t with_vals, size_t* bytes) {
+    if (!p || !bytes) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    *bytes = scratch_needed(p->n, with_vals != 0);
+    return DC_OK;
+}
+
+dc_status dc_plan_set_scratch(dc_plan_t p, void* d, size_t bytes) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (!d || !aligned16(d)) return fail(DC_ERR_INVALID_ARG, "scratch NULL or misaligned");
+    if (bytes < scratch_needed(p->n, false))
+        return fail(DC_ERR_INVALID_ARG, "scratch smaller than dc_plan_scratch_bytes");
+    if (p->scratch && p->own_scratch) cudaFree(p->scratch);
+    p->scratch = d;
+    p->scratch_bytes = bytes;
+    p->own_scratch = false;
+    return DC_OK;
+}
+
+dc_status dc_free(dc_plan_t p) {
+    if (!p) return DC_OK;
+    for (auto& t : p->pending) {
+        cudaEventDestroy(t.e0);
+        cudaEventDestroy(t.e1);
+    }
+    for (auto e : p->event_pool) cudaEventDestroy(e);
+    if (p->scratch && p->own_scratch) cudaFree(p->scratch);
+    if (p->ms_tiles) cudaFree(p->ms_tiles);
+    if (p->d_stage) cudaFree(p->d_stage);
+    delete p;
+    return DC_OK;
+}
+
+int64_t dc_plan_launch_count(dc_plan_t p) { return p ? p->launches : -1; }
+
+dc_status dc_plan_enable_timing(dc_plan_t p, int32_t enable) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    for (auto& t : p->pending) {
+        p->event_pool.push_back(t.e0);
+        p->event_pool.push_back(t.e1);
+    }
+    p->pending.clear();
+    for (int k = 0; k < DC_KERNEL_COUNT; ++k) {
+        p->acc_ms[k] = 0;
+        p->acc_n[k] = 0;
+    }
+    p->timing = enable != 0;
+    return DC_OK;
+}
+
+dc_status dc_plan_kernel_time(dc_plan_t p, int32_t kernel, double* total_ms, int64_t* launches) {
+    if (!p || kernel < 0 || kernel >= DC_KERNEL_COUNT)
+        return fail(DC_ERR_INVALID_ARG, "bad plan or kernel id");
+    for (auto& t : p->pending) {
+        cudaError_t e = cudaEventSynchronize(t.e1);
+        if (e != cudaSuccess) return cuda_fail(p, e, "cudaEventSynchronize");
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, t.e0, t.e1);
+        p->acc_ms[t.kind] += ms;
+        p->acc_n[t.kind] += 1;
+        p->event_pool.push_back(t.e0);
+        p->event_pool.push_back(t.e1);
+    }
+    p->pending.clear();
+    if (total_ms) *total_ms = p->acc_ms[kernel];
+    if (launches) *launches = p->acc_n[kernel];
+    return DC_OK;
+}
+
+dc_status dc_run_mergesort(dc_plan_t p, dc_key_type kt, void* d_keys, uint32_t* d_vals) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (p->a != 2 || p->b != 2)
+        return fail(DC_ERR_UNSUPPORTED, "runs need a == b == 2");
+    if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
+        return fail(DC_ERR_INVALID_ARG, "unknown key type");
+    if (!d_keys || !aligned16(d_keys)) return fail(DC_ERR_INVALID_ARG, "keys NULL or misaligned");
+    if (d_vals && !aligned16(d_vals)) return fail(DC_ERR_INVALID_ARG, "vals misaligned");
+    return sort_dispatch(p, kt, (uint32_t*)d_keys, d_vals);
+}
+
+dc_status dc_run_mergesort_host(dc_plan_t p, dc_key_type kt, void* h_keys, uint32_t* h_vals) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (p->a != 2 || p->b != 2)
+        return fail(DC_ERR_UNSUPPORTED, "runs need a == b == 2");
+    if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
+        return fail(DC_ERR_INVALID_ARG, "unknown key type");
+    if (!h_keys) return fail(DC_ERR_INVALID_ARG, "keys NULL");
+    size_t kb = align_up((size_t)p->n * 4, 256);
+    st = ensure_stage(p, h_vals ? 2 * kb : kb);
+    if (st != DC_OK) return st;
+    uint32_t* dk = (uint32_t*)p->d_stage;
+    uint32_t* dv = h_vals ? (uint32_t*)((char*)p->d_stage + kb) : nullptr;
+    size_t bytes = (size_t)p->n * 4;
+    DC_CUDA(p, cudaMemcpyAsync(dk, h_keys, bytes, cudaMemcpyHostToDevice, p->stream));
+    if (h_vals) DC_CUDA(p, cudaMemcpyAsync(dv, h_vals, bytes, cudaMemcpyHostToDevice, p->stream));
+    st = sort_dispatch(p, kt, dk, dv);
+    if (st != DC_OK) return st;
+    DC_CUDA(p, cudaMemcpyAsync(h_keys, dk, bytes, cudaMemcpyDeviceToHost, p->stream));
+    if (h_vals) DC_CUDA(p, cudaMemcpyAsync(h_vals, dv, bytes, cudaMemcpyDeviceToHost, p->stream));
+    DC_CUDA(p, cudaStreamSynchronize(p->stream));
+    return DC_OK;
+}
+
+dc_status dc_run_maxsubarray_async(dc_plan_t p, const int32_t* d_x, int64_t off,
+                                   dc_maxsub_result* d_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (p->a != 2 || p->b != 2) return fail(DC_ERR_UNSUPPORTED, "runs need a == b == 2");
+    if (!d_x || !aligned16(d_x)) return fail(DC_ERR_INVALID_ARG, "x NULL or misaligned");
+    if (!d_out) return fail(DC_ERR_INVALID_ARG, "out NULL");
+    return maxsub_launch(p, d_x, off, 0, d_out, nullptr);
+}
+
+dc_status dc_run_maxsubarray_tuple_async(dc_plan_t p, const int32_t* d_x, int64_t off,
+                                         dc_maxsub_tuple* d_tuple) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (p->a != 2 || p->b != 2) return fail(DC_ERR_UNSUPPORTED, "runs need a == b == 2");
+    if (!d_x || !aligned16(d_x)) return fail(DC_ERR_INVALID_ARG, "x NULL or misaligned");
+    if (!d_tuple) return fail(DC_ERR_INVALID_ARG, "tuple NULL");
+    return maxsub_launch(p, d_x, off, 1, nullptr, d_tuple);
+}
+
+dc_status dc_run_maxsubarray(dc_plan_t p, const int32_t* d_x, dc_maxsub_result* h_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!h_out) return fail(DC_ERR_INVALID_ARG, "out NULL");
+    st = ensure_ms_state(p);
+    if (st != DC_OK) return st;
+    st = dc_run_maxsubarray_async(p, d_x, 0, p->ms_res);
+    if (st != DC_OK) return st;
+    DC_CUDA(p, cudaMemcpyAsync(h_out, p->ms_res, sizeof(dc_maxsub_result),
+                               cudaMemcpyDeviceToHost, p->stream));
+    DC_CUDA(p, cudaStreamSynchronize(p->stream));
+    return DC_OK;
+}
+
+dc_status dc_run_maxsubarray_host(dc_plan_t p, const int32_t* h_x, dc_maxsub_result* h_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!h_x || !h_out) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    st = ensure_stage(p, align_up((size_t)p->n * 4, 256));
+    if (st != DC_OK) return st;
+    DC_CUDA(p, cudaMemcpyAsync(p->d_stage, h_x, (size_t)p->n * 4, cudaMemcpyHostToDevice,
+                               p->stream));
+    return dc_run_maxsubarray(p, (const int32_t*)p->d_stage, h_out);
+}
+
+dc_status dc_maxsub_combine_async(dc_plan_t p, const dc_maxsub_tuple* d_tuples, int32_t count,
+                                  dc_maxsub_result* d_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_tuples || !d_out || count < 1) return fail(DC_ERR_INVALID_ARG, "bad arguments");
+    dc::nk5_combine_tuples<<<1, 32, 0, p->stream>>>(d_tuples, count, d_out);
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+// Multi-GPU building blocks: implemented in dc_mg.cu.
+
+}  // extern "C"

@@ -1,0 +1,204 @@
+// maxsub_kernels.cuh -- the O(1)-combine instance: maximum-subarray sum.
+//
+// T(n) = 2T(n/2) + O(1) with the segment summary
+//   (tot, pre@pe, suf@ss, best@[bs,be])
+// and the ordered, associative (NOT commutative) combine below (DESIGN.md
+// Sec. 4, readings R9-R12).  Executed breadth-first like Alg 5
+// except that neighbours are combined in order (left operand = lower
+// indices): Alg 5's strided pairing a[id] + a[id+m] is only valid for a
+// commutative combine.
+//   NK4: every thread folds a contiguous chunk left to right (the leaves and
+//        the bottom levels; exact by associativity), then ordered warp-shuffle
+//        and cross-warp combines give one summary per CTA tile;
+//   NK5: the last CTA to finish (atomic ticket) combines the tile summaries in
+//        order: the top levels.
+#pragma once
+#include <cstdint>
+
+namespace dc {
+
+// Identity ("empty segment") sentinel: |any real sum| <= 2^31 * 2^30 = 2^61.
+constexpr long long kMsNeg = -(1LL << 62);
+
+struct MsTup {
+    long long tot, pre, suf, best;
+    long long pe, ss, bs, be;
+};
+
+__device__ __forceinline__ MsTup ms_empty() {
+    MsTup t;
+    t.tot = 0; t.pre = kMsNeg; t.suf = kMsNeg; t.best = kMsNeg;
+    t.pe = 0; t.ss = 0; t.bs = 0; t.be = 0;
+    return t;
+}
+
+// combine(L, R), L immediately left of R.
+//   pre : keep L.pre on ties (smallest end)
+//   suf : prefer R.tot + L.suf on ties (smallest start)
+//   best: L.best, then the crossing (L.ss, R.pe), then R.best; a later
+//         candidate replaces only if strictly larger (lexicographic order of
+//         (start, end) follows candidate order).
+__device__ __forceinline__ MsTup ms_combine(const MsTup& L, const MsTup& R) {
+    MsTup c;
+    c.tot = L.tot + R.tot;
+    long long lp = L.tot + R.pre;
+    if (L.pre >= lp) { c.pre = L.pre; c.pe = L.pe; } else { c.pre = lp; c.pe = R.pe; }
+    long long rs = R.tot + L.suf;
+    if (rs >= R.suf) { c.suf = rs; c.ss = L.ss; } else { c.suf = R.suf; c.ss = R.ss; }
+    c.best = L.best; c.bs = L.bs; c.be = L.be;
+    long long cross = L.suf + R.pre;
+    if (cross > c.best) { c.best = cross; c.bs = L.ss; c.be = R.pe; }
+    if (R.best > c.best) { c.best = R.best; c.bs = R.bs; c.be = R.be; }
+    return c;
+}
+
+// Left-to-right fold of one element x at index i: combine(T, leaf(x, i)).
+struct MsFold {
+    long long tot, pre, suf, best;
+    int pe, ss, bs, be;
+    __device__ __forceinline__ void init() {
+        tot = 0; pre = kMsNeg; suf = kMsNeg; best = kMsNeg;
+        pe = ss = bs = be = 0;
+    }
+    __device__ __forceinline__ void step(int x, int i) {
+        tot += x;
+        if (tot > pre) { pre = tot; pe = i; }
+        if (suf >= 0) suf += x; else { suf = x; ss = i; }
+        if (suf > best) { best = suf; bs = ss; be = i; }
+    }
+    __device__ __forceinline__ MsTup tup() const {
+        MsTup t;
+        t.tot = tot; t.pre = pre; t.suf = suf; t.best = best;
+        t.pe = pe; t.ss = ss; t.bs = bs; t.be = be;
+        return t;
+    }
+};
+
+__device__ __forceinline__ MsTup ms_shfl_down(const MsTup& t, int off) {
+    MsTup r;
+    r.tot = __shfl_down_sync(0xffffffffu, t.tot, off);
+    r.pre = __shfl_down_sync(0xffffffffu, t.pre, off);
+    r.suf = __shfl_down_sync(0xffffffffu, t.suf, off);
+    r.best = __shfl_down_sync(0xffffffffu, t.best, off);
+    r.pe = __shfl_down_sync(0xffffffffu, t.pe, off);
+    r.ss = __shfl_down_sync(0xffffffffu, t.ss, off);
+    r.bs = __shfl_down_sync(0xffffffffu, t.bs, off);
+    r.be = __shfl_down_sync(0xffffffffu, t.be, off);
+    return r;
+}
+
+// Ordered combine of one tuple per thread (thread order == segment order);
+// result valid in thread 0.  red[] holds NT/32 tuples of shared memory.
+template <int NT>
+__device__ __forceinline__ MsTup ms_block_combine(MsTup t, MsTup* red) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        MsTup r = ms_shfl_down(t, off);
+        if ((lane & (2 * off - 1)) == 0) t = ms_combine(t, r);
+    }
+    if (lane == 0) red[warp] = t;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        t = red[0];
+#pragma unroll 1
+        for (int q = 1; q < NT / 32; ++q) t = ms_combine(t, red[q]);
+    }
+    return t;
+}
+
+__device__ __forceinline__ void ms_store(dc_maxsub_tuple* o, const MsTup& t, long long off) {
+    o->tot = t.tot; o->pre = t.pre; o->suf = t.suf; o->best = t.best;
+    o->pe = t.pe + off; o->ss = t.ss + off; o->bs = t.bs + off; o->be = t.be + off;
+}
+
+__device__ __forceinline__ MsTup ms_load(const dc_maxsub_tuple* o) {
+    MsTup t;
+    t.tot = o->tot; t.pre = o->pre; t.suf = o->suf; t.best = o->best;
+    t.pe = o->pe; t.ss = o->ss; t.bs = o->bs; t.be = o->be;
+    return t;
+}
+
+// L2-coherent load of a summary written by another CTA of the same launch.
+__device__ __forceinline__ MsTup ms_load_cg(const dc_maxsub_tuple* o) {
+    const long long* p = reinterpret_cast<const long long*>(o);
+    MsTup t;
+    t.tot = __ldcg(p + 0); t.pre = __ldcg(p + 1); t.suf = __ldcg(p + 2); t.best = __ldcg(p + 3);
+    t.pe = __ldcg(p + 4); t.ss = __ldcg(p + 5); t.bs = __ldcg(p + 6); t.be = __ldcg(p + 7);
+    return t;
+}
+
+// NK4 + NK5.  Tile of NT*C elements per CTA, thread t folds the contiguous
+// chunk [t*C, t*C+C) of its tile.  The tile summaries go to `tiles`; the last
+// CTA combines them in order and writes either the result (mode 0) or the
+// whole-array summary tuple (mode 1), indices offset by `off`.
+template <int NT, int C>
+__global__ void __launch_bounds__(NT)
+nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__ tiles,
+           unsigned int* __restrict__ ticket, long long off, int mode,
+           dc_maxsub_result* __restrict__ out_res, dc_maxsub_tuple* __restrict__ out_tup) {
+    constexpr int TILE = NT * C;
+    __shared__ MsTup red[NT / 32];
+    __shared__ bool am_last;
+    const int tid = threadIdx.x;
+    const long long base = (long long)blockIdx.x * TILE;
+    const long long cbeg = base + (long long)tid * C;
+
+    MsFold f;
+    f.init();
+    if (cbeg + C <= n) {
+        const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
+#pragma unroll
+        for (int q = 0; q < C / 4; ++q) {
+            int4 v = __ldg(p4 + q);
+            int i = (int)(cbeg - base) + 4 * q;   // tile-local index
+            f.step(v.x, i); f.step(v.y, i + 1); f.step(v.z, i + 2); f.step(v.w, i + 3);
+        }
+    } else {
+        for (long long e = cbeg; e < n && e < cbeg + C; ++e) f.step(x[e], (int)(e - base));
+    }
+    MsTup t = f.tup();
+    t = ms_block_combine<NT>(t, red);
+    if (tid == 0) {
+        ms_store(&tiles[blockIdx.x], t, base);   // tile-local -> array index
+        __threadfence();
+        unsigned int prev = atomicAdd(ticket, 1u);
+        am_last = (prev == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!am_last) return;
+
+    // ---- NK5: ordered combine of the gridDim.x tile summaries
+    __threadfence();
+    const int nt = gridDim.x;
+    const int per = (nt + NT - 1) / NT;
+    MsTup acc = ms_empty();
+    for (int q = tid * per; q < min(nt, tid * per + per); ++q) {
+        acc = ms_combine(acc, ms_load_cg(tiles + q));
+    }
+    __syncthreads();
+    acc = ms_block_combine<NT>(acc, red);
+    if (tid == 0) {
+        if (mode == 0) {
+            out_res->sum = acc.best;
+            out_res->start = acc.bs + off;
+            out_res->end = acc.be + off;
+        } else {
+            ms_store(out_tup, acc, off);
+        }
+        *ticket = 0u;   // re-arm for the next launch on this plan
+    }
+}
+
+// Ordered combine of `count` summaries (multi-GPU: one per rank, rank order).
+__global__ void nk5_combine_tuples(const dc_maxsub_tuple* __restrict__ tups, int count,
+                                   dc_maxsub_result* __restrict__ out) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    MsTup acc = ms_empty();
+    for (int q = 0; q < count; ++q) acc = ms_combine(acc, ms_load(tups + q));
+    out->sum = acc.best;
+    out->start = acc.bs;
+    out->end = acc.be;
+}
+
+}  // namespace dc

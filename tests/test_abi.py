@@ -1,0 +1,124 @@
+"""Host-side tests of the C ABI (no GPU needed): the library loads, exports
+every function include/dc.h declares, validates arguments, and its plan
+(level table, schedule, scratch accounting) matches the closed forms of the
+recurrence T(n) = aT(n/b) + f(n) and the paper's 2n
+working space."""
+import ctypes
+import json
+import math
+import os
+import re
+import subprocess
+
+import pytest
+
+import paper_conf_ipps_lopez_ortizss13_b200 as dc
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_functions():
+    names = []
+    for fn in os.listdir(os.path.join(ROOT, "include")):
+        if fn.endswith(".h"):
+            text = open(os.path.join(ROOT, "include", fn)).read()
+            text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+            names += re.findall(r"\b(dc_\w+)\s*\(", text)
+    return sorted(set(names))
+
+
+def test_library_exports_every_declared_symbol():
+    lib = dc.lib()
+    names = declared_functions()
+    assert "dc_plan" in names and "dc_run_mergesort" in names and "dc_free" in names
+    for name in names:
+        assert hasattr(lib, name), name
+    out = subprocess.run(["nm", "-D", "--defined-only", dc._build.LIB], capture_output=True,
+                         text=True, check=True).stdout
+    exported = set(re.findall(r" T (dc_\w+)", out))
+    assert set(names) <= exported
+
+
+def test_library_is_sm100a():
+    out = subprocess.run(["cuobjdump", "--list-elf", dc._build.LIB], capture_output=True,
+                         text=True, check=True).stdout
+    assert "sm_100a" in out
+
+
+def plan_raw(n, a=2, b=2, base=1):
+    h = ctypes.c_void_p()
+    st = dc.lib().dc_plan(n, a, b, base, ctypes.byref(h))
+    return st, h
+
+
+@pytest.mark.parametrize("args", [(0, 2, 2, 1), (-5, 2, 2, 1), (2**31, 2, 2, 1), (16, 1, 2, 1),
+                                  (16, 2, 1, 1), (16, 2, 2, 0), (16, 2, 2, 17), (16, 2000, 2, 1)])
+def test_plan_validation(args):
+    st, h = plan_raw(*args)
+    assert st == 1 and not h.value
+    assert dc.lib().dc_last_error()
+
+
+def test_free_accepts_null():
+    assert dc.lib().dc_free(None) == 0
+
+
+@pytest.mark.parametrize("k", [0, 1, 5, 20, 28, 30])
+def test_level_table_closed_form_binary(k):
+    n = 1 << k
+    p = dc.Plan(n)
+    lv = p.levels()
+    assert len(lv) == k + 1                      # levels 0..log2 n
+    for i, (nodes, size) in enumerate(lv):
+        assert nodes == 2 ** i and size == n // 2 ** i
+    # leaves: n^{log_b a} = n at level log_b n
+    assert lv[-1] == (n, 1)
+
+
+@pytest.mark.parametrize("n,a,b,base", [(1000, 2, 2, 1), (3**7, 3, 3, 1), (12345, 4, 4, 16),
+                                        (10**6, 8, 2, 100), (7, 2, 2, 7)])
+def test_level_table_general(n, a, b, base):
+    lv = dc.Plan(n, a, b, base).levels()
+    for i, (nodes, size) in enumerate(lv):
+        assert nodes == a ** i
+        assert size == -(-n // b ** i)
+    assert lv[-1][1] <= base
+    if len(lv) > 1:
+        assert lv[-2][1] > base
+
+
+def test_runs_need_binary_split():
+    p = dc.Plan(1024, 4, 4, 1)
+    h = p._h
+    st = dc.lib().dc_run_mergesort(h, 0, ctypes.c_void_p(1 << 20), None)
+    assert st == 2                               # UNSUPPORTED, before any device work
+
+
+def test_run_validation_before_device_work():
+    p = dc.Plan(1024)
+    assert dc.lib().dc_run_mergesort(p._h, 0, None, None) == 1
+    assert dc.lib().dc_run_mergesort(p._h, 0, ctypes.c_void_p(0x1004), None) == 1   # misaligned
+    assert dc.lib().dc_run_mergesort(p._h, 7, ctypes.c_void_p(0x1000), None) == 1   # key type
+
+
+@pytest.mark.parametrize("n", [1, 100, 8192, 8193, 1 << 20, 1 << 28, (1 << 31) - 1])
+def test_schedule(n):
+    s = dc.Plan(n).schedule()
+    t = s["tile"]
+    assert t & (t - 1) == 0 and s["fused_levels"] == int(math.log2(t))
+    assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))
+    # fused + global levels cover the whole tree: ceil(log2 n) combine levels
+    if n > 1:
+        assert s["fused_levels"] + s["global_passes"] >= math.ceil(math.log2(n))
+
+
+def test_scratch_is_the_papers_2n_working_space():
+    # "working space of 2n*sizeof(int)" -> input + one n-int temp
+    golden = json.load(open(os.path.join(ROOT, "tests", "golden", "paper_numbers.json")))
+    ws = golden["working_space"]
+    n = ws["n"]
+    p = dc.Plan(n)
+    extra = p.scratch_bytes(False)
+    assert n * 4 + n * 4 <= n * 4 + extra             # input + scratch >= 2n ints
+    assert (n * 4 + extra) - ws["bytes"] < 0.01 * ws["bytes"]   # ... and not much more
+    assert p.scratch_bytes(True) >= 2 * n * 4

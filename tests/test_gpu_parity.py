@@ -1,0 +1,227 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Tolerance 0 everywhere (north star): keys and values are compared bit for bit
+(float keys included: +/-0.0 must keep their input order), max-subarray
+(sum, start, end) exactly.  Sizes span one tile, several tiles and ragged
+tails; BASELINE's full sizes are checked by properties that identify the
+stable sort uniquely (see test_full_size_*).
+"""
+import numpy as np
+import pytest
+import torch
+
+import dcgen
+
+pytestmark = pytest.mark.gpu
+
+TILE = 8192
+
+
+@pytest.fixture(scope="module")
+def dc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_lopez_ortizss13_b200 as m
+    return m
+
+
+def _np_keys(t, key_type):
+    a = t.cpu().numpy()
+    return a.view(np.uint32) if key_type == "u32" else (a.view(np.int32) if key_type == "i32" else a)
+
+
+def run_sort(dc, n, dist, key_type="u32", with_vals=False, seed=1):
+    keys = dcgen.sort_keys(n, dist, seed=seed, key_type=key_type, device="cuda")
+    vals = dcgen.sort_vals(n, device="cuda") if with_vals else None
+    k_in = keys.clone()
+    plan = dc.Plan(n)
+    plan.sort_(keys, vals, key_type=key_type)
+    torch.cuda.synchronize()
+    return k_in, keys, vals
+
+
+SIZES = [1, 2, 3, 4, 5, 15, 16, 17, 255, 1000, TILE - 1, TILE, TILE + 1, 2 * TILE, 3 * TILE + 5,
+         (1 << 16) + 3, 100_003, (1 << 20), (1 << 20) + 12345]
+
+
+@pytest.mark.parametrize("n", SIZES)
+@pytest.mark.parametrize("dist", ["uniform", "few"])
+def test_sort_u32_sizes(dc, oracle_mod, n, dist):
+    k_in, k_out, _ = run_sort(dc, n, dist)
+    expect = oracle_mod.mergesort(_np_keys(k_in, "u32"))
+    assert np.array_equal(_np_keys(k_out, "u32"), expect)
+
+
+@pytest.mark.parametrize("dist", ["uniform", "paper", "sorted", "reverse", "few", "equal"])
+@pytest.mark.parametrize("n", [(1 << 20) + 7, 1 << 22])
+def test_sort_u32_distributions(dc, oracle_mod, n, dist):
+    k_in, k_out, _ = run_sort(dc, n, dist, seed=3)
+    assert np.array_equal(_np_keys(k_out, "u32"), oracle_mod.mergesort(_np_keys(k_in, "u32")))
+
+
+@pytest.mark.parametrize("key_type", ["u32", "i32", "f32"])
+@pytest.mark.parametrize("n", [5, TILE + 3, 300_001, 1 << 21])
+@pytest.mark.parametrize("dist", ["uniform", "few"])
+def test_sort_key_value_stable(dc, oracle_mod, key_type, n, dist):
+    k_in, k_out, v_out = run_sort(dc, n, dist, key_type, with_vals=True, seed=7)
+    ek, ev = oracle_mod.mergesort(_np_keys(k_in, key_type), np.arange(n, dtype=np.uint32),
+                                  key_type=key_type)
+    assert np.array_equal(_np_keys(k_out, key_type).view(np.uint32), ek.view(np.uint32))
+    assert np.array_equal(v_out.cpu().numpy().view(np.uint32), ev)
+
+
+@pytest.mark.parametrize("key_type", ["i32", "f32"])
+@pytest.mark.parametrize("n", [1000, TILE * 5 + 17, 1 << 20])
+def test_sort_keys_only_signed_float(dc, oracle_mod, key_type, n):
+    k_in, k_out, _ = run_sort(dc, n, "uniform", key_type, seed=9)
+    ek = oracle_mod.mergesort(_np_keys(k_in, key_type), key_type=key_type)
+    assert np.array_equal(_np_keys(k_out, key_type).view(np.uint32), ek.view(np.uint32))
+
+
+def test_sort_max_key_values_and_pads(dc, oracle_mod):
+    # real keys equal to the pad value (0xFFFFFFFF) in a ragged last tile
+    n = 3 * TILE + 100
+    keys = torch.full((n,), -1, dtype=torch.int32, device="cuda")
+    keys[::3] = 5
+    vals = dcgen.sort_vals(n, device="cuda")
+    k_in = keys.clone()
+    dc.Plan(n).sort_(keys, vals, key_type="u32")
+    ek, ev = oracle_mod.mergesort(_np_keys(k_in, "u32"), np.arange(n, dtype=np.uint32))
+    assert np.array_equal(_np_keys(keys, "u32"), ek)
+    assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)
+
+
+def test_sort_repeated_runs_same_plan(dc, oracle_mod):
+    n = 50_000
+    plan = dc.Plan(n)
+    for seed in range(3):
+        keys = dcgen.sort_keys(n, "uniform", seed=seed, device="cuda")
+        k_in = keys.clone()
+        plan.sort_(keys, key_type="u32")
+        assert np.array_equal(_np_keys(keys, "u32"), oracle_mod.mergesort(_np_keys(k_in, "u32")))
+
+
+def test_sort_host_buffers(dc, oracle_mod):
+    n = 123_457
+    keys = dcgen.sort_keys(n, "few", seed=2).pin_memory()
+    vals = dcgen.sort_vals(n).pin_memory()
+    k_in = keys.clone()
+    dc.Plan(n).sort_host_(keys, vals, key_type="u32")
+    ek, ev = oracle_mod.mergesort(_np_keys(k_in, "u32"), np.arange(n, dtype=np.uint32))
+    assert np.array_equal(_np_keys(keys, "u32"), ek)
+    assert np.array_equal(vals.numpy().view(np.uint32), ev)
+
+
+def test_sort_2pow24_against_oracle(dc, oracle_mod):
+    n = 1 << 24
+    k_in, k_out, v_out = run_sort(dc, n, "uniform", with_vals=True, seed=3)
+    ek, ev = oracle_mod.mergesort(_np_keys(k_in, "u32"), np.arange(n, dtype=np.uint32))
+    assert np.array_equal(_np_keys(k_out, "u32"), ek)
+    assert np.array_equal(v_out.cpu().numpy().view(np.uint32), ev)
+
+
+def _assert_is_stable_sort(k_in_u32, k_out_u32, v_out):
+    """(k_out, v_out) is THE stable sort of k_in when: v_out is a permutation,
+    k_out[i] == k_in[v_out[i]], keys non-decreasing, and v_out increasing inside
+    every run of equal keys.  Holds at any size, no oracle needed."""
+    n = k_in_u32.numel()
+    v = v_out.to(torch.int64) & 0xFFFFFFFF
+    assert torch.equal(torch.bincount(v, minlength=n), torch.ones(n, dtype=torch.int64,
+                                                                 device=v.device))
+    kin = k_in_u32.to(torch.int64) & 0xFFFFFFFF
+    kout = k_out_u32.to(torch.int64) & 0xFFFFFFFF
+    assert torch.equal(kin[v], kout)
+    assert bool((kout[1:] >= kout[:-1]).all())
+    eq = kout[1:] == kout[:-1]
+    assert bool((v[1:][eq] > v[:-1][eq]).all())
+
+
+@pytest.mark.parametrize("dist", ["uniform", "few"])
+def test_full_size_2pow28_key_value(dc, dist):
+    n = 1 << 28
+    keys = dcgen.sort_keys(n, dist, seed=3, device="cuda")
+    vals = dcgen.sort_vals(n, device="cuda")
+    k_in = keys.clone()
+    dc.Plan(n).sort_(keys, vals, key_type="u32")
+    torch.cuda.synchronize()
+    _assert_is_stable_sort(k_in, keys, vals)
+    # sampled oracle positions: the i-th output is the i-th smallest key
+    del vals
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "few"])
+def test_full_size_2pow28_keys(dc, dist):
+    n = 1 << 28
+    keys = dcgen.sort_keys(n, dist, seed=3, device="cuda")
+    ref = torch.sort(keys.view(torch.uint32).to(torch.int64) & 0xFFFFFFFF, stable=True).values
+    dc.Plan(n).sort_(keys, key_type="u32")
+    torch.cuda.synchronize()
+    assert torch.equal(keys.to(torch.int64) & 0xFFFFFFFF, ref)
+
+
+# ------------------------------------------------------------ max-subarray
+
+MS_SIZES = [1, 2, 3, 31, 32, 33, 1000, 8191, 8192, 8193, 3 * 8192 + 77, 100_003, 1 << 20,
+            (1 << 20) + 5, 1 << 24]
+
+
+@pytest.mark.parametrize("n", MS_SIZES)
+@pytest.mark.parametrize("dist", ["uniform", "small"])
+def test_maxsub_sizes(dc, oracle_mod, n, dist):
+    x = dcgen.maxsub_input(n, dist, seed=2, device="cuda")
+    got = dc.Plan(n).max_subarray(x)
+    assert got == oracle_mod.maxsub(x.cpu().numpy())
+
+
+@pytest.mark.parametrize("dist", ["negative", "positive", "zero"])
+@pytest.mark.parametrize("n", [1, 777, 1 << 16, (1 << 20) + 3])
+def test_maxsub_degenerate(dc, oracle_mod, n, dist):
+    x = dcgen.maxsub_input(n, dist, seed=5, device="cuda")
+    got = dc.Plan(n).max_subarray(x)
+    assert got == oracle_mod.maxsub(x.cpu().numpy())
+
+
+def test_maxsub_extremes_and_ties(dc, oracle_mod):
+    n = 70_000
+    x = torch.full((n,), 2**31 - 1, dtype=torch.int32, device="cuda")
+    assert dc.Plan(n).max_subarray(x) == ((2**31 - 1) * n, 0, n - 1)
+    x = torch.full((n,), -2**31, dtype=torch.int32, device="cuda")
+    assert dc.Plan(n).max_subarray(x) == (-2**31, 0, 0)
+    # many equal maxima spread over tile boundaries: lexicographically smallest wins
+    x = torch.full((n,), -1, dtype=torch.int32, device="cuda")
+    x[8191] = 4; x[8192] = -4; x[8193] = 4; x[20000] = 4
+    got = dc.Plan(n).max_subarray(x)
+    assert got == oracle_mod.maxsub(x.cpu().numpy()) == (4, 8191, 8191)
+    x = torch.zeros(n, dtype=torch.int32, device="cuda")
+    x[100] = -1
+    assert dc.Plan(n).max_subarray(x) == oracle_mod.maxsub(x.cpu().numpy()) == (0, 0, 0)
+
+
+def test_maxsub_tuple_and_combine(dc, oracle_mod):
+    n = 1 << 20
+    g = 4
+    x = dcgen.maxsub_input(n, "small", seed=8, device="cuda")
+    m = n // g
+    tups = torch.empty((g, 8), dtype=torch.int64, device="cuda")
+    plans = [dc.Plan(m) for _ in range(g)]
+    for r in range(g):
+        plans[r].max_subarray_tuple_async(x[r * m:(r + 1) * m], tups[r], index_offset=r * m)
+    out = torch.empty(3, dtype=torch.int64, device="cuda")
+    plans[0].maxsub_combine_async(tups, out)
+    assert tuple(out.cpu().tolist()) == oracle_mod.maxsub(x.cpu().numpy())
+
+
+def test_maxsub_host_buffer(dc, oracle_mod):
+    n = 300_000
+    x = dcgen.maxsub_input(n, "small", seed=6).pin_memory()
+    assert dc.Plan(n).max_subarray_host(x) == oracle_mod.maxsub(x.numpy())
+
+
+def test_launch_counts(dc):
+    n = 1 << 20
+    p = dc.Plan(n)
+    keys = dcgen.sort_keys(n, "uniform", device="cuda")
+    p.sort_(keys, key_type="u32")
+    s = p.schedule()
+    assert p.launch_count() == 1 + 2 * s["global_passes"]
