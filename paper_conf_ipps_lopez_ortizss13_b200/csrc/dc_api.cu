@@ -45,11 +45,11 @@ dc_status fail(dc_status s, const std::string& msg) {
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 int nk1_smem_bytes(bool vals) {
-    const int padded = kTile + kTile / 32 + 1;
+    const int padded = dc::padded_words(kTile);
     return (vals ? 2 * padded + kTile : padded) * 4;
 }
 int nk3_smem_bytes(bool vals) {
-    const int padded = kTout + kTout / 32 + 1;
+    const int padded = dc::padded_words(kTout);
     return (vals ? 2 * padded : padded) * 4;
 }
 

@@ -38,6 +38,10 @@ struct KeyF32 {
 // (thread t owns [t*IT, t*IT+IT)) register<->smem transposes conflict-free.
 __device__ __forceinline__ int pad32(int i) { return i + (i >> 5); }
 
+// Words of a padded tile buffer; a multiple of 4 so that a second buffer
+// placed right after it stays 16-byte aligned (uint4 accesses).
+__host__ __device__ constexpr int padded_words(int tile) { return tile + tile / 32 + 4; }
+
 // Merge-path co-rank (stable): the number i of elements of A among the first
 // `diag` outputs of merge(A, B) where A wins ties:
 //   largest i with  A[i-1] <= B[diag-i]  ... equivalently binary search with
@@ -86,7 +90,7 @@ __global__ void __launch_bounds__(NT)
 nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in_v,
               uint32_t* __restrict__ out_k, uint32_t* __restrict__ out_v, long long n) {
     constexpr int TILE = NT * IT;
-    constexpr int PADDED = TILE + TILE / 32 + 1;
+    constexpr int PADDED = padded_words(TILE);
     extern __shared__ __align__(16) uint32_t smem[];
     uint32_t* sk = smem;                  // [PADDED] keys (padded index)
     uint32_t* si = smem + PADDED;         // [PADDED] indices (V only)
@@ -248,7 +252,7 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
           uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v,
           const int* __restrict__ split, long long n, long long w) {
     constexpr int TOUT = NT * IT;
-    constexpr int PADDED = TOUT + TOUT / 32 + 1;
+    constexpr int PADDED = padded_words(TOUT);
     extern __shared__ __align__(16) uint32_t smem[];
     uint32_t* sk = smem;              // [PADDED]: inputs (linear) then outputs (padded)
     uint32_t* sv = smem + PADDED;     // [PADDED]: values, same layout (V only)
