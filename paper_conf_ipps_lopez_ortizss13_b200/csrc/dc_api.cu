@@ -23,11 +23,11 @@ namespace {
 
 // ---------------------------------------------------------------- config
 constexpr int kNK1Threads = 512;
-constexpr int kNK1Items = 16;
-constexpr int kTile = kNK1Threads * kNK1Items;     // 8192 keys, 13 fused levels
+constexpr int kNK1Items = 15;
+constexpr int kTile = kNK1Threads * kNK1Items;     // 7680 keys per fused tile
 constexpr int kNK3Threads = 256;
-constexpr int kNK3Items = 16;
-constexpr int kTout = kNK3Threads * kNK3Items;      // 4096 outputs per merge CTA
+constexpr int kNK3Items = 15;
+constexpr int kTout = kNK3Threads * kNK3Items;      // 3840 outputs per merge CTA
 static_assert((2 * kTile) % kTout == 0, "merge tiles must not straddle pairs");
 constexpr int kNK4Threads = 256;
 constexpr int kNK4Chunk = 32;
@@ -44,14 +44,8 @@ dc_status fail(dc_status s, const std::string& msg) {
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-int nk1_smem_bytes(bool vals) {
-    const int padded = dc::padded_words(kTile);
-    return (vals ? 2 * padded + kTile : padded) * 4;
-}
-int nk3_smem_bytes(bool vals) {
-    const int padded = dc::padded_words(kTout);
-    return (vals ? 2 * padded : padded) * 4;
-}
+int nk1_smem_bytes(bool vals) { return (vals ? 3 : 1) * dc::tile_words(kTile, 0) * 4; }
+int nk3_smem_bytes(bool vals) { return (vals ? 2 : 1) * dc::tile_words(kTout, kNK3Items) * 4; }
 
 }  // namespace
 
@@ -367,7 +361,7 @@ dc_status dc_plan_schedule(dc_plan_t p, int32_t* tile, int32_t* fused_levels,
                            int32_t* passes) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     if (tile) *tile = kTile;
-    int f = 0;
+    int f = 0;   // levels of the binary tree inside one tile: ceil(log2(tile))
     while ((1 << f) < kTile) ++f;
     if (fused_levels) *fused_levels = f;
     if (passes) *passes = global_passes(p->n);

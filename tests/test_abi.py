@@ -105,7 +105,7 @@ def test_run_validation_before_device_work():
 def test_schedule(n):
     s = dc.Plan(n).schedule()
     t = s["tile"]
-    assert t & (t - 1) == 0 and s["fused_levels"] == int(math.log2(t))
+    assert s["fused_levels"] == math.ceil(math.log2(t))
     assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))
     # fused + global levels cover the whole tree: ceil(log2 n) combine levels
     if n > 1:
