@@ -306,7 +306,7 @@ def run_dc(args, wl):
     sorted_ok = bool((k64[1:] >= k64[:-1]).all())
     del k64
 
-    sched = plan.schedule()
+    sched = plan.schedule("u32", kv)
     peak, peak_src = peaks()
     bytes_per_key = 16 if kv else 8
     nk3_ms, nk3_n = kt["nk3_merge"]

@@ -96,12 +96,13 @@ dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t 
 dc_status dc_plan_levels(dc_plan_t plan, int32_t *num_levels, int64_t *nodes,
                          int64_t *sizes, int32_t capacity);
 
-/* Execution schedule of the a=b=2 runs: the fused bottom kernel sorts tiles
- * of `tile` keys (the leaves plus fused_levels = log2(tile) combine levels,
- * entirely on chip), then global_passes = ceil(log2(ceil(n/tile))) merge
- * passes each combine one level of the tree over HBM. */
-dc_status dc_plan_schedule(dc_plan_t plan, int32_t *tile, int32_t *fused_levels,
-                           int32_t *global_passes);
+/* Execution schedule of an a=b=2 sort of this key type (with or without
+ * values): the fused bottom kernel sorts tiles of `tile` keys (the leaves plus
+ * fused_levels = ceil(log2(tile)) levels of the binary tree, entirely on
+ * chip), then global_passes = ceil(log2(ceil(n/tile))) merge passes each
+ * combine one level of the tree over HBM.  Any output pointer may be NULL. */
+dc_status dc_plan_schedule(dc_plan_t plan, dc_key_type key_type, int32_t with_vals,
+                           int32_t *tile, int32_t *fused_levels, int32_t *global_passes);
 
 /* Stream all device work of this plan is enqueued on (a cudaStream_t). */
 dc_status dc_plan_set_stream(dc_plan_t plan, void *cuda_stream);

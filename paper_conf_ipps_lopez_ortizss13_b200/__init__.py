@@ -54,7 +54,7 @@ _I32 = ctypes.c_int32
 _SIGS = {
     "dc_plan": ([_I64, _I32, _I32, _I64, ctypes.POINTER(_P)], ctypes.c_int),
     "dc_plan_levels": ([_P, ctypes.POINTER(_I32), _P, _P, _I32], ctypes.c_int),
-    "dc_plan_schedule": ([_P, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
+    "dc_plan_schedule": ([_P, ctypes.c_int, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
                           ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_plan_set_stream": ([_P, _P], ctypes.c_int),
     "dc_plan_scratch_bytes": ([_P, _I32, ctypes.POINTER(ctypes.c_size_t)], ctypes.c_int),
@@ -149,9 +149,10 @@ class Plan:
         _check(lib().dc_plan_levels(self._h, ctypes.byref(cnt), nodes, sizes, cnt.value))
         return list(zip(nodes, sizes))
 
-    def schedule(self) -> dict:
+    def schedule(self, key_type: str = "u32", with_vals: bool = False) -> dict:
         t, f, p = _I32(), _I32(), _I32()
-        _check(lib().dc_plan_schedule(self._h, ctypes.byref(t), ctypes.byref(f), ctypes.byref(p)))
+        _check(lib().dc_plan_schedule(self._h, _KEY_NAMES[key_type], int(with_vals),
+                                      ctypes.byref(t), ctypes.byref(f), ctypes.byref(p)))
         return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value}
 
     def scratch_bytes(self, with_vals: bool = False) -> int:

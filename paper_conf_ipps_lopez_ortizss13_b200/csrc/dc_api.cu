@@ -22,13 +22,30 @@
 namespace {
 
 // ---------------------------------------------------------------- config
-constexpr int kNK1Threads = 512;
-constexpr int kNK1Items = 15;
-constexpr int kTile = kNK1Threads * kNK1Items;     // 7680 keys per fused tile
-constexpr int kNK3Threads = 256;
-constexpr int kNK3Items = 15;
-constexpr int kTout = kNK3Threads * kNK3Items;      // 3840 outputs per merge CTA
-static_assert((2 * kTile) % kTout == 0, "merge tiles must not straddle pairs");
+// Sort configuration per instantiation.  Keys-only u32/i32 (any in-register
+// network is fine) use 33 items per thread: tiles of 16896 keys, so a 2^28
+// sort needs 14 global merge passes.  Stable variants (values, or f32 keys
+// whose +0/-0 must keep their order) carry an index through an odd-even
+// transposition network and use 17 items: tiles of 8704 keys.
+struct SortCfg {
+    int nt1, it, nt3;
+    constexpr int tile() const { return nt1 * it; }
+    constexpr int tout() const { return nt3 * it; }
+};
+constexpr SortCfg kCfgFast{512, 33, 128};
+constexpr SortCfg kCfgStable{512, 17, 256};
+static_assert((2 * kCfgFast.tile()) % kCfgFast.tout() == 0, "merge tiles must not straddle pairs");
+static_assert((2 * kCfgStable.tile()) % kCfgStable.tout() == 0, "merge tiles must not straddle pairs");
+constexpr int kMinTout = kCfgFast.tout() < kCfgStable.tout() ? kCfgFast.tout() : kCfgStable.tout();
+
+template <class K, bool V>
+constexpr SortCfg cfg_for() {
+    return (V || K::kNeedStable) ? kCfgStable : kCfgFast;
+}
+SortCfg cfg_for_runtime(dc_key_type kt, bool vals) {
+    return (vals || kt == DC_KEY_F32) ? kCfgStable : kCfgFast;
+}
+
 constexpr int kNK4Threads = 256;
 constexpr int kNK4Chunk = 32;
 constexpr int kMsTile = kNK4Threads * kNK4Chunk;   // 8192 values per CTA
@@ -44,8 +61,12 @@ dc_status fail(dc_status s, const std::string& msg) {
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-int nk1_smem_bytes(bool vals) { return (vals ? 3 : 1) * dc::tile_words(kTile, 0) * 4; }
-int nk3_smem_bytes(bool vals) { return (vals ? 2 : 1) * dc::tile_words(kTout, kNK3Items) * 4; }
+int nk1_smem_bytes(SortCfg c, bool vals) {
+    return (vals ? 3 : 1) * dc::tile_words(c.tile(), 0) * 4;
+}
+int nk3_smem_bytes(SortCfg c, bool vals) {
+    return (vals ? 2 : 1) * dc::tile_words(c.tout(), c.it + 16) * 4;
+}
 
 }  // namespace
 
@@ -81,13 +102,13 @@ namespace {
 
 int64_t num_tiles(int64_t n, int64_t t) { return (n + t - 1) / t; }
 
-int global_passes(int64_t n) {
+int global_passes(int64_t n, int64_t tile) {
     int p = 0;
-    for (int64_t w = kTile; w < n; w *= 2) ++p;
+    for (int64_t w = tile; w < n; w *= 2) ++p;
     return p;
 }
 
-size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kTout) + 1; }
+size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kMinTout) + 1; }
 
 size_t scratch_needed(int64_t n, bool vals) {
     size_t kb = align_up((size_t)n * 4, 256);
@@ -183,18 +204,19 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     uint32_t* sv = hv ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
     int* split = (int*)((char*)p->scratch + kb + (hv ? kb : 0));
 
+    constexpr SortCfg C = cfg_for<K, V>();
+    auto* k1 = dc::nk1_blocksort<C.nt1, C.it, K, V>;
+    auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
     static bool attr_done = false;   // per key/value instantiation
     if (!attr_done) {
-        DC_CUDA(p, cudaFuncSetAttribute(dc::nk1_blocksort<kNK1Threads, kNK1Items, K, V>,
-                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        nk1_smem_bytes(hv)));
-        DC_CUDA(p, cudaFuncSetAttribute(dc::nk3_merge<kNK3Threads, kNK3Items, K, V>,
-                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        nk3_smem_bytes(hv)));
+        DC_CUDA(p, cudaFuncSetAttribute(k1, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        nk1_smem_bytes(C, hv)));
+        DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        nk3_smem_bytes(C, hv)));
         attr_done = true;
     }
 
-    const int P = global_passes(n);
+    const int P = global_passes(n, C.tile());
     // Ping-pong parity: pass P-1 must write the caller's buffer, so NK1
     // writes the caller's buffer iff P is even.
     uint32_t* cur_k = (P % 2 == 0) ? keys : sk;
@@ -204,27 +226,26 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
 
     // NK1: base cases + fused bottom levels (reads the caller's buffer).
     {
-    TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT);
-    dc::nk1_blocksort<kNK1Threads, kNK1Items, K, V>
-        <<<(unsigned)num_tiles(n, kTile), kNK1Threads, nk1_smem_bytes(hv), p->stream>>>(
+        TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT);
+        k1<<<(unsigned)num_tiles(n, C.tile()), C.nt1, nk1_smem_bytes(C, hv), p->stream>>>(
             keys, vals, cur_k, cur_v, n);
-    DC_LAUNCHED(p);
+        DC_LAUNCHED(p);
     }
 
-    const int tiles = (int)num_tiles(n, kTout);
-    for (int64_t w = kTile; w < n; w *= 2) {
+    const int tiles = (int)num_tiles(n, C.tout());
+    for (int64_t w = C.tile(); w < n; w *= 2) {
         {
-        TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-        dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(cur_k, n, w, kTout,
-                                                                        tiles, split);
-        DC_LAUNCHED(p);
+            TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
+            dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(cur_k, n, w,
+                                                                            C.tout(), tiles,
+                                                                            split);
+            DC_LAUNCHED(p);
         }
         {
-        TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-        dc::nk3_merge<kNK3Threads, kNK3Items, K, V>
-            <<<tiles, kNK3Threads, nk3_smem_bytes(hv), p->stream>>>(cur_k, cur_v, oth_k, oth_v,
-                                                                    split, n, w);
-        DC_LAUNCHED(p);
+            TimedScope ts(p, DC_KERNEL_NK3_MERGE);
+            k3<<<tiles, C.nt3, nk3_smem_bytes(C, hv), p->stream>>>(cur_k, cur_v, oth_k, oth_v,
+                                                                   split, n, w);
+            DC_LAUNCHED(p);
         }
         std::swap(cur_k, oth_k);
         std::swap(cur_v, oth_v);
@@ -357,14 +378,17 @@ dc_status dc_plan_levels(dc_plan_t p, int32_t* num_levels, int64_t* nodes, int64
     return DC_OK;
 }
 
-dc_status dc_plan_schedule(dc_plan_t p, int32_t* tile, int32_t* fused_levels,
-                           int32_t* passes) {
+dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32_t* tile,
+                           int32_t* fused_levels, int32_t* passes) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
-    if (tile) *tile = kTile;
+    if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
+        return fail(DC_ERR_INVALID_ARG, "unknown key type");
+    const SortCfg c = cfg_for_runtime(kt, with_vals != 0);
+    if (tile) *tile = c.tile();
     int f = 0;   // levels of the binary tree inside one tile: ceil(log2(tile))
-    while ((1 << f) < kTile) ++f;
+    while ((1 << f) < c.tile()) ++f;
     if (fused_levels) *fused_levels = f;
-    if (passes) *passes = global_passes(p->n);
+    if (passes) *passes = global_passes(p->n, c.tile());
     return DC_OK;
 }
 

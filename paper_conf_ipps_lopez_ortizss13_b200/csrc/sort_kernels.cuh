@@ -17,6 +17,8 @@
 // and the serial merge walks shared memory with +4-byte address steps.
 #pragma once
 #include <cstdint>
+#include <type_traits>
+#include <utility>
 
 namespace dc {
 
@@ -128,20 +130,45 @@ __device__ __forceinline__ void serial_merge(uint32_t ai, uint32_t a_end, uint32
 
 // Batcher odd-even merge sort network on N elements (implicitly padded with
 // +inf to a power of two; comparators touching the padding are dropped).
+// The comparator list is generated at compile time and expanded by a fold
+// expression, so every register index is a constant (the arrays stay in
+// registers; a runtime-unrolled loop nest of this size spills to local memory).
+template <int N>
+struct BatcherPairs {
+    static constexpr int P2 = (N <= 1) ? 1 : (N <= 2) ? 2 : (N <= 4) ? 4 : (N <= 8) ? 8
+                            : (N <= 16) ? 16 : (N <= 32) ? 32 : 64;
+    struct Arr {
+        int cnt;
+        short x[1024];
+        short y[1024];
+    };
+    static constexpr Arr make() {
+        Arr r{};
+        r.cnt = 0;
+        for (int p = 1; p < P2; p <<= 1)
+            for (int k = p; k >= 1; k >>= 1)
+                for (int j = k % p; j + k < P2; j += 2 * k)
+                    for (int i = 0; i < k; ++i)
+                        if (i + j + k < N && (i + j) / (2 * p) == (i + j + k) / (2 * p)) {
+                            r.x[r.cnt] = (short)(i + j);
+                            r.y[r.cnt] = (short)(i + j + k);
+                            ++r.cnt;
+                        }
+        return r;
+    }
+    static constexpr Arr pairs = make();
+};
+
+template <int N, class CAS, int... C>
+__device__ __forceinline__ void batcher_apply(CAS& cas, std::integer_sequence<int, C...>) {
+    (cas(std::integral_constant<int, BatcherPairs<N>::pairs.x[C]>{},
+         std::integral_constant<int, BatcherPairs<N>::pairs.y[C]>{}),
+     ...);
+}
+
 template <int N, class CAS>
 __device__ __forceinline__ void batcher_network(CAS&& cas) {
-    constexpr int P2 = (N <= 1) ? 1 : (N <= 2) ? 2 : (N <= 4) ? 4 : (N <= 8) ? 8
-                     : (N <= 16) ? 16 : (N <= 32) ? 32 : 64;
-#pragma unroll
-    for (int p = 1; p < P2; p <<= 1)
-#pragma unroll
-        for (int k = p; k >= 1; k >>= 1)
-#pragma unroll
-            for (int j = k % p; j + k < P2; j += 2 * k)
-#pragma unroll
-                for (int i = 0; i < k; ++i)
-                    if (i + j + k < N && (i + j) / (2 * p) == (i + j + k) / (2 * p))
-                        cas(i + j, i + j + k);
+    batcher_apply<N>(cas, std::make_integer_sequence<int, BatcherPairs<N>::pairs.cnt>{});
 }
 
 // Sort IT keys held by one thread.  Keys-only u32/i32 (stability unobservable)
@@ -150,11 +177,12 @@ __device__ __forceinline__ void batcher_network(CAS&& cas) {
 template <class K, int IT, bool V>
 __device__ __forceinline__ void thread_sort(uint32_t (&k)[IT], uint32_t (&ix)[IT]) {
     if constexpr (!V && !K::kNeedStable) {
-        batcher_network<IT>([&](int x, int y) {
-            const uint32_t lo = K::mn(k[x], k[y]);
-            const uint32_t hi = K::mx(k[x], k[y]);
-            k[x] = lo;
-            k[y] = hi;
+        batcher_network<IT>([&](auto x, auto y) {
+            constexpr int X = decltype(x)::value, Y = decltype(y)::value;
+            const uint32_t lo = K::mn(k[X], k[Y]);
+            const uint32_t hi = K::mx(k[X], k[Y]);
+            k[X] = lo;
+            k[Y] = hi;
         });
     } else {
 #pragma unroll
@@ -177,16 +205,75 @@ __device__ __forceinline__ void thread_sort(uint32_t (&k)[IT], uint32_t (&ix)[IT
     }
 }
 
+// ------------------------------------------------------- TMA bulk copies
+// 1-D bulk copies (cp.async.bulk, SASS UBLKCP) between global and shared
+// memory, completion tracked by an mbarrier transaction count (loads) or a
+// bulk group (stores).  Addresses and sizes must be multiples of 16 bytes.
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t phase) {
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(bar), "r"(phase)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes,
+                                         uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+        ::"r"(dst), "l"(src), "r"(bytes), "r"(bar)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* dst, uint32_t src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+                 "r"(src), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit_and_wait_read() {
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+// Generic-proxy shared-memory writes -> visible to the async proxy (bulk store).
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// Store words [0, count) of a shared tile to global dst (16-byte aligned):
+// the 16-byte body by one bulk copy issued by thread 0, the < 4-word tail by
+// plain stores.  Caller: every thread has written its part, then
+// fence_proxy_async_smem(); __syncthreads().
+__device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uint32_t* s,
+                                           int count) {
+    const int body = count & ~3;
+    if (threadIdx.x == 0 && body > 0) {
+        bulk_s2g(dst, smem_addr(s), 4u * body);
+        bulk_commit_and_wait_read();
+    }
+    if ((int)threadIdx.x < count - body) dst[body + threadIdx.x] = s[body + threadIdx.x];
+}
+
 // ------------------------------------------------------------------ NK1
 // One CTA sorts one tile of TILE = NT*IT keys (the last tile may be partial:
 // it is padded with K::kPad, which sorts after every real key because every
 // step is stable and the pads sit at the highest positions).
-//   1. coalesced 128-bit loads into shared memory, blocked reads (thread t
-//      holds keys [t*IT, t*IT+IT));
+//   1. one TMA bulk copy brings the tile into shared memory; thread t then
+//      reads its IT consecutive keys (conflict-free: IT is odd);
 //   2. leaves + the levels inside a thread: in-register network;
 //   3. levels with runs IT .. TILE/2: merge-path in shared memory, each
 //      thread merging IT outputs serially;
-//   4. transpose through shared memory, coalesced 128-bit stores.
+//   4. the sorted tile leaves by one TMA bulk store.
 // With values (V): the merges carry the tile-local index of every key; the
 // values wait in shared memory and are gathered by index at the end.
 template <int NT, int IT, class K, bool V>
@@ -195,44 +282,37 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
               uint32_t* __restrict__ out_k, uint32_t* __restrict__ out_v, long long n) {
     static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
     constexpr int TILE = NT * IT;
-    static_assert(TILE % 4 == 0, "tile must be a whole number of uint4");
+    static_assert(TILE % 4 == 0, "tile must be a whole number of 16-byte chunks");
     constexpr int TW = tile_words(TILE, 0);
-    constexpr int Q4 = (TILE / 4 + NT - 1) / NT;     // uint4 per thread (striped)
     extern __shared__ __align__(16) uint32_t smem[];
     uint32_t* sk = smem;              // [TW] keys
-    uint32_t* si = smem + TW;         // [TW] tile-local indices (V only)
-    uint32_t* sv = smem + 2 * TW;     // [TW] values, by original position (V only)
+    uint32_t* si = smem + TW;         // [TW] tile-local indices, then gathered values (V)
+    uint32_t* sv = smem + 2 * TW;     // [TW] values, by original position (V)
+    __shared__ __align__(8) uint64_t bar;
     const uint32_t SK = smem_addr(sk);
+    const uint32_t BAR = smem_addr(&bar);
     constexpr uint32_t SI_OFF = TW * 4;
 
     const int tid = threadIdx.x;
     const long long base = (long long)blockIdx.x * TILE;
     const int count = (int)min((long long)TILE, n - base);
+    const int body = count & ~3;       // 16-byte part moved by TMA
 
     // ---- 1. load
-    if (count == TILE) {
-        const uint4* src4 = reinterpret_cast<const uint4*>(in_k + base);
-#pragma unroll
-        for (int q = 0; q < Q4; ++q) {
-            const int e4 = q * NT + tid;
-            if (e4 < TILE / 4) reinterpret_cast<uint4*>(sk)[e4] = __ldg(src4 + e4);
-        }
-        if (V) {
-            const uint4* vsrc4 = reinterpret_cast<const uint4*>(in_v + base);
-#pragma unroll
-            for (int q = 0; q < Q4; ++q) {
-                const int e4 = q * NT + tid;
-                if (e4 < TILE / 4) reinterpret_cast<uint4*>(sv)[e4] = __ldg(vsrc4 + e4);
-            }
-        }
-    } else {
-#pragma unroll 4
-        for (int e = tid; e < TILE; e += NT) {
-            sk[e] = e < count ? __ldg(in_k + base + e) : K::kPad;
-            if (V) sv[e] = e < count ? __ldg(in_v + base + e) : 0u;
+    if (tid == 0) {
+        mbar_init(BAR, 1);
+        mbar_arrive_expect_tx(BAR, 4u * body * (V ? 2 : 1));
+        if (body > 0) {
+            bulk_g2s(SK, in_k + base, 4u * body, BAR);
+            if (V) bulk_g2s(smem_addr(sv), in_v + base, 4u * body, BAR);
         }
     }
-    __syncthreads();
+    for (int e = body + tid; e < TILE; e += NT) {   // ragged tail + pads
+        sk[e] = e < count ? in_k[base + e] : K::kPad;
+        if (V) sv[e] = e < count ? in_v[base + e] : 0u;
+    }
+    __syncthreads();                  // barrier init + tail visible
+    mbar_wait(BAR, 0);
     uint32_t k[IT];
     uint32_t ix[IT];
 #pragma unroll
@@ -267,38 +347,17 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
         }
     }
 
-    // ---- 4. store through shared memory: blocked write, striped 128-bit reads
+    // ---- 4. store: blocked write into shared memory, one bulk store
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < IT; ++j) {
         sk[tid * IT + j] = k[j];
-        if (V) si[tid * IT + j] = ix[j];
+        if (V) si[tid * IT + j] = sv[ix[j]];    // gather the values by index
     }
+    fence_proxy_async_smem();
     __syncthreads();
-    if (count == TILE) {
-        uint4* dst4 = reinterpret_cast<uint4*>(out_k + base);
-#pragma unroll
-        for (int q = 0; q < Q4; ++q) {
-            const int e4 = q * NT + tid;
-            if (e4 < TILE / 4) dst4[e4] = reinterpret_cast<const uint4*>(sk)[e4];
-        }
-        if (V) {
-            uint4* vdst4 = reinterpret_cast<uint4*>(out_v + base);
-#pragma unroll
-            for (int q = 0; q < Q4; ++q) {
-                const int e4 = q * NT + tid;
-                if (e4 < TILE / 4) {
-                    const uint4 s4 = reinterpret_cast<const uint4*>(si)[e4];
-                    vdst4[e4] = make_uint4(sv[s4.x], sv[s4.y], sv[s4.z], sv[s4.w]);
-                }
-            }
-        }
-    } else {
-        for (int e = tid; e < count; e += NT) {
-            out_k[base + e] = sk[e];
-            if (V) out_v[base + e] = sv[si[e]];
-        }
-    }
+    store_tile(out_k + base, sk, count);
+    if (V) store_tile(out_v + base, si, count);
 }
 
 // ------------------------------------------------------------------ NK2
@@ -318,10 +377,25 @@ __global__ void nk2_partition(const uint32_t* __restrict__ src, long long n, lon
 }
 
 // ------------------------------------------------------------------ NK3
+// Stage global elements [g0, g1) (any alignment) into shared memory at word
+// offset `off` + (g0 & 3): TMA copies the 16-byte-aligned superset that lies
+// below n4 = n & ~3; the caller's threads load the rest (< 4 words past n4).
+// Returns the bytes the TMA will deliver.
+__device__ __forceinline__ uint32_t stage_piece(const uint32_t* __restrict__ g, long long g0,
+                                                long long g1, long long n4, uint32_t dst_off,
+                                                uint32_t sbase, uint32_t bar) {
+    const long long al0 = g0 & ~3LL;
+    long long al1 = (g1 + 3) & ~3LL;
+    if (al1 > n4) al1 = n4;
+    const uint32_t bytes = al1 > al0 ? (uint32_t)(4 * (al1 - al0)) : 0u;
+    if (bytes) bulk_g2s(sbase + 4u * dst_off, g + al0, bytes, bar);
+    return bytes;
+}
+
 // One output tile of TOUT = NT*IT merged keys per CTA.  The A and B pieces
-// that feed the tile (known from the co-ranks) are staged in shared memory,
-// each thread finds its own IT-output diagonal there and merges serially,
-// results are transposed through shared memory for coalesced stores.
+// that feed the tile (known from the co-ranks) are staged in shared memory
+// by TMA, each thread finds its own IT-output diagonal there and merges
+// serially, and the tile leaves by one TMA bulk store.
 template <int NT, int IT, class K, bool V>
 __global__ void __launch_bounds__(NT)
 nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
@@ -329,14 +403,14 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
           const int* __restrict__ split, long long n, long long w) {
     static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
     constexpr int TOUT = NT * IT;
-    static_assert(TOUT % 4 == 0, "tile must be a whole number of uint4");
-    constexpr int TW = tile_words(TOUT, IT);
-    constexpr int Q = (TOUT + NT - 1) / NT;
-    constexpr int Q4 = (TOUT / 4 + NT - 1) / NT;
+    static_assert(TOUT % 4 == 0, "tile must be a whole number of 16-byte chunks");
+    constexpr int TW = tile_words(TOUT, IT + 16);
     extern __shared__ __align__(16) uint32_t smem[];
-    uint32_t* sk = smem;          // [TW]: A piece | B piece, then the merged tile
-    uint32_t* sv = smem + TW;     // [TW]: values, same layout (V only)
-    const uint32_t SK = smem_addr(sk);
+    uint32_t* sk = smem;          // [TW]: A piece, B piece; then the merged tile
+    uint32_t* sv = smem + TW;     // [TW]: values, same layout (V)
+    __shared__ __align__(8) uint64_t bar;
+    const uint32_t SK = smem_addr(sk), SV = smem_addr(sv);
+    const uint32_t BAR = smem_addr(&bar);
     constexpr uint32_t SV_OFF = TW * 4;
 
     const int tid = threadIdx.x;
@@ -351,63 +425,71 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
     const int i1 = (dd1 == a_len + b_len) ? (int)a_len : split[j + 1];
     const int na = i1 - i0;
     const int total = (int)(dd1 - dd0);
-    const uint32_t* gA = src_k + s + i0;
-    const uint32_t* gB = src_k + s + a_len + (dd0 - i0) - na;   // indexed by e in [na, total)
+    const int nb = total - na;
+    const long long a0 = s + i0;                       // A piece: global [a0, a0+na)
+    const long long b0 = s + a_len + (dd0 - i0);       // B piece: global [b0, b0+nb)
+    const int fa = (int)(a0 & 3), fb = (int)(b0 & 3);
+    const int ob = (fa + na + 1 + 3) & ~3;             // B region word offset (16 B aligned)
+    const uint32_t A = SK + 4u * fa, B = SK + 4u * (ob + fb);
+    const long long n4 = n & ~3LL;
 
-#pragma unroll
-    for (int q = 0; q < Q; ++q) {
-        const int e = q * NT + tid;
-        if (e < total) sk[e] = __ldg(e < na ? gA + e : gB + e);
-    }
-    if (V) {
-        const uint32_t* vA = src_v + s + i0;
-        const uint32_t* vB = src_v + s + a_len + (dd0 - i0) - na;
-#pragma unroll
-        for (int q = 0; q < Q; ++q) {
-            const int e = q * NT + tid;
-            if (e < total) sv[e] = __ldg(e < na ? vA + e : vB + e);
-        }
-    }
-    __syncthreads();
-
-    const int diag = min(tid * IT, total);
-    const int i = corank_smem<K>(SK, na, SK + 4u * na, total - na, diag);
-    uint32_t k[IT], src[IT];
-    serial_merge<K, IT, V>(SK + 4u * i, SK + 4u * na, SK + 4u * (na + diag - i),
-                           SK + 4u * total, k, src);
-    uint32_t vv[IT];
-    if (V) {
-#pragma unroll
-        for (int q = 0; q < IT; ++q) vv[q] = lds(src[q] + SV_OFF);
-    }
-    __syncthreads();
-#pragma unroll
-    for (int q = 0; q < IT; ++q) {
-        sk[tid * IT + q] = k[q];
-        if (V) sv[tid * IT + q] = vv[q];
-    }
-    __syncthreads();
-    if (total == TOUT) {
-        uint4* dst4 = reinterpret_cast<uint4*>(dst_k + d0);
-#pragma unroll
-        for (int q = 0; q < Q4; ++q) {
-            const int e4 = q * NT + tid;
-            if (e4 < TOUT / 4) dst4[e4] = reinterpret_cast<const uint4*>(sk)[e4];
-        }
+    if (tid == 0) {
+        mbar_init(BAR, 1);
+        uint32_t bytes = 0;
+        // expect_tx must precede the copies' completion: arm with the exact sum.
+        const long long al0a = a0 & ~3LL, al0b = b0 & ~3LL;
+        long long al1a = (a0 + na + 3) & ~3LL, al1b = (b0 + nb + 3) & ~3LL;
+        if (al1a > n4) al1a = n4;
+        if (al1b > n4) al1b = n4;
+        bytes += al1a > al0a ? (uint32_t)(4 * (al1a - al0a)) : 0u;
+        bytes += al1b > al0b ? (uint32_t)(4 * (al1b - al0b)) : 0u;
+        mbar_arrive_expect_tx(BAR, bytes * (V ? 2 : 1));
+        stage_piece(src_k, a0, a0 + na, n4, 0, SK, BAR);
+        stage_piece(src_k, b0, b0 + nb, n4, ob, SK, BAR);
         if (V) {
-            uint4* vdst4 = reinterpret_cast<uint4*>(dst_v + d0);
-#pragma unroll
-            for (int q = 0; q < Q4; ++q) {
-                const int e4 = q * NT + tid;
-                if (e4 < TOUT / 4) vdst4[e4] = reinterpret_cast<const uint4*>(sv)[e4];
-            }
-        }
-    } else {
-        for (int e = tid; e < total; e += NT) {
-            dst_k[d0 + e] = sk[e];
-            if (V) dst_v[d0 + e] = sv[e];
+            stage_piece(src_v, a0, a0 + na, n4, 0, SV, BAR);
+            stage_piece(src_v, b0, b0 + nb, n4, ob, SV, BAR);
         }
     }
+    // elements at or beyond n4 (only in the last pieces of the array)
+    if (a0 + na > n4) {
+        for (long long g = max(a0, n4) + tid; g < a0 + na; g += NT) {
+            sk[fa + (g - a0)] = src_k[g];
+            if (V) sv[fa + (g - a0)] = src_v[g];
+        }
+    }
+    if (b0 + nb > n4) {
+        for (long long g = max(b0, n4) + tid; g < b0 + nb; g += NT) {
+            sk[ob + fb + (g - b0)] = src_k[g];
+            if (V) sv[ob + fb + (g - b0)] = src_v[g];
+        }
+    }
+    __syncthreads();
+    mbar_wait(BAR, 0);
+
+    const int diag = tid * IT;
+    uint32_t k[IT], src[IT], vv[IT];
+    if (diag < total) {
+        const int i = corank_smem<K>(A, na, B, nb, diag);
+        serial_merge<K, IT, V>(A + 4u * i, A + 4u * na, B + 4u * (diag - i), B + 4u * nb, k,
+                               src);
+        if (V) {
+#pragma unroll
+            for (int q = 0; q < IT; ++q) vv[q] = lds(src[q] + SV_OFF);
+        }
+    }
+    __syncthreads();
+    if (diag < total) {
+#pragma unroll
+        for (int q = 0; q < IT; ++q) {
+            sk[diag + q] = k[q];
+            if (V) sv[diag + q] = vv[q];
+        }
+    }
+    fence_proxy_async_smem();
+    __syncthreads();
+    store_tile(dst_k + d0, sk, total);
+    if (V) store_tile(dst_v + d0, sv, total);
 }
 
 }  // namespace dc

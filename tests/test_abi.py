@@ -102,8 +102,9 @@ def test_run_validation_before_device_work():
 
 
 @pytest.mark.parametrize("n", [1, 100, 8192, 8193, 1 << 20, 1 << 28, (1 << 31) - 1])
-def test_schedule(n):
-    s = dc.Plan(n).schedule()
+@pytest.mark.parametrize("kt,vals", [("u32", False), ("i32", False), ("f32", False), ("u32", True)])
+def test_schedule(n, kt, vals):
+    s = dc.Plan(n).schedule(kt, vals)
     t = s["tile"]
     assert s["fused_levels"] == math.ceil(math.log2(t))
     assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))

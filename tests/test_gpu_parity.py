@@ -223,5 +223,5 @@ def test_launch_counts(dc):
     p = dc.Plan(n)
     keys = dcgen.sort_keys(n, "uniform", device="cuda")
     p.sort_(keys, key_type="u32")
-    s = p.schedule()
+    s = p.schedule("u32", False)
     assert p.launch_count() == 1 + 2 * s["global_passes"]

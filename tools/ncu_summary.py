@@ -1,0 +1,55 @@
+#!/usr/bin/env python
+"""Summarise an ncu --set full report: headline metrics + stall reasons (used for profiles/)."""
+import csv
+import io
+import json
+import re
+import subprocess
+import sys
+
+WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+        "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__throughput.avg.pct_of_peak_sustained_active",
+        "smsp__inst_executed.sum", "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active",
+        "sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active",
+        "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
+        "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum",
+        "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
+        "smsp__issue_active.avg.pct_of_peak_sustained_active"]
+
+
+def summarise(path):
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True,
+                         text=True, check=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    h, units = rows[0], rows[1]
+    res = []
+    for r in rows[2:]:
+        d = {"kernel": r[h.index("Kernel Name")][:80]}
+        for name in WANT:
+            if name in h:
+                d[name] = r[h.index(name)] + (" " + units[h.index(name)] if units[h.index(name)] else "")
+        stalls = {}
+        for i, name in enumerate(h):
+            m = re.match(r"smsp__average_warps_issue_stalled_(\w+)_per_issue_active\.ratio", name)
+            if m:
+                try:
+                    v = float(r[i])
+                except ValueError:
+                    continue
+                if v >= 0.2:
+                    stalls[m.group(1)] = v
+        d["stalls_per_issue"] = dict(sorted(stalls.items(), key=lambda x: -x[1]))
+        res.append(d)
+    return res
+
+
+if __name__ == "__main__":
+    for p in sys.argv[1:]:
+        print(p)
+        print(json.dumps(summarise(p), indent=1))
