@@ -32,8 +32,26 @@ struct SortCfg {
     constexpr int tile() const { return nt1 * it; }
     constexpr int tout() const { return nt3 * it; }
 };
-constexpr SortCfg kCfgFast{512, 33, 128};
-constexpr SortCfg kCfgStable{512, 17, 256};
+#ifndef DC_FAST_NT1
+#define DC_FAST_NT1 512
+#endif
+#ifndef DC_FAST_IT
+#define DC_FAST_IT 33
+#endif
+#ifndef DC_FAST_NT3
+#define DC_FAST_NT3 128
+#endif
+#ifndef DC_STABLE_NT1
+#define DC_STABLE_NT1 512
+#endif
+#ifndef DC_STABLE_IT
+#define DC_STABLE_IT 17
+#endif
+#ifndef DC_STABLE_NT3
+#define DC_STABLE_NT3 256
+#endif
+constexpr SortCfg kCfgFast{DC_FAST_NT1, DC_FAST_IT, DC_FAST_NT3};
+constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3};
 static_assert((2 * kCfgFast.tile()) % kCfgFast.tout() == 0, "merge tiles must not straddle pairs");
 static_assert((2 * kCfgStable.tile()) % kCfgStable.tout() == 0, "merge tiles must not straddle pairs");
 constexpr int kMinTout = kCfgFast.tout() < kCfgStable.tout() ? kCfgFast.tout() : kCfgStable.tout();
