@@ -136,11 +136,11 @@ __device__ __forceinline__ void serial_merge(uint32_t ai, uint32_t a_end, uint32
 template <int N>
 struct BatcherPairs {
     static constexpr int P2 = (N <= 1) ? 1 : (N <= 2) ? 2 : (N <= 4) ? 4 : (N <= 8) ? 8
-                            : (N <= 16) ? 16 : (N <= 32) ? 32 : 64;
+                            : (N <= 16) ? 16 : (N <= 32) ? 32 : (N <= 64) ? 64 : 128;
     struct Arr {
         int cnt;
-        short x[1024];
-        short y[1024];
+        short x[2048];
+        short y[2048];
     };
     static constexpr Arr make() {
         Arr r{};
@@ -171,9 +171,9 @@ __device__ __forceinline__ void batcher_network(CAS&& cas) {
     batcher_apply<N>(cas, std::make_integer_sequence<int, BatcherPairs<N>::pairs.cnt>{});
 }
 
-// Sort IT keys held by one thread.  Keys-only u32/i32 (stability unobservable)
-// use Batcher's network with min/max; otherwise a stable odd-even
-// transposition network carrying the indices.
+// Sort IT keys held by one thread (the leaves and the in-thread levels).
+// Keys-only u32/i32 (stability unobservable) use Batcher's network with
+// min/max; the stable variants run it on (key, index) pairs.
 template <class K, int IT, bool V>
 __device__ __forceinline__ void thread_sort(uint32_t (&k)[IT], uint32_t (&ix)[IT]) {
     if constexpr (!V && !K::kNeedStable) {
@@ -185,23 +185,19 @@ __device__ __forceinline__ void thread_sort(uint32_t (&k)[IT], uint32_t (&ix)[IT
             k[Y] = hi;
         });
     } else {
-#pragma unroll
-        for (int r = 0; r < IT; ++r) {
-#pragma unroll
-            for (int j = r & 1; j + 1 < IT; j += 2) {
-                const bool sw = K::lt(k[j + 1], k[j]);
-                const uint32_t lo = sw ? k[j + 1] : k[j];
-                const uint32_t hi = sw ? k[j] : k[j + 1];
-                k[j] = lo;
-                k[j + 1] = hi;
-                if (V) {
-                    const uint32_t ilo = sw ? ix[j + 1] : ix[j];
-                    const uint32_t ihi = sw ? ix[j] : ix[j + 1];
-                    ix[j] = ilo;
-                    ix[j + 1] = ihi;
-                }
-            }
-        }
+        // Stable: the same network on (key, tile-local index) pairs, ordered
+        // lexicographically; indices are distinct, so the order is total and
+        // the result is the stable order of the keys.
+        batcher_network<IT>([&](auto x, auto y) {
+            constexpr int X = decltype(x)::value, Y = decltype(y)::value;
+            const bool sw = K::lt(k[Y], k[X]) | (!K::lt(k[X], k[Y]) & (ix[Y] < ix[X]));
+            const uint32_t klo = sw ? k[Y] : k[X], khi = sw ? k[X] : k[Y];
+            const uint32_t ilo = sw ? ix[Y] : ix[X], ihi = sw ? ix[X] : ix[Y];
+            k[X] = klo;
+            k[Y] = khi;
+            ix[X] = ilo;
+            ix[Y] = ihi;
+        });
     }
 }
 
