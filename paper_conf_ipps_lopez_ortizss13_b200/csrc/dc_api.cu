@@ -22,11 +22,13 @@
 namespace {
 
 // ---------------------------------------------------------------- config
-// Sort configuration per instantiation.  Keys-only u32/i32 (any in-register
-// network is fine) use 33 items per thread: tiles of 16896 keys, so a 2^28
-// sort needs 14 global merge passes.  Stable variants (values, or f32 keys
-// whose +0/-0 must keep their order) carry an index through an odd-even
-// transposition network and use 17 items: tiles of 8704 keys.
+// Sort configuration per instantiation (tuned on B200 with tools/sweep.sh,
+// see DESIGN.md Sec. 5).  Keys-only u32/i32 (stability unobservable): 512
+// threads x 51 items = tiles of 26112 keys (9 shared-memory merge levels on
+// top of a 51-input register network; 14 global passes at 2^28), merge CTAs
+// of 256 x 51 = 13056 outputs.  Stable variants (values, or f32 keys whose
+// +0/-0 must keep their order) carry a tile-local index: 512 x 33 = 16896-key
+// tiles, merge CTAs of 256 x 33 outputs.
 struct SortCfg {
     int nt1, it, nt3;
     constexpr int tile() const { return nt1 * it; }
@@ -36,16 +38,16 @@ struct SortCfg {
 #define DC_FAST_NT1 512
 #endif
 #ifndef DC_FAST_IT
-#define DC_FAST_IT 33
+#define DC_FAST_IT 51
 #endif
 #ifndef DC_FAST_NT3
-#define DC_FAST_NT3 128
+#define DC_FAST_NT3 256
 #endif
 #ifndef DC_STABLE_NT1
 #define DC_STABLE_NT1 512
 #endif
 #ifndef DC_STABLE_IT
-#define DC_STABLE_IT 17
+#define DC_STABLE_IT 33
 #endif
 #ifndef DC_STABLE_NT3
 #define DC_STABLE_NT3 256

@@ -14,7 +14,7 @@ import dcgen
 
 pytestmark = pytest.mark.gpu
 
-TILE = 8192
+TILE = 26112  # keys-only fused tile (512 x 51); stable tiles are 16896
 
 
 @pytest.fixture(scope="module")
