@@ -66,9 +66,15 @@ SortCfg cfg_for_runtime(dc_key_type kt, bool vals) {
     return (vals || kt == DC_KEY_F32) ? kCfgStable : kCfgFast;
 }
 
-constexpr int kNK4Threads = 256;
-constexpr int kNK4Chunk = 32;
-constexpr int kMsTile = kNK4Threads * kNK4Chunk;   // 8192 values per CTA
+#ifndef DC_MS_NT
+#define DC_MS_NT 256
+#endif
+#ifndef DC_MS_C
+#define DC_MS_C 32
+#endif
+constexpr int kNK4Threads = DC_MS_NT;
+constexpr int kNK4Chunk = DC_MS_C;
+constexpr int kMsTile = kNK4Threads * kNK4Chunk;   // values per max-subarray CTA
 
 constexpr int64_t kMaxN = 2147483647LL;
 

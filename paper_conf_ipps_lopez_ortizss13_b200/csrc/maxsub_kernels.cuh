@@ -20,13 +20,19 @@ namespace dc {
 // Identity ("empty segment") sentinel: |any real sum| <= 2^31 * 2^30 = 2^61.
 constexpr long long kMsNeg = -(1LL << 62);
 
-struct MsTup {
+// Segment summary.  Inside a launch the indices are tile-local (int32);
+// dc_maxsub_tuple (global, int64 indices) is used between CTAs and ranks.
+template <class I>
+struct MsTupT {
     long long tot, pre, suf, best;
-    long long pe, ss, bs, be;
+    I pe, ss, bs, be;
 };
+using MsTup = MsTupT<int>;
+using MsTupG = MsTupT<long long>;
 
-__device__ __forceinline__ MsTup ms_empty() {
-    MsTup t;
+template <class I>
+__device__ __forceinline__ MsTupT<I> ms_empty() {
+    MsTupT<I> t;
     t.tot = 0; t.pre = kMsNeg; t.suf = kMsNeg; t.best = kMsNeg;
     t.pe = 0; t.ss = 0; t.bs = 0; t.be = 0;
     return t;
@@ -38,21 +44,31 @@ __device__ __forceinline__ MsTup ms_empty() {
 //   best: L.best, then the crossing (L.ss, R.pe), then R.best; a later
 //         candidate replaces only if strictly larger (lexicographic order of
 //         (start, end) follows candidate order).
-__device__ __forceinline__ MsTup ms_combine(const MsTup& L, const MsTup& R) {
-    MsTup c;
+template <class I>
+__device__ __forceinline__ MsTupT<I> ms_combine(const MsTupT<I>& L, const MsTupT<I>& R) {
+    MsTupT<I> c;
     c.tot = L.tot + R.tot;
-    long long lp = L.tot + R.pre;
+    const long long lp = L.tot + R.pre;
     if (L.pre >= lp) { c.pre = L.pre; c.pe = L.pe; } else { c.pre = lp; c.pe = R.pe; }
-    long long rs = R.tot + L.suf;
+    const long long rs = R.tot + L.suf;
     if (rs >= R.suf) { c.suf = rs; c.ss = L.ss; } else { c.suf = R.suf; c.ss = R.ss; }
     c.best = L.best; c.bs = L.bs; c.be = L.be;
-    long long cross = L.suf + R.pre;
+    const long long cross = L.suf + R.pre;
     if (cross > c.best) { c.best = cross; c.bs = L.ss; c.be = R.pe; }
     if (R.best > c.best) { c.best = R.best; c.bs = R.bs; c.be = R.be; }
     return c;
 }
 
-// Left-to-right fold of one element x at index i: combine(T, leaf(x, i)).
+// a + x (x sign-extended) as one IMAD.WIDE on the FMA pipe, keeping the
+// integer ALU pipe (the fold's bottleneck) for compares and selects.
+__device__ __forceinline__ long long add_wide(long long a, int x) {
+    long long r;
+    asm("mad.wide.s32 %0, %1, 1, %2;" : "=l"(r) : "r"(x), "l"(a));
+    return r;
+}
+
+// Left-to-right fold of one element x at index i: combine(T, leaf(x, i)),
+// which is Kadane's step with the tie rules above.
 struct MsFold {
     long long tot, pre, suf, best;
     int pe, ss, bs, be;
@@ -61,10 +77,17 @@ struct MsFold {
         pe = ss = bs = be = 0;
     }
     __device__ __forceinline__ void step(int x, int i) {
-        tot += x;
-        if (tot > pre) { pre = tot; pe = i; }
-        if (suf >= 0) suf += x; else { suf = x; ss = i; }
-        if (suf > best) { best = suf; bs = ss; be = i; }
+        tot = add_wide(tot, x);
+        const bool up = tot > pre;                 // strict: smallest end
+        pre = up ? tot : pre;
+        pe = up ? i : pe;
+        const bool restart = suf < 0;              // max(suf + x, x), ties keep suf
+        suf = add_wide(restart ? 0LL : suf, x);
+        ss = restart ? i : ss;
+        const bool better = suf > best;            // strict: smallest (start, end)
+        best = better ? suf : best;
+        bs = better ? ss : bs;
+        be = better ? i : be;
     }
     __device__ __forceinline__ MsTup tup() const {
         MsTup t;
@@ -74,8 +97,9 @@ struct MsFold {
     }
 };
 
-__device__ __forceinline__ MsTup ms_shfl_down(const MsTup& t, int off) {
-    MsTup r;
+template <class I>
+__device__ __forceinline__ MsTupT<I> ms_shfl_down(const MsTupT<I>& t, int off) {
+    MsTupT<I> r;
     r.tot = __shfl_down_sync(0xffffffffu, t.tot, off);
     r.pre = __shfl_down_sync(0xffffffffu, t.pre, off);
     r.suf = __shfl_down_sync(0xffffffffu, t.suf, off);
@@ -87,45 +111,60 @@ __device__ __forceinline__ MsTup ms_shfl_down(const MsTup& t, int off) {
     return r;
 }
 
-// Ordered combine of one tuple per thread (thread order == segment order);
-// result valid in thread 0.  red[] holds NT/32 tuples of shared memory.
-template <int NT>
-__device__ __forceinline__ MsTup ms_block_combine(MsTup t, MsTup* red) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+// Ordered combine across the first `width` lanes (lane order == segment
+// order); the result is valid in lane 0.
+template <int WIDTH, class I>
+__device__ __forceinline__ MsTupT<I> ms_warp_combine(MsTupT<I> t) {
+    const int lane = threadIdx.x & 31;
 #pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-        MsTup r = ms_shfl_down(t, off);
+    for (int off = 1; off < WIDTH; off <<= 1) {
+        MsTupT<I> r = ms_shfl_down(t, off);
         if ((lane & (2 * off - 1)) == 0) t = ms_combine(t, r);
-    }
-    if (lane == 0) red[warp] = t;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        t = red[0];
-#pragma unroll 1
-        for (int q = 1; q < NT / 32; ++q) t = ms_combine(t, red[q]);
     }
     return t;
 }
 
-__device__ __forceinline__ void ms_store(dc_maxsub_tuple* o, const MsTup& t, long long off) {
+// Ordered combine of one tuple per thread of the CTA; result in thread 0.
+template <int NT, class I>
+__device__ __forceinline__ MsTupT<I> ms_block_combine(MsTupT<I> t, MsTupT<I>* red) {
+    static_assert(NT / 32 <= 32, "one warp combines the warp results");
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    t = ms_warp_combine<32>(t);
+    if (lane == 0) red[warp] = t;
+    __syncthreads();
+    if (warp == 0) {
+        t = lane < NT / 32 ? red[lane] : ms_empty<I>();
+        t = ms_warp_combine<NT / 32>(t);
+    }
+    return t;
+}
+
+__device__ __forceinline__ void ms_store(dc_maxsub_tuple* o, const MsTupG& t, long long off) {
     o->tot = t.tot; o->pre = t.pre; o->suf = t.suf; o->best = t.best;
     o->pe = t.pe + off; o->ss = t.ss + off; o->bs = t.bs + off; o->be = t.be + off;
 }
 
-__device__ __forceinline__ MsTup ms_load(const dc_maxsub_tuple* o) {
-    MsTup t;
+__device__ __forceinline__ MsTupG ms_load(const dc_maxsub_tuple* o) {
+    MsTupG t;
     t.tot = o->tot; t.pre = o->pre; t.suf = o->suf; t.best = o->best;
     t.pe = o->pe; t.ss = o->ss; t.bs = o->bs; t.be = o->be;
     return t;
 }
 
 // L2-coherent load of a summary written by another CTA of the same launch.
-__device__ __forceinline__ MsTup ms_load_cg(const dc_maxsub_tuple* o) {
+__device__ __forceinline__ MsTupG ms_load_cg(const dc_maxsub_tuple* o) {
     const long long* p = reinterpret_cast<const long long*>(o);
-    MsTup t;
+    MsTupG t;
     t.tot = __ldcg(p + 0); t.pre = __ldcg(p + 1); t.suf = __ldcg(p + 2); t.best = __ldcg(p + 3);
     t.pe = __ldcg(p + 4); t.ss = __ldcg(p + 5); t.bs = __ldcg(p + 6); t.be = __ldcg(p + 7);
     return t;
+}
+
+__device__ __forceinline__ MsTupG ms_widen(const MsTup& t, long long base) {
+    MsTupG g;
+    g.tot = t.tot; g.pre = t.pre; g.suf = t.suf; g.best = t.best;
+    g.pe = t.pe + base; g.ss = t.ss + base; g.bs = t.bs + base; g.be = t.be + base;
+    return g;
 }
 
 // NK4 + NK5.  Tile of NT*C elements per CTA, thread t folds the contiguous
@@ -139,6 +178,7 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
            dc_maxsub_result* __restrict__ out_res, dc_maxsub_tuple* __restrict__ out_tup) {
     constexpr int TILE = NT * C;
     __shared__ MsTup red[NT / 32];
+    __shared__ MsTupG redg[NT / 32];
     __shared__ bool am_last;
     const int tid = threadIdx.x;
     const long long base = (long long)blockIdx.x * TILE;
@@ -148,36 +188,38 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
     f.init();
     if (cbeg + C <= n) {
         const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
+        int4 v[C / 4];
+#pragma unroll
+        for (int q = 0; q < C / 4; ++q) v[q] = __ldg(p4 + q);
+        const int i0 = tid * C;                    // tile-local index
 #pragma unroll
         for (int q = 0; q < C / 4; ++q) {
-            int4 v = __ldg(p4 + q);
-            int i = (int)(cbeg - base) + 4 * q;   // tile-local index
-            f.step(v.x, i); f.step(v.y, i + 1); f.step(v.z, i + 2); f.step(v.w, i + 3);
+            f.step(v[q].x, i0 + 4 * q);
+            f.step(v[q].y, i0 + 4 * q + 1);
+            f.step(v[q].z, i0 + 4 * q + 2);
+            f.step(v[q].w, i0 + 4 * q + 3);
         }
     } else {
         for (long long e = cbeg; e < n && e < cbeg + C; ++e) f.step(x[e], (int)(e - base));
     }
-    MsTup t = f.tup();
-    t = ms_block_combine<NT>(t, red);
+    MsTup t = ms_block_combine<NT>(f.tup(), red);
     if (tid == 0) {
-        ms_store(&tiles[blockIdx.x], t, base);   // tile-local -> array index
+        ms_store(&tiles[blockIdx.x], ms_widen(t, 0), base);   // tile-local -> array index
         __threadfence();
-        unsigned int prev = atomicAdd(ticket, 1u);
+        const unsigned int prev = atomicAdd(ticket, 1u);
         am_last = (prev == gridDim.x - 1);
     }
     __syncthreads();
     if (!am_last) return;
 
-    // ---- NK5: ordered combine of the gridDim.x tile summaries
+    // ---- NK5: ordered combine of the gridDim.x tile summaries (top levels)
     __threadfence();
     const int nt = gridDim.x;
     const int per = (nt + NT - 1) / NT;
-    MsTup acc = ms_empty();
-    for (int q = tid * per; q < min(nt, tid * per + per); ++q) {
+    MsTupG acc = ms_empty<long long>();
+    for (int q = tid * per; q < min(nt, tid * per + per); ++q)
         acc = ms_combine(acc, ms_load_cg(tiles + q));
-    }
-    __syncthreads();
-    acc = ms_block_combine<NT>(acc, red);
+    acc = ms_block_combine<NT>(acc, redg);
     if (tid == 0) {
         if (mode == 0) {
             out_res->sum = acc.best;
@@ -194,7 +236,7 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
 __global__ void nk5_combine_tuples(const dc_maxsub_tuple* __restrict__ tups, int count,
                                    dc_maxsub_result* __restrict__ out) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    MsTup acc = ms_empty();
+    MsTupG acc = ms_empty<long long>();
     for (int q = 0; q < count; ++q) acc = ms_combine(acc, ms_load(tups + q));
     out->sum = acc.best;
     out->start = acc.bs;

@@ -10,7 +10,7 @@ for spec in $1; do
   python -c "
 import json,sys
 d=json.loads(open('gpurun_out/sweep_$name.json').read().strip().splitlines()[-1])
-k=d['kernels']
-print('$name', round(d['ms_per_step'],3), 'ms', ' '.join(f\"{n}={v['avg_ms']*v['launches_per_step']:.3f}\" for n,v in k.items()))
+k=d.get('kernels', {})
+print('$name', round(d['ms_per_step'],4), 'ms', ' '.join(f\"{n}={v['avg_ms']*v['launches_per_step']:.4f}\" for n,v in k.items()), 'roof', round(d['roofline']['frac'],3))
 " || tail -3 gpurun_out/sweep_$name.json
 done
