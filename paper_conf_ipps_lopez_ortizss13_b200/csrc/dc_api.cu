@@ -295,18 +295,34 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
     return fail(DC_ERR_INVALID_ARG, "unknown key type");
 }
 
+// Max-subarray grid: about one wave of resident CTAs (occupancy x SMs),
+// never more CTAs than tiles.
+int ms_grid(dc_plan_t p) {
+    static int grid = 0;
+    if (!grid) {
+        int dev = 0, sms = 148, occ = 4;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, dc::nk4_maxsub<kNK4Threads, kNK4Chunk>,
+                                                      kNK4Threads, 0);
+        grid = sms * (occ > 0 ? occ : 1);
+    }
+    const int64_t tiles = num_tiles(p->n, kMsTile);
+    return (int)(tiles < grid ? tiles : grid);
+}
+
 dc_status ensure_ms_state(dc_plan_t p) {
     if (p->ms_tiles) return DC_OK;
-    size_t tiles = (size_t)num_tiles(p->n, kMsTile);
+    const size_t parts = (size_t)ms_grid(p);
     void* ptr = nullptr;
-    size_t bytes = align_up(tiles * sizeof(dc_maxsub_tuple), 256) + 256 + 256;
+    const size_t bytes = align_up(parts * sizeof(dc_maxsub_tuple), 256) + 256 + 256;
     if (cudaMalloc(&ptr, bytes) != cudaSuccess) {
         cudaGetLastError();
         return fail(DC_ERR_OUT_OF_MEMORY, "max-subarray state cudaMalloc failed");
     }
     DC_CUDA(p, cudaMemsetAsync(ptr, 0, bytes, p->stream));
     p->ms_tiles = (dc_maxsub_tuple*)ptr;
-    p->ms_ticket = (unsigned int*)((char*)ptr + align_up(tiles * sizeof(dc_maxsub_tuple), 256));
+    p->ms_ticket = (unsigned int*)((char*)ptr + align_up(parts * sizeof(dc_maxsub_tuple), 256));
     p->ms_res = (dc_maxsub_result*)((char*)p->ms_ticket + 256);
     return DC_OK;
 }
@@ -315,9 +331,8 @@ dc_status maxsub_launch(dc_plan_t p, const int32_t* d_x, int64_t off, int mode,
                         dc_maxsub_result* out_res, dc_maxsub_tuple* out_tup) {
     dc_status st = ensure_ms_state(p);
     if (st != DC_OK) return st;
-    const int64_t tiles = num_tiles(p->n, kMsTile);
     TimedScope ts(p, DC_KERNEL_NK4_MAXSUB);
-    dc::nk4_maxsub<kNK4Threads, kNK4Chunk><<<(unsigned)tiles, kNK4Threads, 0, p->stream>>>(
+    dc::nk4_maxsub<kNK4Threads, kNK4Chunk><<<ms_grid(p), kNK4Threads, 0, p->stream>>>(
         d_x, p->n, p->ms_tiles, p->ms_ticket, off, mode, out_res, out_tup);
     DC_LAUNCHED(p);
     return DC_OK;

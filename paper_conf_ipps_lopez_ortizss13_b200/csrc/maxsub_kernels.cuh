@@ -167,13 +167,15 @@ __device__ __forceinline__ MsTupG ms_widen(const MsTup& t, long long base) {
     return g;
 }
 
-// NK4 + NK5.  Tile of NT*C elements per CTA, thread t folds the contiguous
-// chunk [t*C, t*C+C) of its tile.  The tile summaries go to `tiles`; the last
-// CTA combines them in order and writes either the result (mode 0) or the
-// whole-array summary tuple (mode 1), indices offset by `off`.
+// NK4 + NK5.  Tiles of NT*C elements; CTA c folds the contiguous range of
+// tiles [c*nt/G, (c+1)*nt/G) (G = gridDim.x, about one wave of resident
+// CTAs), thread t folding the contiguous chunk [t*C, t*C+C) of each tile, and
+// combines them in order into one summary.  The last CTA to finish (atomic
+// ticket) combines the G summaries in order and writes either the result
+// (mode 0) or the whole-array summary tuple (mode 1), indices offset by `off`.
 template <int NT, int C>
 __global__ void __launch_bounds__(NT)
-nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__ tiles,
+nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__ parts,
            unsigned int* __restrict__ ticket, long long off, int mode,
            dc_maxsub_result* __restrict__ out_res, dc_maxsub_tuple* __restrict__ out_tup) {
     constexpr int TILE = NT * C;
@@ -181,30 +183,38 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
     __shared__ MsTupG redg[NT / 32];
     __shared__ bool am_last;
     const int tid = threadIdx.x;
-    const long long base = (long long)blockIdx.x * TILE;
-    const long long cbeg = base + (long long)tid * C;
+    const long long ntiles = (n + TILE - 1) / TILE;
+    const long long t0 = ntiles * blockIdx.x / gridDim.x;
+    const long long t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
 
-    MsFold f;
-    f.init();
-    if (cbeg + C <= n) {
-        const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
-        int4 v[C / 4];
+    MsTupG acc = ms_empty<long long>();   // thread 0: this CTA's running summary
+    for (long long tile = t0; tile < t1; ++tile) {
+        const long long base = tile * TILE;
+        const long long cbeg = base + (long long)tid * C;
+        MsFold f;
+        f.init();
+        if (cbeg + C <= n) {
+            const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
+            int4 v[C / 4];
 #pragma unroll
-        for (int q = 0; q < C / 4; ++q) v[q] = __ldg(p4 + q);
-        const int i0 = tid * C;                    // tile-local index
+            for (int q = 0; q < C / 4; ++q) v[q] = __ldg(p4 + q);
+            const int i0 = tid * C;                // tile-local index
 #pragma unroll
-        for (int q = 0; q < C / 4; ++q) {
-            f.step(v[q].x, i0 + 4 * q);
-            f.step(v[q].y, i0 + 4 * q + 1);
-            f.step(v[q].z, i0 + 4 * q + 2);
-            f.step(v[q].w, i0 + 4 * q + 3);
+            for (int q = 0; q < C / 4; ++q) {
+                f.step(v[q].x, i0 + 4 * q);
+                f.step(v[q].y, i0 + 4 * q + 1);
+                f.step(v[q].z, i0 + 4 * q + 2);
+                f.step(v[q].w, i0 + 4 * q + 3);
+            }
+        } else {
+            for (long long e = cbeg; e < n && e < cbeg + C; ++e) f.step(x[e], (int)(e - base));
         }
-    } else {
-        for (long long e = cbeg; e < n && e < cbeg + C; ++e) f.step(x[e], (int)(e - base));
+        const MsTup t = ms_block_combine<NT>(f.tup(), red);
+        if (tid == 0) acc = ms_combine(acc, ms_widen(t, base));
+        __syncthreads();                           // red[] reused by the next tile
     }
-    MsTup t = ms_block_combine<NT>(f.tup(), red);
     if (tid == 0) {
-        ms_store(&tiles[blockIdx.x], ms_widen(t, 0), base);   // tile-local -> array index
+        ms_store(&parts[blockIdx.x], acc, 0);
         __threadfence();
         const unsigned int prev = atomicAdd(ticket, 1u);
         am_last = (prev == gridDim.x - 1);
@@ -212,21 +222,20 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
     __syncthreads();
     if (!am_last) return;
 
-    // ---- NK5: ordered combine of the gridDim.x tile summaries (top levels)
+    // ---- NK5: ordered combine of the G part summaries (top levels)
     __threadfence();
-    const int nt = gridDim.x;
-    const int per = (nt + NT - 1) / NT;
-    MsTupG acc = ms_empty<long long>();
-    for (int q = tid * per; q < min(nt, tid * per + per); ++q)
-        acc = ms_combine(acc, ms_load_cg(tiles + q));
-    acc = ms_block_combine<NT>(acc, redg);
+    const int np = gridDim.x;
+    const int per = (np + NT - 1) / NT;
+    MsTupG a = ms_empty<long long>();
+    for (int q = tid * per; q < min(np, tid * per + per); ++q) a = ms_combine(a, ms_load_cg(parts + q));
+    a = ms_block_combine<NT>(a, redg);
     if (tid == 0) {
         if (mode == 0) {
-            out_res->sum = acc.best;
-            out_res->start = acc.bs + off;
-            out_res->end = acc.be + off;
+            out_res->sum = a.best;
+            out_res->start = a.bs + off;
+            out_res->end = a.be + off;
         } else {
-            ms_store(out_tup, acc, off);
+            ms_store(out_tup, a, off);
         }
         *ticket = 0u;   // re-arm for the next launch on this plan
     }
