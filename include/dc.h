@@ -154,6 +154,66 @@ dc_status dc_maxsub_combine_async(dc_plan_t plan, const dc_maxsub_tuple *d_tuple
 /* Host buffers end to end: copy h_x to the device, run, return the result. */
 dc_status dc_run_maxsubarray_host(dc_plan_t plan, const int32_t *h_x, dc_maxsub_result *h_out);
 
+/* ------------------------------------------- multi-GPU building blocks */
+/* The top log2(G) levels of a G-way sharded sort (not in
+ * the paper, which notes the method "could easily be extended to multiple gpu
+ * cards").  Rank r holds global positions [r*m, (r+1)*m) and has
+ * sorted them with dc_run_mergesort.  The collectives between these steps
+ * run in torch.distributed (NCCL over NVLink); these calls are the per-rank
+ * device work.  All are enqueue-only on the plan stream unless stated.
+ * Composite order: element (key, rank, position) -- the global stable order.
+ */
+
+/* Words of one rank's splitter send buffer for `world` ranks and windows of
+ * wcap keys: 6*(world-1) header words (three int64 per boundary) followed by
+ * (world-1)*wcap key words.  0 if world < 2. */
+int64_t dc_mg_sendbuf_words(int32_t world, int64_t wcap);
+
+/* Samples of a sorted shard: d_samples[j] = d_keys[j*stride] for
+ * j < ceil(n/stride). */
+dc_status dc_mg_sample(dc_plan_t plan, const uint32_t *d_keys, int64_t n, int64_t stride,
+                       uint32_t *d_samples);
+
+/* Composite counts.  d_cand holds the all-gathered samples of every rank,
+ * rank-major (candidate c = owner*per_rank + j is the element at position
+ * j*stride of rank `owner`), cands = world*per_rank < 2^24.  Writes, for
+ * every candidate, the number of elements of this rank's sorted shard
+ * d_keys[0..n) strictly below it in composite order (int64 d_counts[c]).
+ * Summing d_counts over ranks gives every candidate's global position. */
+dc_status dc_mg_count(dc_plan_t plan, dc_key_type key_type, const uint32_t *d_keys, int64_t n,
+                      int32_t rank, const uint32_t *d_cand, int64_t per_rank, int64_t stride,
+                      int64_t cands, int64_t *d_counts);
+
+/* Splitter windows.  d_ranks: global positions of the candidates (the
+ * all-reduced sum of every rank's d_counts).  For every boundary k_d = d*n,
+ * d = 1..world-1, brackets k_d between two consecutive candidates and writes
+ * into d_sendbuf (dc_mg_sendbuf_words words) this rank's elements strictly
+ * between them (< stride of them, window capacity wcap >= stride) with
+ * {lo, len, t}: their shard range and how many window elements of all ranks
+ * belong to the first k_d. */
+dc_status dc_mg_windows(dc_plan_t plan, const uint32_t *d_keys, int64_t n, int32_t rank,
+                        int32_t world, const int64_t *d_counts, const int64_t *d_ranks,
+                        int64_t per_rank, int64_t cands, int64_t wcap, uint32_t *d_sendbuf);
+
+/* Exact split matrix from the all-gathered send buffers of all ranks (rank
+ * order, back to back): d_cmat[r*(world+1) + d] = number of rank-r elements
+ * among the first d*shard_n of the global stable order (d = 0..world).
+ * Requires world*wcap*4 <= 200 KiB. */
+dc_status dc_mg_split_matrix(dc_plan_t plan, dc_key_type key_type, const uint32_t *d_gathered,
+                             int32_t world, int64_t shard_n, int64_t wcap, int64_t *d_cmat);
+
+/* Synchronises and reports whether a window overflowed its capacity
+ * (*h_err != 0 means the shard was not sorted or wcap < stride). */
+dc_status dc_mg_error(dc_plan_t plan, int32_t *h_err);
+
+/* Local stable merge of `runs` sorted runs stored back to back in d_in_keys
+ * (run r has h_run_len[r] elements, host array; total <= plan n) into
+ * d_out_keys; earlier runs win ties.  Values (nullable, both or neither)
+ * move with their keys.  d_in_* is used as ping-pong space and clobbered. */
+dc_status dc_mg_merge_runs(dc_plan_t plan, dc_key_type key_type, uint32_t *d_in_keys,
+                           uint32_t *d_in_vals, uint32_t *d_out_keys, uint32_t *d_out_vals,
+                           const int64_t *h_run_len, int32_t runs);
+
 /* ------------------------------------------------------ instrumentation */
 
 /* Kernel classes for dc_plan_kernel_time. */

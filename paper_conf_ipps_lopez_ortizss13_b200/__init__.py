@@ -77,6 +77,16 @@ _SIGS = {
                             ctypes.c_int),
 }
 
+_SIGS.update({
+    "dc_mg_sendbuf_words": ([_I32, _I64], _I64),
+    "dc_mg_sample": ([_P, _P, _I64, _I64, _P], ctypes.c_int),
+    "dc_mg_count": ([_P, ctypes.c_int, _P, _I64, _I32, _P, _I64, _I64, _I64, _P], ctypes.c_int),
+    "dc_mg_windows": ([_P, _P, _I64, _I32, _I32, _P, _P, _I64, _I64, _I64, _P], ctypes.c_int),
+    "dc_mg_split_matrix": ([_P, ctypes.c_int, _P, _I32, _I64, _I64, _P], ctypes.c_int),
+    "dc_mg_error": ([_P, ctypes.POINTER(_I32)], ctypes.c_int),
+    "dc_mg_merge_runs": ([_P, ctypes.c_int, _P, _P, _P, _P, _P, _I32], ctypes.c_int),
+})
+
 #: kernel classes of dc_plan_kernel_time
 KERNELS = {"nk1_blocksort": 0, "nk2_partition": 1, "nk3_merge": 2, "nk4_maxsub": 3}
 
@@ -253,6 +263,63 @@ class Plan:
         r = MaxsubResult()
         _check(lib().dc_run_maxsubarray_host(self._h, x.data_ptr(), ctypes.byref(r)))
         return (r.sum, r.start, r.end)
+
+
+    # ------------------------------------------ multi-GPU building blocks
+    def mg_sample(self, keys: torch.Tensor, stride: int) -> torch.Tensor:
+        """Every stride-th key of this rank's sorted shard (uint32 bits as int32)."""
+        _require_cuda(keys, "keys")
+        out = torch.empty((keys.numel() + stride - 1) // stride, dtype=torch.int32,
+                          device=keys.device)
+        self._bind_stream(keys)
+        _check(lib().dc_mg_sample(self._h, keys.data_ptr(), keys.numel(), stride, out.data_ptr()))
+        return out
+
+    def mg_count(self, keys: torch.Tensor, rank: int, cand: torch.Tensor, per_rank: int,
+                 stride: int, key_type: str | None = None) -> torch.Tensor:
+        """Composite counts of this rank's elements below every candidate (int64)."""
+        out = torch.empty(cand.numel(), dtype=torch.int64, device=keys.device)
+        self._bind_stream(keys)
+        _check(lib().dc_mg_count(self._h, _key_type(keys, key_type), keys.data_ptr(),
+                                 keys.numel(), rank, cand.data_ptr(), per_rank, stride,
+                                 cand.numel(), out.data_ptr()))
+        return out
+
+    def mg_windows(self, keys: torch.Tensor, rank: int, world: int, counts: torch.Tensor,
+                   ranks: torch.Tensor, per_rank: int, wcap: int) -> torch.Tensor:
+        words = int(lib().dc_mg_sendbuf_words(world, wcap))
+        out = torch.zeros(words, dtype=torch.int32, device=keys.device)
+        self._bind_stream(keys)
+        _check(lib().dc_mg_windows(self._h, keys.data_ptr(), keys.numel(), rank, world,
+                                   counts.data_ptr(), ranks.data_ptr(), per_rank, counts.numel(),
+                                   wcap, out.data_ptr()))
+        return out
+
+    def mg_split_matrix(self, gathered: torch.Tensor, world: int, shard_n: int, wcap: int,
+                        key_type: str) -> torch.Tensor:
+        out = torch.empty((world, world + 1), dtype=torch.int64, device=gathered.device)
+        self._bind_stream(gathered)
+        _check(lib().dc_mg_split_matrix(self._h, _KEY_NAMES[key_type], gathered.data_ptr(),
+                                        world, shard_n, wcap, out.data_ptr()))
+        return out
+
+    def mg_error(self) -> int:
+        e = _I32()
+        _check(lib().dc_mg_error(self._h, ctypes.byref(e)))
+        return e.value
+
+    def mg_merge_runs(self, in_keys: torch.Tensor, in_vals: torch.Tensor | None,
+                      out_keys: torch.Tensor, out_vals: torch.Tensor | None, run_len: list[int],
+                      key_type: str | None = None) -> torch.Tensor:
+        """Stable merge of back-to-back sorted runs (earlier runs win ties)."""
+        lens = (_I64 * len(run_len))(*run_len)
+        self._bind_stream(in_keys)
+        _check(lib().dc_mg_merge_runs(self._h, _key_type(in_keys, key_type), in_keys.data_ptr(),
+                                      None if in_vals is None else in_vals.data_ptr(),
+                                      out_keys.data_ptr(),
+                                      None if out_vals is None else out_vals.data_ptr(),
+                                      lens, len(run_len)))
+        return out_keys
 
 
 _plans: dict = {}

@@ -17,6 +17,7 @@
 
 #include "dc.h"
 #include "maxsub_kernels.cuh"
+#include "mg_kernels.cuh"
 #include "sort_kernels.cuh"
 
 namespace {
@@ -112,6 +113,8 @@ struct dc_plan_s {
     dc_maxsub_tuple* ms_tiles = nullptr;
     unsigned int* ms_ticket = nullptr;
     dc_maxsub_result* ms_res = nullptr;
+    // multi-GPU splitter state: bracket packs [64] lo, [64] hi, error flag
+    unsigned long long* mg_state = nullptr;
     // host-buffer (end-to-end) staging
     void* d_stage = nullptr;
     size_t d_stage_bytes = 0;
@@ -262,15 +265,14 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     for (int64_t w = C.tile(); w < n; w *= 2) {
         {
             TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-            dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(cur_k, n, w,
-                                                                            C.tout(), tiles,
-                                                                            split);
+            dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
+                cur_k, dc::PairGeom{0, w, w, n}, C.tout(), tiles, split);
             DC_LAUNCHED(p);
         }
         {
             TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-            k3<<<tiles, C.nt3, nk3_smem_bytes(C, hv), p->stream>>>(cur_k, cur_v, oth_k, oth_v,
-                                                                   split, n, w);
+            k3<<<tiles, C.nt3, nk3_smem_bytes(C, hv), p->stream>>>(
+                cur_k, cur_v, oth_k, oth_v, split, dc::PairGeom{0, w, w, n});
             DC_LAUNCHED(p);
         }
         std::swap(cur_k, oth_k);
@@ -348,6 +350,81 @@ dc_status ensure_stage(dc_plan_t p, size_t bytes) {
         return fail(DC_ERR_OUT_OF_MEMORY, "staging cudaMalloc failed");
     }
     p->d_stage_bytes = bytes;
+    return DC_OK;
+}
+
+
+// a9: local stable G-way merge.  Adjacent runs are merged pairwise, log2(runs)
+// rounds, one NK2 + NK3 launch pair per run pair (pair mode: arbitrary
+// lengths and offsets); ping-pong between the input buffer and the plan
+// scratch, the last round writes the output buffer.
+template <class K, bool V>
+dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* out_k,
+                         uint32_t* out_v, std::vector<int64_t> runs) {
+    int64_t total = 0;
+    for (int64_t r : runs) total += r;
+    if (total > p->n) return fail(DC_ERR_INVALID_ARG, "runs exceed the plan size");
+    dc_status st = ensure_scratch(p, V);
+    if (st != DC_OK) return st;
+    const size_t kb = align_up((size_t)p->n * 4, 256);
+    uint32_t* sk = (uint32_t*)p->scratch;
+    uint32_t* sv = V ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
+    int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
+    constexpr SortCfg C = cfg_for<K, V>();
+    auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
+    static bool attr_done = false;
+    if (!attr_done) {
+        DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        nk3_smem_bytes(C, V)));
+        attr_done = true;
+    }
+    int rounds = 0;
+    for (size_t c = runs.size(); c > 1; c = (c + 1) / 2) ++rounds;
+    if (rounds == 0) rounds = 1;                       // a single run: one copy round
+    uint32_t *cur_k = in_k, *cur_v = in_v;
+    for (int rd = 0; rd < rounds; ++rd) {
+        const bool last = rd == rounds - 1;
+        uint32_t* dst_k = last ? out_k : ((cur_k == in_k) ? sk : in_k);
+        uint32_t* dst_v = last ? out_v : ((cur_k == in_k) ? sv : in_v);
+        std::vector<int64_t> next;
+        int64_t org = 0;
+        for (size_t r = 0; r < runs.size(); r += 2) {
+            const int64_t la = runs[r], lb = (r + 1 < runs.size()) ? runs[r + 1] : 0;
+            if (la + lb > 0) {
+                const dc::PairGeom g{org, la, lb, org + la + lb};
+                const int tiles = (int)num_tiles(la + lb, C.tout());
+                {
+                    TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
+                    dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
+                        cur_k, g, C.tout(), tiles, split);
+                    DC_LAUNCHED(p);
+                }
+                {
+                    TimedScope ts(p, DC_KERNEL_NK3_MERGE);
+                    k3<<<tiles, C.nt3, nk3_smem_bytes(C, V), p->stream>>>(cur_k, cur_v, dst_k,
+                                                                          dst_v, split, g);
+                    DC_LAUNCHED(p);
+                }
+            }
+            next.push_back(la + lb);
+            org += la + lb;
+        }
+        runs.swap(next);
+        cur_k = dst_k;
+        cur_v = dst_v;
+    }
+    return DC_OK;
+}
+
+dc_status ensure_mg_state(dc_plan_t p) {
+    if (p->mg_state) return DC_OK;
+    void* ptr = nullptr;
+    if (cudaMalloc(&ptr, 129 * sizeof(unsigned long long)) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DC_ERR_OUT_OF_MEMORY, "splitter state cudaMalloc failed");
+    }
+    p->mg_state = (unsigned long long*)ptr;
+    DC_CUDA(p, cudaMemsetAsync(p->mg_state + 128, 0, sizeof(unsigned long long), p->stream));
     return DC_OK;
 }
 
@@ -467,6 +544,7 @@ dc_status dc_free(dc_plan_t p) {
     if (p->scratch && p->own_scratch) cudaFree(p->scratch);
     if (p->ms_tiles) cudaFree(p->ms_tiles);
     if (p->d_stage) cudaFree(p->d_stage);
+    if (p->mg_state) cudaFree(p->mg_state);
     delete p;
     return DC_OK;
 }
@@ -598,6 +676,164 @@ dc_status dc_maxsub_combine_async(dc_plan_t p, const dc_maxsub_tuple* d_tuples, 
     return DC_OK;
 }
 
-// Multi-GPU building blocks: implemented in dc_mg.cu.
+// ------------------------------------------------ multi-GPU building blocks
+
+int64_t dc_mg_sendbuf_words(int32_t world, int64_t wcap) {
+    return world < 2 ? 0 : dc::mg_sendbuf_words(world, wcap);
+}
+
+dc_status dc_mg_sample(dc_plan_t p, const uint32_t* d_keys, int64_t n, int64_t stride,
+                       uint32_t* d_samples) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_keys || !d_samples || n < 1 || stride < 1)
+        return fail(DC_ERR_INVALID_ARG, "bad sample arguments");
+    const int64_t cnt = (n + stride - 1) / stride;
+    dc::mg_sample<<<(unsigned)((cnt + 255) / 256), 256, 0, p->stream>>>(d_keys, stride, cnt,
+                                                                       d_samples);
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+dc_status dc_mg_count(dc_plan_t p, dc_key_type kt, const uint32_t* d_keys, int64_t n,
+                      int32_t rank, const uint32_t* d_cand, int64_t per_rank, int64_t stride,
+                      int64_t cands, int64_t* d_counts) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_keys || !d_cand || !d_counts || per_rank < 1 || cands < 1 || cands >= (1LL << 24))
+        return fail(DC_ERR_INVALID_ARG, "bad count arguments");
+    const unsigned grid = (unsigned)((cands + 255) / 256);
+    switch (kt) {
+        case DC_KEY_U32:
+            dc::mg_count<dc::KeyU32><<<grid, 256, 0, p->stream>>>(d_keys, n, rank, d_cand,
+                                                                  per_rank, stride, cands,
+                                                                  d_counts);
+            break;
+        case DC_KEY_I32:
+            dc::mg_count<dc::KeyI32><<<grid, 256, 0, p->stream>>>(d_keys, n, rank, d_cand,
+                                                                  per_rank, stride, cands,
+                                                                  d_counts);
+            break;
+        case DC_KEY_F32:
+            dc::mg_count<dc::KeyF32><<<grid, 256, 0, p->stream>>>(d_keys, n, rank, d_cand,
+                                                                  per_rank, stride, cands,
+                                                                  d_counts);
+            break;
+        default:
+            return fail(DC_ERR_INVALID_ARG, "unknown key type");
+    }
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+dc_status dc_mg_windows(dc_plan_t p, const uint32_t* d_keys, int64_t n, int32_t rank,
+                        int32_t world, const int64_t* d_counts, const int64_t* d_ranks,
+                        int64_t per_rank, int64_t cands, int64_t wcap, uint32_t* d_sendbuf) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_keys || !d_counts || !d_ranks || !d_sendbuf || world < 2 || world > 64 ||
+        rank < 0 || rank >= world || cands < 1 || cands >= (1LL << 24))
+        return fail(DC_ERR_INVALID_ARG, "bad window arguments");
+    st = ensure_mg_state(p);
+    if (st != DC_OK) return st;
+    unsigned long long* lo = p->mg_state;
+    unsigned long long* hi = p->mg_state + 64;
+    DC_CUDA(p, cudaMemsetAsync(lo, 0x00, 64 * sizeof(unsigned long long), p->stream));
+    DC_CUDA(p, cudaMemsetAsync(hi, 0xFF, 64 * sizeof(unsigned long long), p->stream));
+    dc::mg_brackets<<<(unsigned)((cands + 255) / 256), 256, 0, p->stream>>>(d_ranks, cands, world,
+                                                                          n, lo, hi);
+    DC_LAUNCHED(p);
+    dc::mg_windows<<<world - 1, 256, 0, p->stream>>>(d_keys, n, rank, world, n, d_counts, d_ranks,
+                                                      per_rank, wcap, lo, hi, d_sendbuf,
+                                                      (int*)(p->mg_state + 128));
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+dc_status dc_mg_split_matrix(dc_plan_t p, dc_key_type kt, const uint32_t* d_gathered,
+                             int32_t world, int64_t shard_n, int64_t wcap, int64_t* d_cmat) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_gathered || !d_cmat || world < 2 || world > 64 || wcap < 1)
+        return fail(DC_ERR_INVALID_ARG, "bad split-matrix arguments");
+    const size_t smem = (size_t)world * wcap * 4;
+    if (smem > 200 * 1024) return fail(DC_ERR_INVALID_ARG, "world * wcap too large");
+    switch (kt) {
+        case DC_KEY_U32: {
+            auto* k = dc::mg_split_matrix<dc::KeyU32>;
+            DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)smem));
+            k<<<world - 1, 64, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
+            break;
+        }
+        case DC_KEY_I32: {
+            auto* k = dc::mg_split_matrix<dc::KeyI32>;
+            DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)smem));
+            k<<<world - 1, 64, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
+            break;
+        }
+        case DC_KEY_F32: {
+            auto* k = dc::mg_split_matrix<dc::KeyF32>;
+            DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)smem));
+            k<<<world - 1, 64, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
+            break;
+        }
+        default:
+            return fail(DC_ERR_INVALID_ARG, "unknown key type");
+    }
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+dc_status dc_mg_error(dc_plan_t p, int32_t* h_err) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!h_err) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    *h_err = 0;
+    if (!p->mg_state) return DC_OK;
+    int v = 0;
+    DC_CUDA(p, cudaMemcpyAsync(&v, p->mg_state + 128, sizeof(int), cudaMemcpyDeviceToHost,
+                               p->stream));
+    DC_CUDA(p, cudaStreamSynchronize(p->stream));
+    *h_err = v;
+    return DC_OK;
+}
+
+dc_status dc_mg_merge_runs(dc_plan_t p, dc_key_type kt, uint32_t* d_in_keys, uint32_t* d_in_vals,
+                           uint32_t* d_out_keys, uint32_t* d_out_vals, const int64_t* h_run_len,
+                           int32_t runs) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_in_keys || !d_out_keys || !h_run_len || runs < 1 ||
+        (d_in_vals == nullptr) != (d_out_vals == nullptr))
+        return fail(DC_ERR_INVALID_ARG, "bad merge arguments");
+    if (!aligned16(d_in_keys) || !aligned16(d_out_keys) ||
+        (d_in_vals && (!aligned16(d_in_vals) || !aligned16(d_out_vals))))
+        return fail(DC_ERR_INVALID_ARG, "buffers must be 16-byte aligned");
+    std::vector<int64_t> lens(h_run_len, h_run_len + runs);
+    for (int64_t l : lens)
+        if (l < 0) return fail(DC_ERR_INVALID_ARG, "negative run length");
+    const bool v = d_in_vals != nullptr;
+    switch (kt) {
+        case DC_KEY_U32:
+            return v ? mg_merge_typed<dc::KeyU32, true>(p, d_in_keys, d_in_vals, d_out_keys,
+                                                        d_out_vals, lens)
+                     : mg_merge_typed<dc::KeyU32, false>(p, d_in_keys, nullptr, d_out_keys,
+                                                         nullptr, lens);
+        case DC_KEY_I32:
+            return v ? mg_merge_typed<dc::KeyI32, true>(p, d_in_keys, d_in_vals, d_out_keys,
+                                                        d_out_vals, lens)
+                     : mg_merge_typed<dc::KeyI32, false>(p, d_in_keys, nullptr, d_out_keys,
+                                                         nullptr, lens);
+        case DC_KEY_F32:
+            return v ? mg_merge_typed<dc::KeyF32, true>(p, d_in_keys, d_in_vals, d_out_keys,
+                                                        d_out_vals, lens)
+                     : mg_merge_typed<dc::KeyF32, false>(p, d_in_keys, nullptr, d_out_keys,
+                                                         nullptr, lens);
+    }
+    return fail(DC_ERR_INVALID_ARG, "unknown key type");
+}
 
 }  // extern "C"

@@ -246,18 +246,24 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
-// Store words [0, count) of a shared tile to global dst (16-byte aligned):
-// the 16-byte body by one bulk copy issued by thread 0, the < 4-word tail by
-// plain stores.  Caller: every thread has written its part, then
-// fence_proxy_async_smem(); __syncthreads().
-__device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uint32_t* s,
+// Store a shared tile to global memory.  Element e of the tile sits at shared
+// word e + h and goes to dst[e], where h = (dst - 16-byte-aligned base) in
+// words, so both sides of the bulk copy are congruent mod 16 bytes: the
+// 16-byte body leaves by one TMA bulk copy issued by thread 0, the < 4-word
+// head and tail by plain stores.  Caller: every thread has written its part,
+// then fence_proxy_async_smem(); __syncthreads().
+__device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uint32_t* s, int h,
                                            int count) {
-    const int body = count & ~3;
+    const int head = min(count, (4 - h) & 3);              // words before the aligned body
+    const int body = (count - head) & ~3;
     if (threadIdx.x == 0 && body > 0) {
-        bulk_s2g(dst, smem_addr(s), 4u * body);
+        bulk_s2g(dst + head, smem_addr(s + h + head), 4u * body);
         bulk_commit_and_wait_read();
     }
-    if ((int)threadIdx.x < count - body) dst[body + threadIdx.x] = s[body + threadIdx.x];
+    const int t = threadIdx.x;
+    if (t < head) dst[t] = s[h + t];
+    const int tail0 = head + body;
+    if (t < count - tail0) dst[tail0 + t] = s[h + tail0 + t];
 }
 
 // ------------------------------------------------------------------ NK1
@@ -352,78 +358,77 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     }
     fence_proxy_async_smem();
     __syncthreads();
-    store_tile(out_k + base, sk, count);
-    if (V) store_tile(out_v + base, si, count);
+    store_tile(out_k + base, sk, 0, count);
+    if (V) store_tile(out_v + base, si, 0, count);
 }
 
 // ------------------------------------------------------------------ NK2
-// Co-rank of the first output of every merge tile at run width w: tile j
-// covers merged positions [j*TOUT, (j+1)*TOUT); its pair p starts at s = p*2w
-// (TOUT divides 2w, so a tile never straddles two pairs).
+// Geometry of one merge level over [org, end) of a buffer: pairs of adjacent
+// runs (A of width wa, then B of width wb) with stride wa + wb starting at
+// org; the last pair may be short.  The breadth-first sort uses org = 0 and
+// wa = wb = w; the local G-way merge of the multi-GPU path merges one pair of
+// arbitrary lengths at an arbitrary offset per launch.  Indices are absolute
+// (the buffer base stays 16-byte aligned for TMA).
+struct PairGeom {
+    long long org, wa, wb, end;
+    // pair containing merged position d0 (relative to org): absolute start s
+    __device__ __forceinline__ void pair_of(long long d0, long long& s, long long& a_len,
+                                            long long& b_len) const {
+        s = org + (d0 / (wa + wb)) * (wa + wb);
+        a_len = min(wa, end - s);
+        b_len = max(0LL, min(wb, end - s - a_len));
+    }
+};
+
+// Co-rank of the first output of every merge tile: tile j covers merged
+// positions [j*tout, (j+1)*tout) (tout divides wa + wb, or there is one pair).
 template <class K>
-__global__ void nk2_partition(const uint32_t* __restrict__ src, long long n, long long w,
-                              int tout, int num_tiles, int* __restrict__ split) {
+__global__ void nk2_partition(const uint32_t* __restrict__ src, PairGeom g, int tout,
+                              int num_tiles, int* __restrict__ split) {
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= num_tiles) return;
     const long long d0 = (long long)j * tout;
-    const long long s = (d0 / (2 * w)) * (2 * w);
-    const long long a_len = min(w, n - s);
-    const long long b_len = max(0LL, min(w, n - s - w));
-    split[j] = (int)corank_global<K>(src + s, a_len, src + s + a_len, b_len, d0 - s);
+    long long s, a_len, b_len;
+    g.pair_of(d0, s, a_len, b_len);
+    split[j] = (int)corank_global<K>(src + s, a_len, src + s + a_len, b_len, d0 - (s - g.org));
 }
 
 // ------------------------------------------------------------------ NK3
 // Stage global elements [g0, g1) (any alignment) into shared memory at word
 // offset `off` + (g0 & 3): TMA copies the 16-byte-aligned superset that lies
 // below n4 = n & ~3; the caller's threads load the rest (< 4 words past n4).
-// Returns the bytes the TMA will deliver.
-__device__ __forceinline__ uint32_t stage_piece(const uint32_t* __restrict__ g, long long g0,
-                                                long long g1, long long n4, uint32_t dst_off,
-                                                uint32_t sbase, uint32_t bar) {
+__device__ __forceinline__ uint32_t piece_bytes(long long g0, long long g1, long long n4) {
     const long long al0 = g0 & ~3LL;
     long long al1 = (g1 + 3) & ~3LL;
     if (al1 > n4) al1 = n4;
-    const uint32_t bytes = al1 > al0 ? (uint32_t)(4 * (al1 - al0)) : 0u;
-    if (bytes) bulk_g2s(sbase + 4u * dst_off, g + al0, bytes, bar);
-    return bytes;
+    return al1 > al0 ? (uint32_t)(4 * (al1 - al0)) : 0u;
+}
+__device__ __forceinline__ void stage_piece(const uint32_t* __restrict__ g, long long g0,
+                                            long long g1, long long n4, uint32_t dst_off,
+                                            uint32_t sbase, uint32_t bar) {
+    const uint32_t bytes = piece_bytes(g0, g1, n4);
+    if (bytes) bulk_g2s(sbase + 4u * dst_off, g + (g0 & ~3LL), bytes, bar);
 }
 
-// One output tile of TOUT = NT*IT merged keys per CTA.  The A and B pieces
-// that feed the tile (known from the co-ranks) are staged in shared memory
-// by TMA, each thread finds its own IT-output diagonal there and merges
-// serially, and the tile leaves by one TMA bulk store.
+// One output tile of the merge of A = src[a0, a0+na) and B = src[b0, b0+nb)
+// (total = na + nb <= NT*IT outputs) written to dst[o0, o0+total).  The
+// pieces are staged in shared memory by TMA, each thread finds its own
+// IT-output diagonal there and merges serially, and the tile leaves by one
+// TMA bulk store.  n bounds the readable part of src.
 template <int NT, int IT, class K, bool V>
-__global__ void __launch_bounds__(NT)
-nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
-          uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v,
-          const int* __restrict__ split, long long n, long long w) {
-    static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
+__device__ __forceinline__ void merge_tile(const uint32_t* __restrict__ src_k,
+                                           const uint32_t* __restrict__ src_v,
+                                           uint32_t* __restrict__ dst_k,
+                                           uint32_t* __restrict__ dst_v, long long n,
+                                           long long a0, int na, long long b0, int nb,
+                                           long long o0, uint32_t* sk, uint32_t* sv,
+                                           uint32_t BAR) {
     constexpr int TOUT = NT * IT;
-    static_assert(TOUT % 4 == 0, "tile must be a whole number of 16-byte chunks");
     constexpr int TW = tile_words(TOUT, IT + 16);
-    extern __shared__ __align__(16) uint32_t smem[];
-    uint32_t* sk = smem;          // [TW]: A piece, B piece; then the merged tile
-    uint32_t* sv = smem + TW;     // [TW]: values, same layout (V)
-    __shared__ __align__(8) uint64_t bar;
-    const uint32_t SK = smem_addr(sk), SV = smem_addr(sv);
-    const uint32_t BAR = smem_addr(&bar);
     constexpr uint32_t SV_OFF = TW * 4;
-
+    const uint32_t SK = smem_addr(sk), SV = smem_addr(sv);
     const int tid = threadIdx.x;
-    const int j = blockIdx.x;
-    const long long d0 = (long long)j * TOUT;
-    const long long s = (d0 / (2 * w)) * (2 * w);
-    const long long a_len = min(w, n - s);
-    const long long b_len = max(0LL, min(w, n - s - w));
-    const long long dd0 = d0 - s;
-    const long long dd1 = min(dd0 + TOUT, a_len + b_len);
-    const int i0 = split[j];
-    const int i1 = (dd1 == a_len + b_len) ? (int)a_len : split[j + 1];
-    const int na = i1 - i0;
-    const int total = (int)(dd1 - dd0);
-    const int nb = total - na;
-    const long long a0 = s + i0;                       // A piece: global [a0, a0+na)
-    const long long b0 = s + a_len + (dd0 - i0);       // B piece: global [b0, b0+nb)
+    const int total = na + nb;
     const int fa = (int)(a0 & 3), fb = (int)(b0 & 3);
     const int ob = (fa + na + 1 + 3) & ~3;             // B region word offset (16 B aligned)
     const uint32_t A = SK + 4u * fa, B = SK + 4u * (ob + fb);
@@ -431,14 +436,7 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
 
     if (tid == 0) {
         mbar_init(BAR, 1);
-        uint32_t bytes = 0;
-        // expect_tx must precede the copies' completion: arm with the exact sum.
-        const long long al0a = a0 & ~3LL, al0b = b0 & ~3LL;
-        long long al1a = (a0 + na + 3) & ~3LL, al1b = (b0 + nb + 3) & ~3LL;
-        if (al1a > n4) al1a = n4;
-        if (al1b > n4) al1b = n4;
-        bytes += al1a > al0a ? (uint32_t)(4 * (al1a - al0a)) : 0u;
-        bytes += al1b > al0b ? (uint32_t)(4 * (al1b - al0b)) : 0u;
+        const uint32_t bytes = piece_bytes(a0, a0 + na, n4) + piece_bytes(b0, b0 + nb, n4);
         mbar_arrive_expect_tx(BAR, bytes * (V ? 2 : 1));
         stage_piece(src_k, a0, a0 + na, n4, 0, SK, BAR);
         stage_piece(src_k, b0, b0 + nb, n4, ob, SK, BAR);
@@ -475,17 +473,45 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
         }
     }
     __syncthreads();
+    const int h = (int)(o0 & 3);                       // output alignment shift
     if (diag < total) {
 #pragma unroll
         for (int q = 0; q < IT; ++q) {
-            sk[diag + q] = k[q];
-            if (V) sv[diag + q] = vv[q];
+            sk[h + diag + q] = k[q];
+            if (V) sv[h + diag + q] = vv[q];
         }
     }
     fence_proxy_async_smem();
     __syncthreads();
-    store_tile(dst_k + d0, sk, total);
-    if (V) store_tile(dst_v + d0, sv, total);
+    store_tile(dst_k + o0, sk, h, total);
+    if (V) store_tile(dst_v + o0, sv, h, total);
+}
+
+// One merge level (Alg 7 lines 3-5): CTA j produces merged positions
+// [j*TOUT, (j+1)*TOUT) of the pair that contains them, in place in dst.
+template <int NT, int IT, class K, bool V>
+__global__ void __launch_bounds__(NT)
+nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
+          uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v,
+          const int* __restrict__ split, PairGeom g) {
+    static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
+    constexpr int TOUT = NT * IT;
+    constexpr int TW = tile_words(TOUT, IT + 16);
+    extern __shared__ __align__(16) uint32_t smem[];
+    __shared__ __align__(8) uint64_t bar;
+    const int j = blockIdx.x;
+    const long long d0 = (long long)j * TOUT;
+    long long s, a_len, b_len;
+    g.pair_of(d0, s, a_len, b_len);
+    const long long dd0 = d0 - (s - g.org);
+    const long long dd1 = min(dd0 + TOUT, a_len + b_len);
+    const int i0 = split[j];
+    const int i1 = (dd1 == a_len + b_len) ? (int)a_len : split[j + 1];
+    const int na = i1 - i0;
+    const int nb = (int)(dd1 - dd0) - na;
+    merge_tile<NT, IT, K, V>(src_k, src_v, dst_k, dst_v, g.end, s + i0, na,
+                             s + a_len + (dd0 - i0), nb, g.org + d0, smem, smem + TW,
+                             smem_addr(&bar));
 }
 
 }  // namespace dc

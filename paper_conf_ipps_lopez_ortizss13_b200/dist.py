@@ -1,0 +1,322 @@
+"""Multi-GPU path: the top log2(G) levels of the breadth-first sort (rows a7-a10).
+
+One process per GPU (torchrun); rank r holds the shard of global positions
+[r*m, (r+1)*m).  Levels below log2(G) are independent subproblems: each rank
+sorts its shard with the single-GPU path (NK1 + NK2/NK3 levels).  The top
+log2(G) levels become one exchange step:
+
+  a7  exact splitters: samples -> all-gather -> composite counts (kernel) ->
+      all-reduce -> brackets + windows (kernels) -> all-gather -> split matrix
+      (kernel); composite order (key, rank, position) = the global stable order;
+  a8  all-to-all of the key (and value) ranges over NVLink (NCCL);
+  a9  local stable G-way merge of the received runs (kernels);
+  a10 max-subarray: per-rank summary tuple -> all-gather -> ordered combine.
+
+Collectives go through a tiny interface (:class:`Comm`): :class:`TorchComm`
+wraps a torch.distributed process group (NCCL on GPUs; gloo in the CPU tests)
+and :class:`LoopbackComm` runs G virtual ranks as threads in one process on
+one GPU (the 1-GPU test of the whole protocol).  Every step on the data runs
+in the library's kernels; this module only moves tensors between them.
+"""
+from __future__ import annotations
+
+import threading
+from dataclasses import dataclass
+
+import torch
+
+from . import Plan, _KEY_NAMES
+
+DEFAULT_STRIDE = 4096     # sample stride S: candidates = G*ceil(m/S); windows < S keys
+
+
+# ------------------------------------------------------------------- comms
+
+class Comm:
+    """Collectives used by the protocol (all ranks call them in the same order)."""
+
+    rank: int
+    world: int
+
+    def all_gather(self, t: torch.Tensor) -> torch.Tensor:  # [world * t.numel()], rank order
+        raise NotImplementedError
+
+    def all_reduce_sum_(self, t: torch.Tensor) -> None:
+        raise NotImplementedError
+
+    def all_to_all(self, send: torch.Tensor, send_splits: list[int],
+                   recv_splits: list[int]) -> torch.Tensor:
+        raise NotImplementedError
+
+    def barrier(self) -> None:
+        raise NotImplementedError
+
+
+class TorchComm(Comm):
+    """torch.distributed process group (NCCL over NVLink on B200 boxes)."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+
+        self.dist = dist
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+
+    def all_gather(self, t):
+        t = t.contiguous()
+        out = torch.empty(self.world * t.numel(), dtype=t.dtype, device=t.device)
+        self.dist.all_gather_into_tensor(out, t.view(-1), group=self.group)
+        return out
+
+    def all_reduce_sum_(self, t):
+        self.dist.all_reduce(t, op=self.dist.ReduceOp.SUM, group=self.group)
+
+    def all_to_all(self, send, send_splits, recv_splits):
+        out = torch.empty(sum(recv_splits), dtype=send.dtype, device=send.device)
+        self.dist.all_to_all_single(out, send, recv_splits, send_splits, group=self.group)
+        return out
+
+    def barrier(self):
+        self.dist.barrier(group=self.group)
+
+
+class _LoopbackState:
+    def __init__(self, world):
+        self.world = world
+        self.barrier = threading.Barrier(world)
+        self.slots = [None] * world
+
+
+class LoopbackComm(Comm):
+    """G virtual ranks as threads of one process sharing one GPU (testing)."""
+
+    def __init__(self, state: _LoopbackState, rank: int):
+        self.s = state
+        self.rank = rank
+        self.world = state.world
+
+    def _exchange(self, obj):
+        if torch.cuda.is_available():
+            torch.cuda.synchronize()
+        self.s.slots[self.rank] = obj
+        self.s.barrier.wait()
+        everyone = list(self.s.slots)
+        self.s.barrier.wait()
+        return everyone
+
+    def all_gather(self, t):
+        return torch.cat([x.reshape(-1) for x in self._exchange(t.contiguous())])
+
+    def all_reduce_sum_(self, t):
+        parts = self._exchange(t.clone())
+        acc = parts[0].clone()
+        for x in parts[1:]:
+            acc += x
+        t.copy_(acc)
+
+    def all_to_all(self, send, send_splits, recv_splits):
+        pieces = self._exchange(list(torch.split(send, send_splits)))
+        out = torch.cat([pieces[r][self.rank] for r in range(self.world)])
+        assert out.numel() == sum(recv_splits)
+        return out
+
+    def barrier(self):
+        self._exchange(None)
+
+
+def run_loopback(world: int, fn):
+    """Run fn(comm) for `world` virtual ranks (threads); returns the results."""
+    state = _LoopbackState(world)
+    results, errors = [None] * world, []
+
+    def body(r):
+        try:
+            results[r] = fn(LoopbackComm(state, r))
+        except BaseException as e:   # noqa: BLE001 - surfaced below
+            errors.append(e)
+            state.barrier.abort()
+
+    threads = [threading.Thread(target=body, args=(r,)) for r in range(world)]
+    for t in threads:
+        t.start()
+    for t in threads:
+        t.join()
+    if errors:
+        raise errors[0]
+    return results
+
+
+# -------------------------------------------------------------- local ops
+
+class DcOps:
+    """Per-rank device steps of the protocol, all in libdcb200 kernels."""
+
+    def __init__(self, n: int):
+        self.plan = Plan(n)
+
+    def sort_(self, keys, vals, key_type):
+        self.plan.sort_(keys, vals, key_type=key_type)
+
+    def sample(self, keys, stride):
+        return self.plan.mg_sample(keys, stride)
+
+    def count(self, keys, rank, cand, per_rank, stride, key_type):
+        return self.plan.mg_count(keys, rank, cand, per_rank, stride, key_type=key_type)
+
+    def windows(self, keys, rank, world, counts, ranks, per_rank, wcap):
+        return self.plan.mg_windows(keys, rank, world, counts, ranks, per_rank, wcap)
+
+    def split_matrix(self, gathered, world, shard_n, wcap, key_type):
+        return self.plan.mg_split_matrix(gathered, world, shard_n, wcap, key_type)
+
+    def check(self):
+        if self.plan.mg_error():
+            raise RuntimeError("splitter window overflow (unsorted shard?)")
+
+    def merge_runs(self, in_k, in_v, out_k, out_v, runs, key_type):
+        self.plan.mg_merge_runs(in_k, in_v, out_k, out_v, runs, key_type=key_type)
+
+    def maxsub_tuple(self, x, offset):
+        out = torch.empty(8, dtype=torch.int64, device=x.device)
+        return self.plan.max_subarray_tuple_async(x, out, index_offset=offset)
+
+    def maxsub_combine(self, tuples):
+        out = torch.empty(3, dtype=torch.int64, device=tuples.device)
+        return self.plan.maxsub_combine_async(tuples, out)
+
+    def launches(self) -> int:
+        return self.plan.launch_count()
+
+
+# ---------------------------------------------------------------- protocol
+
+@dataclass
+class ExchangeInfo:
+    cmat: list            # world x (world+1): c[r][d]
+    send_splits: list
+    recv_splits: list
+
+
+def split_sizes(cmat, rank: int):
+    """Send / receive counts of `rank` from the split matrix c[r][d] (host logic):
+    rank r sends [c[r][d], c[r][d+1]) to rank d and receives [c[s][r], c[s][r+1])
+    from every rank s."""
+    world = len(cmat)
+    send = [int(cmat[rank][d + 1] - cmat[rank][d]) for d in range(world)]
+    recv = [int(cmat[s][rank + 1] - cmat[s][rank]) for s in range(world)]
+    return send, recv
+
+
+def sort_(keys: torch.Tensor, vals: torch.Tensor | None = None, comm: Comm | None = None,
+          key_type: str = "u32", stride: int = DEFAULT_STRIDE, ops=None) -> ExchangeInfo | None:
+    """Distributed stable sort, in place.
+
+    On entry rank r's ``keys`` (and ``vals``) hold global positions
+    [r*m, (r+1)*m) of the input (every rank the same m); on exit they hold
+    global positions [r*m, (r+1)*m) of the stable sorted order.
+    """
+    if key_type not in _KEY_NAMES:
+        raise ValueError(f"unknown key type {key_type!r}")
+    m = keys.numel()
+    ops = ops or DcOps(m)
+    ops.sort_(keys, vals, key_type)                                  # levels >= log2 G
+    if comm is None or comm.world == 1:
+        return None
+    G, me = comm.world, comm.rank
+    wcap = stride
+    q = -(-m // stride)
+    samples = ops.sample(keys, stride)                               # a7
+    cand = comm.all_gather(samples)                                  # C1: all-gather
+    counts = ops.count(keys, me, cand, q, stride, key_type)
+    granks = counts.clone()
+    comm.all_reduce_sum_(granks)                                     # C2: all-reduce
+    sendbuf = ops.windows(keys, me, G, counts, granks, q, wcap)
+    gathered = comm.all_gather(sendbuf)                              # C3: all-gather
+    cmat_t = ops.split_matrix(gathered, G, m, wcap, key_type)
+    ops.check()
+    cmat = cmat_t.cpu().tolist()                                     # the one host sync
+    send, recv = split_sizes(cmat, me)
+    rk = comm.all_to_all(keys, send, recv)                           # a8: all-to-all
+    rv = comm.all_to_all(vals, send, recv) if vals is not None else None
+    ops.merge_runs(rk, rv, keys, vals, recv, key_type)               # a9: local G-way merge
+    return ExchangeInfo(cmat, send, recv)
+
+
+def max_subarray(x: torch.Tensor, comm: Comm | None = None, ops=None):
+    """(sum, start, end) of the whole distributed array; rank r holds the r-th
+    consecutive piece (pieces may differ in length).  Same answer on every rank."""
+    ops = ops or DcOps(x.numel())
+    if comm is None or comm.world == 1:
+        t = ops.maxsub_tuple(x, 0)
+        return tuple(int(v) for v in ops.maxsub_combine(t.view(1, 8)).cpu().tolist())
+    sizes = comm.all_gather(torch.tensor([x.numel()], dtype=torch.int64, device=x.device))
+    offset = int(sizes[:comm.rank].sum().item())
+    t = ops.maxsub_tuple(x, offset)                                  # a10: local summary
+    allt = comm.all_gather(t)                                        # all-gather G tuples
+    res = ops.maxsub_combine(allt.view(comm.world, 8))               # ordered combine
+    return tuple(int(v) for v in res.cpu().tolist())
+
+
+# ------------------------------------------------------------ N>1 bench
+
+def bench_main(args, wl, workloads, metric):
+    """bench.py under torchrun: 2^30 keys sharded over WORLD_SIZE GPUs (configs[4])."""
+    import json
+    import os
+    import statistics
+
+    import torch.distributed as tdist
+
+    import dcgen
+
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    comm = TorchComm()
+    G, me = comm.world, comm.rank
+    desc, n_total, kind = workloads[wl]
+    if n_total % G:
+        raise SystemExit("n must be divisible by the number of GPUs")
+    m = n_total // G
+    dev = torch.device("cuda", local)
+    pristine = dcgen.sort_keys(n_total, args.dist, seed=5, start=me * m, count=m, device=dev)
+    keys = torch.empty_like(pristine)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    ops = DcOps(m)
+    stream = torch.cuda.current_stream(dev)
+    times = []
+    l0 = None
+    for i in range(args.warmup + args.steps):
+        keys.copy_(pristine)
+        flush.zero_()
+        if i == args.warmup:
+            l0 = ops.launches()
+        comm.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        sort_(keys, None, comm, "u32", ops=ops)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if i >= args.warmup:
+            t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+            tdist.all_reduce(t, op=tdist.ReduceOp.MAX)                # max over ranks
+            times.append(float(t.item()))
+    launches = ops.launches() - l0
+    ok = bool((keys[1:].to(torch.int64) & 0xFFFFFFFF >= keys[:-1].to(torch.int64) & 0xFFFFFFFF)
+              .all())
+    ms = statistics.mean(times)
+    if me == 0:
+        print(json.dumps({
+            "metric": metric, "value": n_total / (ms / 1e3), "unit": "keys/s", "n_gpus": G,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic (counter-based splitmix64)",
+            "config": {"workload": wl, "description": desc, "n": n_total, "per_gpu": m,
+                       "dist": args.dist, "parallelism": f"key-range sharding x{G}",
+                       "l2": "flushed before every step (512 MiB write)",
+                       "local_sorted_check": ok},
+            "gpu_launches": launches, "e2e": None, "cpu_baseline": None,
+        }), flush=True)
+    tdist.destroy_process_group()
