@@ -96,33 +96,42 @@ class LoopbackComm(Comm):
         self.rank = rank
         self.world = state.world
 
-    def _exchange(self, obj):
-        if torch.cuda.is_available():
+    def _exchange(self, obj, consume):
+        """Publish obj, then consume(everyone's objs) while all ranks still hold
+        their inputs unchanged (between the two barriers)."""
+        cuda = torch.cuda.is_available()
+        if cuda:
             torch.cuda.synchronize()
         self.s.slots[self.rank] = obj
         self.s.barrier.wait()
-        everyone = list(self.s.slots)
+        out = consume(list(self.s.slots))
+        if cuda:
+            torch.cuda.synchronize()
         self.s.barrier.wait()
-        return everyone
+        return out
 
     def all_gather(self, t):
-        return torch.cat([x.reshape(-1) for x in self._exchange(t.contiguous())])
+        return self._exchange(t.contiguous(),
+                              lambda xs: torch.cat([x.reshape(-1) for x in xs]))
 
     def all_reduce_sum_(self, t):
-        parts = self._exchange(t.clone())
-        acc = parts[0].clone()
-        for x in parts[1:]:
-            acc += x
-        t.copy_(acc)
+        def add(xs):
+            acc = xs[0].clone()
+            for x in xs[1:]:
+                acc += x
+            return acc
+
+        t.copy_(self._exchange(t, add))
 
     def all_to_all(self, send, send_splits, recv_splits):
-        pieces = self._exchange(list(torch.split(send, send_splits)))
-        out = torch.cat([pieces[r][self.rank] for r in range(self.world)])
+        pieces = list(torch.split(send, send_splits))
+        out = self._exchange(pieces, lambda ps: torch.cat([ps[r][self.rank]
+                                                           for r in range(self.world)]))
         assert out.numel() == sum(recv_splits)
         return out
 
     def barrier(self):
-        self._exchange(None)
+        self._exchange(None, lambda xs: None)
 
 
 def run_loopback(world: int, fn):
