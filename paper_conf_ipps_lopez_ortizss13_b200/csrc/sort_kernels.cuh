@@ -266,6 +266,65 @@ __device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uin
     if (t < count - tail0) dst[tail0 + t] = s[h + tail0 + t];
 }
 
+// ------------------------------------------- keys-only bitonic merge levels
+// Keys-only u32/i32 (equal keys are identical bit patterns, so which copy of
+// an equal key is emitted first is unobservable): every B run is stored
+// DESCENDING after its ascending A run, so each pair is a bitonic sequence.
+// A thread merges upward from the front of A and downward from the end of
+// the pair (B's smallest).  When one run is exhausted, its pointer walks
+// into the other run from that run's LARGEST end, so the value it reads is
+// >= every element still pending and the plain comparison "b < a" keeps
+// selecting the right side: no bounds checks, one tracked pointer.
+template <int NT, int IT, class K>
+__device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t* sk) {
+    constexpr int TILE = NT * IT;
+    const int tid = threadIdx.x;
+    const uint32_t SK = smem_addr(sk);
+#pragma unroll 1
+    for (int w = IT; w < TILE; w *= 2) {
+        __syncthreads();
+        {   // write this thread's IT ascending keys: A runs ascending, B runs descending
+            const int pos = tid * IT;
+            const int r = pos / w;                        // run index at width w
+            const int o = pos - r * w;                    // offset inside the run
+            const int pr = (r >> 1) * (2 * w);            // pair start
+            if ((r & 1) == 0) {
+#pragma unroll
+                for (int j = 0; j < IT; ++j) sk[pr + o + j] = k[j];
+            } else {
+#pragma unroll
+                for (int j = 0; j < IT; ++j) sk[pr + 2 * w - 1 - o - j] = k[j];
+            }
+        }
+        __syncthreads();
+        const int tpg = (2 * w) / IT;                     // threads per merged pair
+        const int s = (tid / tpg) * (2 * w);              // pair start
+        const int diag = (tid % tpg) * IT;
+        // co-rank: A[m] at s + m, B[diag-1-m] at s + 2w - 1 - (diag-1-m) = s + 2w - diag + m
+        const uint32_t Ab = SK + 4u * s, Bb = SK + 4u * (s + 2 * w - diag);
+        int lo = max(0, diag - w), hi = min(diag, w);
+        while (lo < hi) {
+            const int m = (lo + hi) >> 1;
+            if (!K::lt(lds(Bb + 4u * m), lds(Ab + 4u * m))) lo = m + 1;
+            else hi = m;
+        }
+        // heads: A[lo] ascending pointer, B[diag-lo] at s + 2w - 1 - (diag - lo), descending
+        uint32_t ai = Ab + 4u * lo;
+        const uint32_t bi0 = SK + 4u * (s + 2 * w - 1 - (diag - lo));
+        const uint32_t D = ai - bi0;                      // ai - bi grows by 4 per output
+        uint32_t a = lds(ai), b = lds(bi0);
+#pragma unroll
+        for (int j = 0; j < IT; ++j) {
+            const bool p = K::lt(b, a);                   // take B
+            k[j] = p ? b : a;
+            if (!p) ai += 4u;
+            const uint32_t bi = ai - D - 4u * (j + 1);
+            const uint32_t v = lds(p ? bi : ai);
+            if (p) b = v; else a = v;
+        }
+    }
+}
+
 // ------------------------------------------------------------------ NK1
 // One CTA sorts one tile of TILE = NT*IT keys (the last tile may be partial:
 // it is padded with K::kPad, which sorts after every real key because every
@@ -327,25 +386,29 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     thread_sort<K, IT, V>(k, ix);
 
     // ---- 3. shared-memory merge levels: run width w -> 2w
+    if constexpr (!V && !K::kNeedStable) {
+        merge_levels_bitonic<NT, IT, K>(k, sk);
+    } else {
 #pragma unroll 1
-    for (int w = IT; w < TILE; w *= 2) {
-        __syncthreads();
+        for (int w = IT; w < TILE; w *= 2) {
+            __syncthreads();
 #pragma unroll
-        for (int j = 0; j < IT; ++j) {
-            sk[tid * IT + j] = k[j];
-            if (V) si[tid * IT + j] = ix[j];
-        }
-        __syncthreads();
-        const int tpg = (2 * w) / IT;            // threads per merged pair
-        const int s = (tid / tpg) * (2 * w);     // pair start
-        const int diag = (tid % tpg) * IT;
-        const uint32_t A = SK + 4u * s, B = A + 4u * w;
-        const int i = corank_smem<K>(A, w, B, w, diag);
-        uint32_t src[IT];
-        serial_merge<K, IT, V>(A + 4u * i, B, B + 4u * (diag - i), B + 4u * w, k, src);
-        if (V) {
+            for (int j = 0; j < IT; ++j) {
+                sk[tid * IT + j] = k[j];
+                if (V) si[tid * IT + j] = ix[j];
+            }
+            __syncthreads();
+            const int tpg = (2 * w) / IT;            // threads per merged pair
+            const int s = (tid / tpg) * (2 * w);     // pair start
+            const int diag = (tid % tpg) * IT;
+            const uint32_t A = SK + 4u * s, B = A + 4u * w;
+            const int i = corank_smem<K>(A, w, B, w, diag);
+            uint32_t src[IT];
+            serial_merge<K, IT, V>(A + 4u * i, B, B + 4u * (diag - i), B + 4u * w, k, src);
+            if (V) {
 #pragma unroll
-            for (int j = 0; j < IT; ++j) ix[j] = lds(src[j] + SI_OFF);
+                for (int j = 0; j < IT; ++j) ix[j] = lds(src[j] + SI_OFF);
+            }
         }
     }
 
