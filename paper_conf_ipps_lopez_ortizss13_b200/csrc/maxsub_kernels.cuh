@@ -194,17 +194,30 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
         MsFold f;
         f.init();
         if (cbeg + C <= n) {
+            // batches of 32 elements (8 x 128-bit loads in flight), the next
+            // batch's loads issued before the current batch is folded
+            constexpr int B4 = 8;
+            static_assert(C % (4 * B4) == 0, "chunk must be whole batches");
             const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
-            int4 v[C / 4];
+            int4 v[B4], nv[B4];
 #pragma unroll
-            for (int q = 0; q < C / 4; ++q) v[q] = __ldg(p4 + q);
-            const int i0 = tid * C;                // tile-local index
+            for (int q = 0; q < B4; ++q) v[q] = __ldg(p4 + q);
+#pragma unroll 1
+            for (int bt = 0; bt < C / (4 * B4); ++bt) {
+                if (bt + 1 < C / (4 * B4)) {
 #pragma unroll
-            for (int q = 0; q < C / 4; ++q) {
-                f.step(v[q].x, i0 + 4 * q);
-                f.step(v[q].y, i0 + 4 * q + 1);
-                f.step(v[q].z, i0 + 4 * q + 2);
-                f.step(v[q].w, i0 + 4 * q + 3);
+                    for (int q = 0; q < B4; ++q) nv[q] = __ldg(p4 + (bt + 1) * B4 + q);
+                }
+                const int i0 = tid * C + bt * 4 * B4;   // tile-local index
+#pragma unroll
+                for (int q = 0; q < B4; ++q) {
+                    f.step(v[q].x, i0 + 4 * q);
+                    f.step(v[q].y, i0 + 4 * q + 1);
+                    f.step(v[q].z, i0 + 4 * q + 2);
+                    f.step(v[q].w, i0 + 4 * q + 3);
+                }
+#pragma unroll
+                for (int q = 0; q < B4; ++q) v[q] = nv[q];
             }
         } else {
             for (long long e = cbeg; e < n && e < cbeg + C; ++e) f.step(x[e], (int)(e - base));
