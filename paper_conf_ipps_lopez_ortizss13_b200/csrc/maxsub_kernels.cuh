@@ -59,30 +59,28 @@ __device__ __forceinline__ MsTupT<I> ms_combine(const MsTupT<I>& L, const MsTupT
     return c;
 }
 
-// a + x (x sign-extended) as one IMAD.WIDE on the FMA pipe, keeping the
-// integer ALU pipe (the fold's bottleneck) for compares and selects.
-__device__ __forceinline__ long long add_wide(long long a, int x) {
-    long long r;
-    asm("mad.wide.s32 %0, %1, 1, %2;" : "=l"(r) : "r"(x), "l"(a));
-    return r;
-}
-
 // Left-to-right fold of one element x at index i: combine(T, leaf(x, i)),
-// which is Kadane's step with the tie rules above.
+// which is Kadane's step with the tie rules above.  The running values are
+// kept in FP64: a thread folds at most 2^8 int32 elements, so every value is
+// an integer of magnitude < 2^40 (sentinel -2^62 is a power of two) and FP64
+// adds and compares are EXACT.  This moves the adds and compares onto the
+// FP64 pipe and leaves only the selects on the integer ALU pipe, which the
+// int64 version saturated.  tup() converts back to int64.
 struct MsFold {
-    long long tot, pre, suf, best;
+    double tot, pre, suf, best;
     int pe, ss, bs, be;
     __device__ __forceinline__ void init() {
-        tot = 0; pre = kMsNeg; suf = kMsNeg; best = kMsNeg;
+        tot = 0.0; pre = (double)kMsNeg; suf = (double)kMsNeg; best = (double)kMsNeg;
         pe = ss = bs = be = 0;
     }
     __device__ __forceinline__ void step(int x, int i) {
-        tot = add_wide(tot, x);
+        const double xd = (double)x;
+        tot += xd;
         const bool up = tot > pre;                 // strict: smallest end
         pre = up ? tot : pre;
         pe = up ? i : pe;
-        const bool restart = suf < 0;              // max(suf + x, x), ties keep suf
-        suf = add_wide(restart ? 0LL : suf, x);
+        const bool restart = suf < 0.0;            // max(suf + x, x), ties keep suf
+        suf = (restart ? 0.0 : suf) + xd;
         ss = restart ? i : ss;
         const bool better = suf > best;            // strict: smallest (start, end)
         best = better ? suf : best;
@@ -91,7 +89,8 @@ struct MsFold {
     }
     __device__ __forceinline__ MsTup tup() const {
         MsTup t;
-        t.tot = tot; t.pre = pre; t.suf = suf; t.best = best;
+        t.tot = (long long)tot; t.pre = (long long)pre; t.suf = (long long)suf;
+        t.best = (long long)best;
         t.pe = pe; t.ss = ss; t.bs = bs; t.be = be;
         return t;
     }
@@ -198,6 +197,7 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
             // batch's loads issued before the current batch is folded
             constexpr int B4 = 8;
             static_assert(C % (4 * B4) == 0, "chunk must be whole batches");
+            static_assert(C <= 256, "FP64 fold is exact only for chunks <= 2^8 elements");
             const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
             int4 v[B4], nv[B4];
 #pragma unroll
