@@ -71,7 +71,7 @@ SortCfg cfg_for_runtime(dc_key_type kt, bool vals) {
 #define DC_MS_NT 256
 #endif
 #ifndef DC_MS_C
-#define DC_MS_C 32
+#define DC_MS_C 256
 #endif
 constexpr int kNK4Threads = DC_MS_NT;
 constexpr int kNK4Chunk = DC_MS_C;

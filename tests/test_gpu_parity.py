@@ -162,8 +162,10 @@ def test_full_size_2pow28_keys(dc, dist):
 
 # ------------------------------------------------------------ max-subarray
 
-MS_SIZES = [1, 2, 3, 31, 32, 33, 1000, 8191, 8192, 8193, 3 * 8192 + 77, 100_003, 1 << 20,
-            (1 << 20) + 5, 1 << 24]
+MS_TILE = 256 * 256      # max-subarray CTA tile (256 threads x 256-element chunks)
+MS_SIZES = [1, 2, 3, 31, 32, 33, 255, 256, 257, 1000, 8191, 8192, 8193, 3 * 8192 + 77,
+            MS_TILE - 1, MS_TILE, MS_TILE + 1, 5 * MS_TILE + 4097, 100_003, 1 << 20,
+            (1 << 20) + 5, 1 << 24, (1 << 24) + 3]
 
 
 @pytest.mark.parametrize("n", MS_SIZES)
