@@ -56,7 +56,8 @@ _SIGS = {
     "dc_plan": ([_I64, _I32, _I32, _I64, ctypes.POINTER(_P)], ctypes.c_int),
     "dc_plan_levels": ([_P, ctypes.POINTER(_I32), _P, _P, _I32], ctypes.c_int),
     "dc_plan_schedule": ([_P, ctypes.c_int, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
-                          ctypes.POINTER(_I32)], ctypes.c_int),
+                          ctypes.POINTER(_I32), ctypes.POINTER(_I32)], ctypes.c_int),
+    "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_stream": ([_P, _P], ctypes.c_int),
     "dc_plan_scratch_bytes": ([_P, _I32, ctypes.POINTER(ctypes.c_size_t)], ctypes.c_int),
     "dc_plan_set_scratch": ([_P, _P, ctypes.c_size_t], ctypes.c_int),
@@ -164,10 +165,16 @@ class Plan:
         return list(zip(nodes, sizes))
 
     def schedule(self, key_type: str = "u32", with_vals: bool = False) -> dict:
-        t, f, p = _I32(), _I32(), _I32()
+        t, f, p, h = _I32(), _I32(), _I32(), _I32()
         _check(lib().dc_plan_schedule(self._h, _KEY_NAMES[key_type], int(with_vals),
-                                      ctypes.byref(t), ctypes.byref(f), ctypes.byref(p)))
-        return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value}
+                                      ctypes.byref(t), ctypes.byref(f), ctypes.byref(p),
+                                      ctypes.byref(h)))
+        return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value,
+                "hbm_passes": h.value}
+
+    def set_two_level(self, enable: bool) -> None:
+        """Two merge levels per HBM pass for keys-only sorts (default on)."""
+        _check(lib().dc_plan_set_two_level(self._h, int(enable)))
 
     def scratch_bytes(self, with_vals: bool = False) -> int:
         b = ctypes.c_size_t()

@@ -19,6 +19,7 @@
 #include "maxsub_kernels.cuh"
 #include "mg_kernels.cuh"
 #include "sort_kernels.cuh"
+#include "sort2_kernels.cuh"
 
 namespace {
 
@@ -91,6 +92,7 @@ size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 int nk1_smem_bytes(SortCfg c, bool vals) {
     return (vals ? 3 : 1) * dc::tile_words(c.tile(), 0) * 4;
 }
+int nk3_2l_smem_bytes();
 int nk3_smem_bytes(SortCfg c, bool vals) {
     return (vals ? 2 : 1) * dc::tile_words(c.tout(), c.it + 16) * 4;
 }
@@ -113,6 +115,8 @@ struct dc_plan_s {
     dc_maxsub_tuple* ms_tiles = nullptr;
     unsigned int* ms_ticket = nullptr;
     dc_maxsub_result* ms_res = nullptr;
+    // two levels of the merge tree per HBM pass for keys-only sorts (f1)
+    bool two_level = true;
     // multi-GPU splitter state: bracket packs [64] lo, [64] hi, error flag
     unsigned long long* mg_state = nullptr;
     // host-buffer (end-to-end) staging
@@ -139,9 +143,26 @@ int global_passes(int64_t n, int64_t tile) {
 
 size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kMinTout) + 1; }
 
+// Two-level passes (keys-only): granule g = T/4 of the 4-way output tile T.
+constexpr int kTwoT = kCfgFast.tout();
+int nk3_2l_smem_bytes() {   // staging (T + 48) + intermediate (T + IT + 16) words
+    return (kCfgFast.tout() + 48 + kCfgFast.tout() + kCfgFast.it + 16) * 4;
+}
+constexpr int kTwoG = kTwoT / 4;
+static_assert(kTwoT % 4 == 0 && (4 * kCfgFast.tile()) % kTwoT == 0, "two-level tiling");
+
+size_t two_level_tab_entries(int64_t n) {
+    // pairs at the smallest width (w = tile): 2*ceil(n/4w), (2w/g + 1) entries each
+    const int64_t w = kCfgFast.tile();
+    const int64_t pairs = 2 * ((n + 4 * w - 1) / (4 * w));
+    return (size_t)(pairs * (2 * w / kTwoG + 1));
+}
+size_t two_level_bnd_entries(int64_t n) { return 3 * ((size_t)num_tiles(n, kTwoT) + 2); }
+
 size_t scratch_needed(int64_t n, bool vals) {
     size_t kb = align_up((size_t)n * 4, 256);
-    return kb + (vals ? kb : 0) + align_up(split_entries(n) * 4, 256);
+    return kb + (vals ? kb : 0) + align_up(split_entries(n) * 4, 256) +
+           align_up(two_level_tab_entries(n) * 4, 256) + align_up(two_level_bnd_entries(n) * 4, 256);
 }
 
 dc_status check_plan(dc_plan_t p) {
@@ -245,13 +266,20 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
         attr_done = true;
     }
 
+    // Levels over HBM: P = ceil(log2(ceil(n/tile))).  Keys-only sorts fold
+    // two levels into one pass (4-way groups, sort2_kernels.cuh); with P odd
+    // one single-level pass goes first.
     const int P = global_passes(n, C.tile());
-    // Ping-pong parity: pass P-1 must write the caller's buffer, so NK1
-    // writes the caller's buffer iff P is even.
-    uint32_t* cur_k = (P % 2 == 0) ? keys : sk;
-    uint32_t* cur_v = (P % 2 == 0) ? vals : sv;
-    uint32_t* oth_k = (P % 2 == 0) ? sk : keys;
-    uint32_t* oth_v = (P % 2 == 0) ? sv : vals;
+    constexpr bool kTwoCapable = !V && !K::kNeedStable;
+    const bool two = kTwoCapable && p->two_level && P >= 2;
+    const int single = two ? (P % 2) : P;
+    const int passes = two ? single + (P - single) / 2 : P;
+    // Ping-pong parity: the last pass must write the caller's buffer, so NK1
+    // writes the caller's buffer iff the number of passes is even.
+    uint32_t* cur_k = (passes % 2 == 0) ? keys : sk;
+    uint32_t* cur_v = (passes % 2 == 0) ? vals : sv;
+    uint32_t* oth_k = (passes % 2 == 0) ? sk : keys;
+    uint32_t* oth_v = (passes % 2 == 0) ? sv : vals;
 
     // NK1: base cases + fused bottom levels (reads the caller's buffer).
     {
@@ -261,8 +289,9 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
         DC_LAUNCHED(p);
     }
 
+    int64_t w = C.tile();
     const int tiles = (int)num_tiles(n, C.tout());
-    for (int64_t w = C.tile(); w < n; w *= 2) {
+    for (int lv = 0; lv < single; ++lv, w *= 2) {
         {
             TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
             dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
@@ -277,6 +306,40 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
         }
         std::swap(cur_k, oth_k);
         std::swap(cur_v, oth_v);
+    }
+    if constexpr (kTwoCapable) {
+        if (two) {
+            int* tab = split + align_up(split_entries(n) * 4, 256) / 4;
+            int* bnd = tab + align_up(two_level_tab_entries(n) * 4, 256) / 4;
+            auto* k32 = dc::nk3_merge2<C.nt3, C.it, K>;
+            const int smem2 = nk3_2l_smem_bytes();
+            static bool attr2 = false;
+            if (!attr2) {
+                DC_CUDA(p, cudaFuncSetAttribute(k32, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                smem2));
+                attr2 = true;
+            }
+            const int tiles2 = (int)num_tiles(n, kTwoT);
+            for (; w < n; w *= 4) {
+                const int K1 = (int)(2 * w / kTwoG + 1);
+                const int64_t entries = 2 * ((n + 4 * w - 1) / (4 * w)) * K1;
+                {
+                    TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
+                    dc::nk2a_granules<K><<<(unsigned)((entries + 255) / 256), 256, 0, p->stream>>>(
+                        cur_k, n, w, kTwoG, K1, entries, tab);
+                    DC_LAUNCHED(p);
+                    dc::nk2b_partition2<K><<<(tiles2 + 127) / 128, 128, 0, p->stream>>>(
+                        cur_k, n, w, kTwoT, kTwoG, K1, tab, tiles2, bnd);
+                    DC_LAUNCHED(p);
+                }
+                {
+                    TimedScope ts(p, DC_KERNEL_NK3_MERGE);
+                    k32<<<tiles2, C.nt3, smem2, p->stream>>>(cur_k, oth_k, n, w, bnd);
+                    DC_LAUNCHED(p);
+                }
+                std::swap(cur_k, oth_k);
+            }
+        }
     }
     return DC_OK;
 }
@@ -497,7 +560,7 @@ dc_status dc_plan_levels(dc_plan_t p, int32_t* num_levels, int64_t* nodes, int64
 }
 
 dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32_t* tile,
-                           int32_t* fused_levels, int32_t* passes) {
+                           int32_t* fused_levels, int32_t* passes, int32_t* hbm_passes) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
@@ -506,7 +569,16 @@ dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32
     int f = 0;   // levels of the binary tree inside one tile: ceil(log2(tile))
     while ((1 << f) < c.tile()) ++f;
     if (fused_levels) *fused_levels = f;
-    if (passes) *passes = global_passes(p->n, c.tile());
+    const int P = global_passes(p->n, c.tile());
+    if (passes) *passes = P;
+    const bool two = p->two_level && !with_vals && kt != DC_KEY_F32 && P >= 2;
+    if (hbm_passes) *hbm_passes = two ? (P % 2) + (P - P % 2) / 2 : P;
+    return DC_OK;
+}
+
+dc_status dc_plan_set_two_level(dc_plan_t p, int32_t enable) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    p->two_level = enable != 0;
     return DC_OK;
 }
 

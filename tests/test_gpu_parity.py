@@ -78,6 +78,26 @@ def test_sort_keys_only_signed_float(dc, oracle_mod, key_type, n):
     assert np.array_equal(_np_keys(k_out, key_type).view(np.uint32), ek.view(np.uint32))
 
 
+TWO_LEVEL_SIZES = [2 * TILE, 2 * TILE + 1, 3 * TILE + 7, 4 * TILE, 5 * TILE + 11, 8 * TILE,
+                   9 * TILE + 3, 16 * TILE + 1, 37 * TILE + 12345, (1 << 22) + 5, 1 << 24]
+
+
+@pytest.mark.parametrize("n", TWO_LEVEL_SIZES)
+@pytest.mark.parametrize("dist", ["uniform", "few", "sorted", "reverse", "equal"])
+@pytest.mark.parametrize("key_type", ["u32", "i32"])
+def test_sort_two_level_vs_one_level(dc, oracle_mod, n, dist, key_type):
+    """Two merge levels per HBM pass (f1) and one level per pass give the oracle's result."""
+    keys = dcgen.sort_keys(n, dist, seed=13, key_type=key_type, device="cuda")
+    k_in = _np_keys(keys, key_type)
+    expect = oracle_mod.mergesort(k_in, key_type=key_type).view(np.uint32)
+    for two in (True, False):
+        k = keys.clone()
+        plan = dc.Plan(n)
+        plan.set_two_level(two)
+        plan.sort_(k, key_type=key_type)
+        assert np.array_equal(_np_keys(k, key_type).view(np.uint32), expect), two
+
+
 def test_sort_max_key_values_and_pads(dc, oracle_mod):
     # real keys equal to the pad value (0xFFFFFFFF) in a ragged last tile
     n = 3 * TILE + 100
@@ -226,4 +246,6 @@ def test_launch_counts(dc):
     keys = dcgen.sort_keys(n, "uniform", device="cuda")
     p.sort_(keys, key_type="u32")
     s = p.schedule("u32", False)
-    assert p.launch_count() == 1 + 2 * s["global_passes"]
+    P, H = s["global_passes"], s["hbm_passes"]
+    single = P - 2 * (P - H)          # one-level passes: 2 launches; two-level: 3 launches
+    assert p.launch_count() == 1 + 2 * single + 3 * (H - single)
