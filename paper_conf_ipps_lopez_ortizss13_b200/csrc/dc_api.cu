@@ -145,9 +145,7 @@ size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kMinTout) + 1; }
 
 // Two-level passes (keys-only): granule g = T/4 of the 4-way output tile T.
 constexpr int kTwoT = kCfgFast.tout();
-int nk3_2l_smem_bytes() {   // staging (T + 48) + intermediate (T + IT + 16) words
-    return (kCfgFast.tout() + 48 + kCfgFast.tout() + kCfgFast.it + 16) * 4;
-}
+int nk3_2l_smem_bytes() { return dc::nk3_2l_words(kCfgFast.tout(), kCfgFast.it) * 4; }
 constexpr int kTwoG = kTwoT / 4;
 static_assert(kTwoT % 4 == 0 && (4 * kCfgFast.tile()) % kTwoT == 0, "two-level tiling");
 
@@ -328,13 +326,13 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
                     dc::nk2a_granules<K><<<(unsigned)((entries + 255) / 256), 256, 0, p->stream>>>(
                         cur_k, n, w, kTwoG, K1, entries, tab);
                     DC_LAUNCHED(p);
-                    dc::nk2b_partition2<K><<<(tiles2 + 127) / 128, 128, 0, p->stream>>>(
+                    dc::nk2b_partition2<K><<<(tiles2 + 3) / 4, 128, 0, p->stream>>>(
                         cur_k, n, w, kTwoT, kTwoG, K1, tab, tiles2, bnd);
                     DC_LAUNCHED(p);
                 }
                 {
                     TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                    k32<<<tiles2, C.nt3, smem2, p->stream>>>(cur_k, oth_k, n, w, bnd);
+                    k32<<<tiles2, C.nt3 + 32, smem2, p->stream>>>(cur_k, oth_k, n, w, bnd);
                     DC_LAUNCHED(p);
                 }
                 std::swap(cur_k, oth_k);

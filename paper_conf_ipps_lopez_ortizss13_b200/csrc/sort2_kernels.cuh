@@ -95,15 +95,44 @@ __global__ void nk2a_granules(const uint32_t* __restrict__ src, long long n, lon
     tab[e] = (int)corank_global<K>(src + s, la, src + s + la, lb, p);
 }
 
-// NK2b: exact two-level co-ranks of every output tile boundary.  Tile j
-// starts at global output j*T inside group G = j*T / 4w (T divides 4w, g
-// divides T).  Writes bnd[3j..3j+2] = {c, x, y}.
+// First index in [a, b] where a monotone (true ... false) predicate on [a, b)
+// is false (b if none), found by one warp: every round the 32 lanes evaluate
+// f at 32 evenly spaced points (__ballot), shrinking the interval 33-fold.
+template <class F>
+__device__ __forceinline__ long long warp_first_false(long long a, long long b, F f) {
+    const int lane = threadIdx.x & 31;
+    while (a < b) {
+        const long long span = b - a;
+        const long long pos = a + ((lane + 1) * span) / 33;       // < b
+        const unsigned fm = __ballot_sync(0xffffffffu, !f(pos));
+        if (fm == 0) {
+            a = a + (32 * span) / 33 + 1;
+        } else {
+            const int L = __ffs(fm) - 1;
+            const long long posL = a + ((L + 1) * span) / 33;
+            const long long posP = L > 0 ? a + (L * span) / 33 : a - 1;
+            b = posL;
+            a = posP + 1;
+        }
+    }
+    return a;
+}
+
+// NK2b: exact two-level co-ranks of every output tile boundary, one warp per
+// boundary.  Tile j starts at global output j*T inside group G = j*T / 4w (T
+// divides 4w, g divides T).  f(m) = M1[m] <= M2[d-1-m] is true then false on
+// [lo, hi); c = its first false index: a coarse warp search over the granule
+// points m = k*g (O(1) each from the table), then a fine warp search inside
+// one granule (each probe two granule-restricted co-rank searches).  Writes
+// bnd[3j..3j+2] = {c, x, y}: x = #R1 among the first c of M1, y = #R3 among
+// the first d - c of M2.
 template <class K>
 __global__ void nk2b_partition2(const uint32_t* __restrict__ src, long long n, long long w,
                                 long long T, long long g, int K1, const int* __restrict__ tab,
                                 int num_tiles, int* __restrict__ bnd) {
-    const int j = blockIdx.x * blockDim.x + threadIdx.x;
-    if (j >= num_tiles) return;
+    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    if (j >= num_tiles) return;                       // warp-uniform
+    const int lane = threadIdx.x & 31;
     const long long G = ((long long)j * T) / (4 * w);
     long long s, l1, l2, l3, l4;
     group_runs(n, w, G, s, l1, l2, l3, l4);
@@ -112,62 +141,44 @@ __global__ void nk2b_partition2(const uint32_t* __restrict__ src, long long n, l
     const GPair<K> M2{src + s + 2 * w, l3, src + s + 2 * w + l3, l4, tab + (2 * G + 1) * K1, g};
     const long long m1 = l1 + l2, m2 = l3 + l4;
     long long lo = max(0LL, d - m2), hi = min(d, m1);
-    // f(m) = M1[m] <= M2[d-1-m] is true then false on [lo, hi); c = first false.
     if (lo < hi) {
         const long long klo = (lo + g - 1) / g, khi = (hi - 1) / g;
-        if (klo <= khi) {               // coarse: granule points m = k*g, O(1) each
-            long long a = klo, b = khi + 1;
-            while (a < b) {
-                const long long k = (a + b) >> 1, m = k * g;
+        if (klo <= khi) {                             // coarse: granule points
+            const long long a = warp_first_false(klo, khi + 1, [&](long long k) {
+                const long long m = k * g;
                 const uint32_t x1 = M1.at_i(m, M1.tab[k]);
-                const long long q = d - m;                  // multiple of g, >= 1
+                const long long q = d - m;            // multiple of g, >= 1
                 const uint32_t y1 = M2.last_i(q, M2.tab[q / g]);
-                if (!K::lt(y1, x1)) a = k + 1; else b = k;
-            }
+                return !K::lt(y1, x1);
+            });
             if (a > klo) lo = max(lo, (a - 1) * g + 1);
             if (a <= khi) hi = min(hi, a * g);
         }
-        while (lo < hi) {               // fine: inside one granule
-            const long long m = (lo + hi) >> 1;
+        lo = warp_first_false(lo, hi, [&](long long m) {   // fine: one granule
             const uint32_t x1 = M1.at(m);
             const uint32_t y1 = M2.at(d - 1 - m);
-            if (!K::lt(y1, x1)) lo = m + 1; else hi = m;
-        }
+            return !K::lt(y1, x1);
+        });
     }
     const long long c = lo;
-    bnd[3 * j + 0] = (int)c;
-    bnd[3 * j + 1] = (int)M1.corank(c);
-    bnd[3 * j + 2] = (int)M2.corank(d - c);
+    if (lane == 0) bnd[3 * j + 0] = (int)c;
+    if (lane == 1) bnd[3 * j + 1] = (int)M1.corank(c);
+    if (lane == 2) bnd[3 * j + 2] = (int)M2.corank(d - c);
 }
 
-// Stable serial merge of the window [diag, diag + IT) of merge(A, B) (shared
-// byte addresses, lengths na, nb) written to shared words out[diag + q] for
-// the valid q < total - diag.
-template <class K, int IT>
-__device__ __forceinline__ void merge_window_to_smem(uint32_t A, int na, uint32_t B, int nb,
-                                                     int diag, uint32_t* out) {
-    const int i = corank_smem<K>(A, na, B, nb, diag);
-    uint32_t k[IT], src[IT];
-    serial_merge<K, IT, false>(A + 4u * i, A + 4u * na, B + 4u * (diag - i), B + 4u * nb, k,
-                               src);
-    const int valid = min(IT, na + nb - diag);
-#pragma unroll
-    for (int q = 0; q < IT; ++q)
-        if (q < valid) out[diag + q] = k[q];
-}
-
-// NK3-2L: tile J of the two-level pass (keys only).
+// NK3-2L: tile J of the two-level pass (keys only), T = NT*IT outputs.
+// NT + 32 threads: stage 1 has up to NT + 1 windows of IT outputs (the M1
+// and M2 pieces are windowed separately).  Stage-1 results wait in registers
+// and then overwrite the staging buffer, so one T-sized buffer serves the
+// four pieces, the two intermediate pieces and the output tile.
 template <int NT, int IT, class K>
-__global__ void __launch_bounds__(NT)
+__global__ void __launch_bounds__(NT + 32)
 nk3_merge2(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long long n, long long w,
            const int* __restrict__ bnd) {
     constexpr int T = NT * IT;
-    constexpr int SW = T + 4 * 8 + 16;     // staging words: 4 pieces + alignment slack
-    extern __shared__ __align__(16) uint32_t smem[];
-    uint32_t* st = smem;                   // staging: P1 | P2 | P3 | P4, later the output
-    uint32_t* mid = smem + SW;             // M1 piece | M2 piece
+    extern __shared__ __align__(16) uint32_t st[];   // nk3_2l_words(T, IT) words
     __shared__ __align__(8) uint64_t bar;
-    const uint32_t ST = smem_addr(st), MID = smem_addr(mid), BAR = smem_addr(&bar);
+    const uint32_t ST = smem_addr(st), BAR = smem_addr(&bar);
     const int tid = threadIdx.x;
     const long long J = blockIdx.x;
     const long long G = (J * T) / (4 * w);
@@ -203,36 +214,48 @@ nk3_merge2(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
     }
     for (int p = 0; p < 4; ++p) {          // elements at or past n4 (array tail only)
         if (g0[p] + len[p] > n4) {
-            for (long long e = max(g0[p], n4) + tid; e < g0[p] + len[p]; e += NT)
+            for (long long e = max(g0[p], n4) + tid; e < g0[p] + len[p]; e += NT + 32)
                 st[off[p] + (int)(g0[p] & 3) + (e - g0[p])] = src[e];
         }
     }
     __syncthreads();
     mbar_wait(BAR, 0);
 
-    // stage 1: M1 piece = merge(P1, P2) -> mid[0, n1); M2 piece = merge(P3, P4) -> mid[o2, ...)
+    // stage 1 (registers): window tid of [M1 piece windows | M2 piece windows]
     const int n1 = len[0] + len[1], n2 = len[2] + len[3];
-    const int o2 = n1 + 4;                 // slack words between the two intermediate pieces
-    const uint32_t P[4] = {ST + 4u * (off[0] + (int)(g0[0] & 3)), ST + 4u * (off[1] + (int)(g0[1] & 3)),
-                           ST + 4u * (off[2] + (int)(g0[2] & 3)), ST + 4u * (off[3] + (int)(g0[3] & 3))};
     const int w1 = (n1 + IT - 1) / IT, w2 = (n2 + IT - 1) / IT;
-    for (int win = tid; win < w1 + w2; win += NT) {
-        if (win < w1) merge_window_to_smem<K, IT>(P[0], len[0], P[1], len[1], win * IT, mid);
-        else merge_window_to_smem<K, IT>(P[2], len[2], P[3], len[3], (win - w1) * IT, mid + o2);
+    uint32_t k[IT], srcb[IT];
+    int out0 = 0, valid = 0;
+    const int o2 = n1 + 4;                 // intermediate layout: M1 piece | 4 slack | M2 piece
+    if (tid < w1 + w2) {
+        const bool first = tid < w1;
+        const int pa = first ? 0 : 2;
+        const uint32_t A = ST + 4u * (off[pa] + (int)(g0[pa] & 3));
+        const uint32_t B = ST + 4u * (off[pa + 1] + (int)(g0[pa + 1] & 3));
+        const int na = len[pa], nb = len[pa + 1];
+        const int diag = (first ? tid : tid - w1) * IT;
+        const int i = corank_smem<K>(A, na, B, nb, diag);
+        serial_merge<K, IT, false>(A + 4u * i, A + 4u * na, B + 4u * (diag - i), B + 4u * nb, k,
+                                   srcb);
+        valid = min(IT, na + nb - diag);
+        out0 = (first ? 0 : o2) + diag;
     }
+    __syncthreads();                       // all pieces consumed
+#pragma unroll
+    for (int q = 0; q < IT; ++q)
+        if (q < valid) st[out0 + q] = k[q];
     __syncthreads();
 
     // stage 2: merge the M1 and M2 pieces -> T outputs, blocked into `st`
     const int total = n1 + n2;
     const int diag = tid * IT;
-    uint32_t k[IT], srcb[IT];
-    if (diag < total) {
-        const int i = corank_smem<K>(MID, n1, MID + 4u * o2, n2, diag);
-        serial_merge<K, IT, false>(MID + 4u * i, MID + 4u * n1, MID + 4u * (o2 + diag - i),
-                                   MID + 4u * (o2 + n2), k, srcb);
+    if (tid < NT && diag < total) {
+        const int i = corank_smem<K>(ST, n1, ST + 4u * o2, n2, diag);
+        serial_merge<K, IT, false>(ST + 4u * i, ST + 4u * n1, ST + 4u * (o2 + diag - i),
+                                   ST + 4u * (o2 + n2), k, srcb);
     }
     __syncthreads();
-    if (diag < total) {
+    if (tid < NT && diag < total) {
 #pragma unroll
         for (int q = 0; q < IT; ++q) st[diag + q] = k[q];
     }
@@ -240,5 +263,10 @@ nk3_merge2(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
     __syncthreads();
     store_tile(dst + J * T, st, 0, total);
 }
+
+// Shared words of nk3_merge2: the four staged pieces (T + 28 with alignment
+// slack), the intermediate pieces (T + 4) and the serial merges' past-the-end
+// reads (up to IT words), rounded to 16 bytes.
+__host__ __device__ constexpr int nk3_2l_words(int T, int IT) { return (T + IT + 64 + 3) / 4 * 4; }
 
 }  // namespace dc
