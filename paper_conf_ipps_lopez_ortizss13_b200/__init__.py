@@ -173,7 +173,7 @@ class Plan:
                 "hbm_passes": h.value}
 
     def set_two_level(self, enable: bool) -> None:
-        """Two merge levels per HBM pass for keys-only sorts (default on)."""
+        """Two merge levels per HBM pass for keys-only sorts (default off)."""
         _check(lib().dc_plan_set_two_level(self._h, int(enable)))
 
     def scratch_bytes(self, with_vals: bool = False) -> int:

@@ -115,8 +115,11 @@ struct dc_plan_s {
     dc_maxsub_tuple* ms_tiles = nullptr;
     unsigned int* ms_ticket = nullptr;
     dc_maxsub_result* ms_res = nullptr;
-    // two levels of the merge tree per HBM pass for keys-only sorts (f1)
-    bool two_level = true;
+    // two levels of the merge tree per HBM pass for keys-only sorts (f1).
+    // Off by default: bit-exact, and its 4-way tile merge beats two one-level
+    // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
+    // two-level partition costs 0.21 ms per pass vs 2 x 0.03.
+    bool two_level = false;
     // multi-GPU splitter state: bracket packs [64] lo, [64] hi, error flag
     unsigned long long* mg_state = nullptr;
     // host-buffer (end-to-end) staging

@@ -108,9 +108,13 @@ def test_schedule(n, kt, vals):
     t = s["tile"]
     assert s["fused_levels"] == math.ceil(math.log2(t))
     assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))
-    # keys-only sorts fold two levels per HBM pass
+    # one level per HBM pass by default; keys-only sorts can fold two (f1)
     P = s["global_passes"]
-    assert s["hbm_passes"] == (P if (vals or kt == "f32" or P < 2) else P % 2 + P // 2)
+    assert s["hbm_passes"] == P
+    p2 = dc.Plan(n)
+    p2.set_two_level(True)
+    s2 = p2.schedule(kt, vals)
+    assert s2["hbm_passes"] == (P if (vals or kt == "f32" or P < 2) else P % 2 + P // 2)
     # fused + global levels cover the whole tree: ceil(log2 n) combine levels
     if n > 1:
         assert s["fused_levels"] + s["global_passes"] >= math.ceil(math.log2(n))
