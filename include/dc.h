@@ -110,6 +110,12 @@ dc_status dc_plan_schedule(dc_plan_t plan, dc_key_type key_type, int32_t with_va
  * sorts (a 4-way merge per HBM pass).  Results are identical. */
 dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
 
+/* Enable (default) or disable CUDA-graph replay of the sort's launch sequence:
+ * the first dc_run_mergesort for a given (keys, vals, key type) runs eagerly,
+ * the second captures a graph, later ones replay it.  Disabled automatically
+ * while per-kernel timing is on.  Results are identical. */
+dc_status dc_plan_set_graphs(dc_plan_t plan, int32_t enable);
+
 /* Stream all device work of this plan is enqueued on (a cudaStream_t). */
 dc_status dc_plan_set_stream(dc_plan_t plan, void *cuda_stream);
 

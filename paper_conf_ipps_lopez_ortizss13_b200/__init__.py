@@ -58,6 +58,7 @@ _SIGS = {
     "dc_plan_schedule": ([_P, ctypes.c_int, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
                           ctypes.POINTER(_I32), ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
+    "dc_plan_set_graphs": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_stream": ([_P, _P], ctypes.c_int),
     "dc_plan_scratch_bytes": ([_P, _I32, ctypes.POINTER(ctypes.c_size_t)], ctypes.c_int),
     "dc_plan_set_scratch": ([_P, _P, ctypes.c_size_t], ctypes.c_int),
@@ -171,6 +172,10 @@ class Plan:
                                       ctypes.byref(h)))
         return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value,
                 "hbm_passes": h.value}
+
+    def set_graphs(self, enable: bool) -> None:
+        """CUDA-graph replay of the sort's launch sequence (default on)."""
+        _check(lib().dc_plan_set_graphs(self._h, int(enable)))
 
     def set_two_level(self, enable: bool) -> None:
         """Two merge levels per HBM pass for keys-only sorts (default off)."""

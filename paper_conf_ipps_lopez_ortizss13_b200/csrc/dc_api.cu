@@ -56,16 +56,28 @@ struct SortCfg {
 #endif
 constexpr SortCfg kCfgFast{DC_FAST_NT1, DC_FAST_IT, DC_FAST_NT3};
 constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3};
+// Small inputs (n < kSmallN, L2-resident): quarter-size tiles so that the
+// fused kernel and every merge level still launch >= ~150 CTAs.
+constexpr SortCfg kCfgFastSmall{128, DC_FAST_IT, 128};
+constexpr SortCfg kCfgStableSmall{128, DC_STABLE_IT, 128};
+constexpr int64_t kSmallN = 1LL << 23;
 static_assert((2 * kCfgFast.tile()) % kCfgFast.tout() == 0, "merge tiles must not straddle pairs");
 static_assert((2 * kCfgStable.tile()) % kCfgStable.tout() == 0, "merge tiles must not straddle pairs");
-constexpr int kMinTout = kCfgFast.tout() < kCfgStable.tout() ? kCfgFast.tout() : kCfgStable.tout();
+static_assert((2 * kCfgFastSmall.tile()) % kCfgFastSmall.tout() == 0, "tiles straddle pairs");
+static_assert((2 * kCfgStableSmall.tile()) % kCfgStableSmall.tout() == 0, "tiles straddle pairs");
+constexpr int cmin(int a, int b) { return a < b ? a : b; }
+constexpr int kMinTout = cmin(cmin(kCfgFast.tout(), kCfgStable.tout()),
+                              cmin(kCfgFastSmall.tout(), kCfgStableSmall.tout()));
 
-template <class K, bool V>
+template <class K, bool V, bool SMALL>
 constexpr SortCfg cfg_for() {
-    return (V || K::kNeedStable) ? kCfgStable : kCfgFast;
+    return (V || K::kNeedStable) ? (SMALL ? kCfgStableSmall : kCfgStable)
+                                 : (SMALL ? kCfgFastSmall : kCfgFast);
 }
-SortCfg cfg_for_runtime(dc_key_type kt, bool vals) {
-    return (vals || kt == DC_KEY_F32) ? kCfgStable : kCfgFast;
+SortCfg cfg_for_runtime(dc_key_type kt, bool vals, int64_t n) {
+    const bool small = n < kSmallN;
+    return (vals || kt == DC_KEY_F32) ? (small ? kCfgStableSmall : kCfgStable)
+                                      : (small ? kCfgFastSmall : kCfgFast);
 }
 
 #ifndef DC_MS_NT
@@ -115,6 +127,18 @@ struct dc_plan_s {
     dc_maxsub_tuple* ms_tiles = nullptr;
     unsigned int* ms_ticket = nullptr;
     dc_maxsub_result* ms_res = nullptr;
+    // CUDA graphs of the sort's launch sequence, per (keys, vals, key type)
+    struct GraphCache {
+        uint32_t* keys;
+        uint32_t* vals;
+        dc_key_type kt;
+        cudaGraph_t graph;
+        cudaGraphExec_t exec;
+        int64_t launches;
+    };
+    bool use_graphs = true;
+    std::vector<GraphCache> graphs;
+    cudaStream_t cap_stream = nullptr;
     // two levels of the merge tree per HBM pass for keys-only sorts (f1).
     // Off by default: bit-exact, and its 4-way tile merge beats two one-level
     // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
@@ -244,7 +268,7 @@ dc_status ensure_scratch(dc_plan_t p, bool vals) {
     return DC_OK;
 }
 
-template <class K, bool V>
+template <class K, bool V, bool SMALL>
 dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     const int64_t n = p->n;
     const bool hv = V;
@@ -255,7 +279,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     uint32_t* sv = hv ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
     int* split = (int*)((char*)p->scratch + kb + (hv ? kb : 0));
 
-    constexpr SortCfg C = cfg_for<K, V>();
+    constexpr SortCfg C = cfg_for<K, V, SMALL>();
     auto* k1 = dc::nk1_blocksort<C.nt1, C.it, K, V>;
     auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
     static bool attr_done = false;   // per key/value instantiation
@@ -271,7 +295,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     // two levels into one pass (4-way groups, sort2_kernels.cuh); with P odd
     // one single-level pass goes first.
     const int P = global_passes(n, C.tile());
-    constexpr bool kTwoCapable = !V && !K::kNeedStable;
+    constexpr bool kTwoCapable = !V && !K::kNeedStable && !SMALL;
     const bool two = kTwoCapable && p->two_level && P >= 2;
     const int single = two ? (P % 2) : P;
     const int passes = two ? single + (P - single) / 2 : P;
@@ -295,8 +319,12 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     for (int lv = 0; lv < single; ++lv, w *= 2) {
         {
             TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-            dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
-                cur_k, dc::PairGeom{0, w, w, n}, C.tout(), tiles, split);
+            if (SMALL)   // L2-resident: 33-ary warp searches, few dependent rounds
+                dc::nk2_partition_warp<K><<<(tiles + 3) / 4, 128, 0, p->stream>>>(
+                    cur_k, dc::PairGeom{0, w, w, n}, C.tout(), tiles, split);
+            else
+                dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
+                    cur_k, dc::PairGeom{0, w, w, n}, C.tout(), tiles, split);
             DC_LAUNCHED(p);
         }
         {
@@ -345,20 +373,59 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     return DC_OK;
 }
 
-dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
-    const bool v = vals != nullptr;
+template <class K>
+dc_status sort_kv_dispatch(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
+    const bool small = p->n < kSmallN;
+    if (vals) return small ? sort_typed<K, true, true>(p, keys, vals)
+                           : sort_typed<K, true, false>(p, keys, vals);
+    return small ? sort_typed<K, false, true>(p, keys, nullptr)
+                 : sort_typed<K, false, false>(p, keys, nullptr);
+}
+
+dc_status sort_direct(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
     switch (kt) {
-        case DC_KEY_U32:
-            return v ? sort_typed<dc::KeyU32, true>(p, keys, vals)
-                     : sort_typed<dc::KeyU32, false>(p, keys, nullptr);
-        case DC_KEY_I32:
-            return v ? sort_typed<dc::KeyI32, true>(p, keys, vals)
-                     : sort_typed<dc::KeyI32, false>(p, keys, nullptr);
-        case DC_KEY_F32:
-            return v ? sort_typed<dc::KeyF32, true>(p, keys, vals)
-                     : sort_typed<dc::KeyF32, false>(p, keys, nullptr);
+        case DC_KEY_U32: return sort_kv_dispatch<dc::KeyU32>(p, keys, vals);
+        case DC_KEY_I32: return sort_kv_dispatch<dc::KeyI32>(p, keys, vals);
+        case DC_KEY_F32: return sort_kv_dispatch<dc::KeyF32>(p, keys, vals);
     }
     return fail(DC_ERR_INVALID_ARG, "unknown key type");
+}
+
+// CUDA-graph replay of the whole level sequence (launch-bound small sorts).
+// The first run for a given (keys, vals, key type) executes eagerly (it
+// allocates scratch and sets kernel attributes); the second captures the
+// launches on a plan-owned stream and instantiates a graph; later runs
+// replay it on the plan stream.  Off while per-kernel timing is enabled.
+dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
+    if (!p->use_graphs || p->timing) return sort_direct(p, kt, keys, vals);
+    for (auto& gc : p->graphs) {
+        if (gc.keys == keys && gc.vals == vals && gc.kt == kt) {
+            if (!gc.exec) {                                   // second sighting: capture
+                if (!p->cap_stream)
+                    DC_CUDA(p, cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking));
+                cudaStream_t user = p->stream;
+                p->stream = p->cap_stream;
+                DC_CUDA(p, cudaStreamBeginCapture(p->cap_stream, cudaStreamCaptureModeThreadLocal));
+                const int64_t l0 = p->launches;
+                dc_status st = sort_direct(p, kt, keys, vals);
+                cudaGraph_t graph = nullptr;
+                cudaError_t e = cudaStreamEndCapture(p->cap_stream, &graph);
+                p->stream = user;
+                if (st != DC_OK) return st;
+                if (e != cudaSuccess) return cuda_fail(p, e, "cudaStreamEndCapture");
+                gc.graph = graph;
+                gc.launches = p->launches - l0;
+                p->launches = l0;
+                DC_CUDA(p, cudaGraphInstantiate(&gc.exec, graph, 0));
+            }
+            DC_CUDA(p, cudaGraphLaunch(gc.exec, p->stream));
+            p->launches += gc.launches;
+            return DC_OK;
+        }
+    }
+    if (p->graphs.size() >= 8) return sort_direct(p, kt, keys, vals);
+    p->graphs.push_back({keys, vals, kt, nullptr, nullptr, 0});   // first sighting: eager
+    return sort_direct(p, kt, keys, vals);
 }
 
 // Max-subarray grid: about one wave of resident CTAs (occupancy x SMs),
@@ -434,7 +501,7 @@ dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* 
     uint32_t* sk = (uint32_t*)p->scratch;
     uint32_t* sv = V ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
     int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
-    constexpr SortCfg C = cfg_for<K, V>();
+    constexpr SortCfg C = cfg_for<K, V, false>();
     auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
     static bool attr_done = false;
     if (!attr_done) {
@@ -565,21 +632,37 @@ dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
-    const SortCfg c = cfg_for_runtime(kt, with_vals != 0);
+    const SortCfg c = cfg_for_runtime(kt, with_vals != 0, p->n);
     if (tile) *tile = c.tile();
     int f = 0;   // levels of the binary tree inside one tile: ceil(log2(tile))
     while ((1 << f) < c.tile()) ++f;
     if (fused_levels) *fused_levels = f;
     const int P = global_passes(p->n, c.tile());
     if (passes) *passes = P;
-    const bool two = p->two_level && !with_vals && kt != DC_KEY_F32 && P >= 2;
+    const bool two = p->two_level && !with_vals && kt != DC_KEY_F32 && P >= 2 && p->n >= kSmallN;
     if (hbm_passes) *hbm_passes = two ? (P % 2) + (P - P % 2) / 2 : P;
     return DC_OK;
+}
+
+static void drop_graphs(dc_plan_t p) {
+    for (auto& gc : p->graphs) {
+        if (gc.exec) cudaGraphExecDestroy(gc.exec);
+        if (gc.graph) cudaGraphDestroy(gc.graph);
+    }
+    p->graphs.clear();
 }
 
 dc_status dc_plan_set_two_level(dc_plan_t p, int32_t enable) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     p->two_level = enable != 0;
+    drop_graphs(p);
+    return DC_OK;
+}
+
+dc_status dc_plan_set_graphs(dc_plan_t p, int32_t enable) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    p->use_graphs = enable != 0;
+    drop_graphs(p);
     return DC_OK;
 }
 
@@ -601,6 +684,7 @@ dc_status dc_plan_set_scratch(dc_plan_t p, void* d, size_t bytes) {
     if (bytes < scratch_needed(p->n, false))
         return fail(DC_ERR_INVALID_ARG, "scratch smaller than dc_plan_scratch_bytes");
     if (p->scratch && p->own_scratch) cudaFree(p->scratch);
+    drop_graphs(p);
     p->scratch = d;
     p->scratch_bytes = bytes;
     p->own_scratch = false;
@@ -618,6 +702,11 @@ dc_status dc_free(dc_plan_t p) {
     if (p->ms_tiles) cudaFree(p->ms_tiles);
     if (p->d_stage) cudaFree(p->d_stage);
     if (p->mg_state) cudaFree(p->mg_state);
+    for (auto& gc : p->graphs) {
+        if (gc.exec) cudaGraphExecDestroy(gc.exec);
+        if (gc.graph) cudaGraphDestroy(gc.graph);
+    }
+    if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
     delete p;
     return DC_OK;
 }

@@ -95,29 +95,6 @@ __global__ void nk2a_granules(const uint32_t* __restrict__ src, long long n, lon
     tab[e] = (int)corank_global<K>(src + s, la, src + s + la, lb, p);
 }
 
-// First index in [a, b] where a monotone (true ... false) predicate on [a, b)
-// is false (b if none), found by one warp: every round the 32 lanes evaluate
-// f at 32 evenly spaced points (__ballot), shrinking the interval 33-fold.
-template <class F>
-__device__ __forceinline__ long long warp_first_false(long long a, long long b, F f) {
-    const int lane = threadIdx.x & 31;
-    while (a < b) {
-        const long long span = b - a;
-        const long long pos = a + ((lane + 1) * span) / 33;       // < b
-        const unsigned fm = __ballot_sync(0xffffffffu, !f(pos));
-        if (fm == 0) {
-            a = a + (32 * span) / 33 + 1;
-        } else {
-            const int L = __ffs(fm) - 1;
-            const long long posL = a + ((L + 1) * span) / 33;
-            const long long posP = L > 0 ? a + (L * span) / 33 : a - 1;
-            b = posL;
-            a = posP + 1;
-        }
-    }
-    return a;
-}
-
 // NK2b: exact two-level co-ranks of every output tile boundary, one warp per
 // boundary.  Tile j starts at global output j*T inside group G = j*T / 4w (T
 // divides 4w, g divides T).  f(m) = M1[m] <= M2[d-1-m] is true then false on

@@ -456,6 +456,50 @@ __global__ void nk2_partition(const uint32_t* __restrict__ src, PairGeom g, int 
     split[j] = (int)corank_global<K>(src + s, a_len, src + s + a_len, b_len, d0 - (s - g.org));
 }
 
+// First index in [a, b] where a monotone (true ... false) predicate on [a, b)
+// is false (b if none), found by one warp: every round the 32 lanes evaluate
+// f at 32 evenly spaced points (__ballot), shrinking the interval 33-fold.
+template <class F>
+__device__ __forceinline__ long long warp_first_false(long long a, long long b, F f) {
+    const int lane = threadIdx.x & 31;
+    while (a < b) {
+        const long long span = b - a;
+        const long long pos = a + ((lane + 1) * span) / 33;       // < b
+        const unsigned fm = __ballot_sync(0xffffffffu, !f(pos));
+        if (fm == 0) {
+            a = a + (32 * span) / 33 + 1;
+        } else {
+            const int L = __ffs(fm) - 1;
+            const long long posL = a + ((L + 1) * span) / 33;
+            const long long posP = L > 0 ? a + (L * span) / 33 : a - 1;
+            b = posL;
+            a = posP + 1;
+        }
+    }
+    return a;
+}
+
+// NK2, warp per tile (small, L2-resident inputs): the same co-rank found by a
+// 33-ary warp search -- ~log33(w) dependent rounds instead of log2(w).  Used
+// when the array fits in L2, where the extra probes cost no HBM traffic.
+template <class K>
+__global__ void nk2_partition_warp(const uint32_t* __restrict__ src, PairGeom g, int tout,
+                                   int num_tiles, int* __restrict__ split) {
+    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    if (j >= num_tiles) return;                       // warp-uniform
+    const long long d0 = (long long)j * tout;
+    long long s, a_len, b_len;
+    g.pair_of(d0, s, a_len, b_len);
+    const long long diag = d0 - (s - g.org);
+    const uint32_t* A = src + s;
+    const uint32_t* B = src + s + a_len;
+    const long long lo = max(0LL, diag - b_len), hi = min(diag, a_len);
+    const long long c = warp_first_false(lo, hi, [&](long long m) {
+        return !K::lt(__ldg(B + (diag - 1 - m)), __ldg(A + m));
+    });
+    if ((threadIdx.x & 31) == 0) split[j] = (int)c;
+}
+
 // ------------------------------------------------------------------ NK3
 // Stage global elements [g0, g1) (any alignment) into shared memory at word
 // offset `off` + (g0 & 3): TMA copies the 16-byte-aligned superset that lies

@@ -114,7 +114,8 @@ def test_schedule(n, kt, vals):
     p2 = dc.Plan(n)
     p2.set_two_level(True)
     s2 = p2.schedule(kt, vals)
-    assert s2["hbm_passes"] == (P if (vals or kt == "f32" or P < 2) else P % 2 + P // 2)
+    folds = not (vals or kt == "f32" or P < 2 or n < (1 << 23))   # small n: small tiles, one level
+    assert s2["hbm_passes"] == (P % 2 + P // 2 if folds else P)
     # fused + global levels cover the whole tree: ceil(log2 n) combine levels
     if n > 1:
         assert s["fused_levels"] + s["global_passes"] >= math.ceil(math.log2(n))
