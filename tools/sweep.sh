@@ -11,6 +11,6 @@ for spec in $1; do
 import json,sys
 d=json.loads(open('gpurun_out/sweep_$name.json').read().strip().splitlines()[-1])
 k=d.get('kernels', {})
-print('$name', round(d['ms_per_step'],4), 'ms', ' '.join(f\"{n}={v['avg_ms']*v['launches_per_step']:.4f}\" for n,v in k.items()), 'roof', round(d['roofline']['frac'],3))
+print('$name', round(d['ms_per_step'],4), 'ms', ' '.join(f\"{n}={v['avg_ms']*v['launches_per_step']:.4f}\" for n,v in k.items() if isinstance(v, dict)), 'roof', round(d['roofline']['frac'],3))
 " || tail -3 gpurun_out/sweep_$name.json
 done
