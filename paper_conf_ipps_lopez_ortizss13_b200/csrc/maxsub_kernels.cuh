@@ -15,6 +15,10 @@
 #pragma once
 #include <cstdint>
 
+#ifndef DC_MS_B4
+#define DC_MS_B4 8
+#endif
+
 namespace dc {
 
 // Identity ("empty segment") sentinel: |any real sum| <= 2^31 * 2^30 = 2^61.
@@ -193,9 +197,9 @@ nk4_maxsub(const int* __restrict__ x, long long n, dc_maxsub_tuple* __restrict__
         MsFold f;
         f.init();
         if (cbeg + C <= n) {
-            // batches of 32 elements (8 x 128-bit loads in flight), the next
+            // batches of 4*B4 elements (B4 x 128-bit loads in flight), the next
             // batch's loads issued before the current batch is folded
-            constexpr int B4 = 8;
+            constexpr int B4 = DC_MS_B4;
             static_assert(C % (4 * B4) == 0, "chunk must be whole batches");
             static_assert(C <= 256, "FP64 fold is exact only for chunks <= 2^8 elements");
             const int4* p4 = reinterpret_cast<const int4*>(x + cbeg);
