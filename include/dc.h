@@ -166,6 +166,23 @@ dc_status dc_maxsub_combine_async(dc_plan_t plan, const dc_maxsub_tuple *d_tuple
 /* Host buffers end to end: copy h_x to the device, run, return the result. */
 dc_status dc_run_maxsubarray_host(dc_plan_t plan, const int32_t *h_x, dc_maxsub_result *h_out);
 
+/* ---------------------------------------------- D&C sum */
+/* The paper's own D&C example, Alg 4: sum(a, size) recurses on
+ * the halves and combines with a[0] += a[size/2].  Third instance of the
+ * breadth-first O(1)-combine template include/dc_reduce.cuh (also usable
+ * with user monoids from CUDA code). */
+
+/* Exact int64 sum of d_x[0..n) (device int32).  Synchronises; *h_out. */
+dc_status dc_run_sum(dc_plan_t plan, const int32_t *d_x, int64_t *h_out);
+
+/* Enqueue-only variant writing the int64 result to device memory d_out. */
+dc_status dc_run_sum_async(dc_plan_t plan, const int32_t *d_x, int64_t *d_out);
+
+/* Alg 5 literally: one kernel launch per level, the id-th of m
+ * work-items computes a[id] <- a[id] + a[id+m]; d_work (device int64, n
+ * elements) is overwritten; synchronises and returns a[0] in *h_out. */
+dc_status dc_run_sum_alg5(dc_plan_t plan, int64_t *d_work, int64_t *h_out);
+
 /* ------------------------------------------- multi-GPU building blocks */
 /* The top log2(G) levels of a G-way sharded sort (not in
  * the paper, which notes the method "could easily be extended to multiple gpu

@@ -89,6 +89,12 @@ _SIGS.update({
     "dc_mg_merge_runs": ([_P, ctypes.c_int, _P, _P, _P, _P, _P, _I32], ctypes.c_int),
 })
 
+_SIGS.update({
+    "dc_run_sum": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
+    "dc_run_sum_async": ([_P, _P, _P], ctypes.c_int),
+    "dc_run_sum_alg5": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
+})
+
 #: kernel classes of dc_plan_kernel_time
 KERNELS = {"nk1_blocksort": 0, "nk2_partition": 1, "nk3_merge": 2, "nk4_maxsub": 3}
 
@@ -276,6 +282,30 @@ class Plan:
         _check(lib().dc_run_maxsubarray_host(self._h, x.data_ptr(), ctypes.byref(r)))
         return (r.sum, r.start, r.end)
 
+
+    # ---------------------------------------------------- D&C sum (f4)
+    def sum(self, x: torch.Tensor) -> int:
+        """Exact int64 sum of an int32 CUDA tensor (Alg 4 through dc_reduce.cuh)."""
+        _require_cuda(x, "x")
+        self._bind_stream(x)
+        r = _I64()
+        _check(lib().dc_run_sum(self._h, x.data_ptr(), ctypes.byref(r)))
+        return r.value
+
+    def sum_async(self, x: torch.Tensor, out: torch.Tensor) -> torch.Tensor:
+        _require_cuda(x, "x")
+        self._bind_stream(x)
+        _check(lib().dc_run_sum_async(self._h, x.data_ptr(), out.data_ptr()))
+        return out
+
+    def sum_alg5(self, work: torch.Tensor) -> int:
+        """Alg 5 literally (one launch per level) on an int64 CUDA work tensor (clobbered)."""
+        if not work.is_cuda or work.dtype != torch.int64:
+            raise ValueError("work must be a CUDA int64 tensor")
+        self._bind_stream(work)
+        r = _I64()
+        _check(lib().dc_run_sum_alg5(self._h, work.data_ptr(), ctypes.byref(r)))
+        return r.value
 
     # ------------------------------------------ multi-GPU building blocks
     def mg_sample(self, keys: torch.Tensor, stride: int) -> torch.Tensor:

@@ -16,6 +16,7 @@
 #include <vector>
 
 #include "dc.h"
+#include "dc_reduce.cuh"
 #include "maxsub_kernels.cuh"
 #include "mg_kernels.cuh"
 #include "sort_kernels.cuh"
@@ -144,6 +145,9 @@ struct dc_plan_s {
     // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
     // two-level partition costs 0.21 ms per pass vs 2 x 0.03.
     bool two_level = false;
+    // D&C sum (f4): per-CTA parts + ticket + result
+    long long* sum_state = nullptr;
+    int sum_grid = 0;
     // multi-GPU splitter state: bracket packs [64] lo, [64] hi, error flag
     unsigned long long* mg_state = nullptr;
     // host-buffer (end-to-end) staging
@@ -559,6 +563,32 @@ dc_status ensure_mg_state(dc_plan_t p) {
     return DC_OK;
 }
 
+
+// f4: the D&C sum through the generic O(1)-combine template (dc_reduce.cuh).
+constexpr int kSumThreads = 256;
+constexpr int kSumChunk = 64;
+
+dc_status ensure_sum_state(dc_plan_t p) {
+    if (p->sum_state) return DC_OK;
+    int dev = 0, sms = 148, occ = 4;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+        &occ, dc::breadth_first_reduce<dc::SumI64, kSumThreads, kSumChunk>, kSumThreads, 0);
+    const int64_t tiles = num_tiles(p->n, (int64_t)kSumThreads * kSumChunk);
+    const int64_t grid = (int64_t)sms * (occ > 0 ? occ : 1);
+    p->sum_grid = (int)(tiles < grid ? tiles : grid);
+    void* ptr = nullptr;
+    // parts[grid] | ticket (8 B) | result (8 B)
+    if (cudaMalloc(&ptr, (size_t)(p->sum_grid + 2) * 8) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(DC_ERR_OUT_OF_MEMORY, "sum state cudaMalloc failed");
+    }
+    p->sum_state = (long long*)ptr;
+    DC_CUDA(p, cudaMemsetAsync(ptr, 0, (size_t)(p->sum_grid + 2) * 8, p->stream));
+    return DC_OK;
+}
+
 }  // namespace
 
 // =================================================================== ABI
@@ -702,6 +732,7 @@ dc_status dc_free(dc_plan_t p) {
     if (p->ms_tiles) cudaFree(p->ms_tiles);
     if (p->d_stage) cudaFree(p->d_stage);
     if (p->mg_state) cudaFree(p->mg_state);
+    if (p->sum_state) cudaFree(p->sum_state);
     for (auto& gc : p->graphs) {
         if (gc.exec) cudaGraphExecDestroy(gc.exec);
         if (gc.graph) cudaGraphDestroy(gc.graph);
@@ -996,6 +1027,53 @@ dc_status dc_mg_merge_runs(dc_plan_t p, dc_key_type kt, uint32_t* d_in_keys, uin
                                                          nullptr, lens);
     }
     return fail(DC_ERR_INVALID_ARG, "unknown key type");
+}
+
+// --------------------------------------------------- D&C sum
+
+dc_status dc_run_sum_async(dc_plan_t p, const int32_t* d_x, int64_t* d_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (p->a != 2 || p->b != 2) return fail(DC_ERR_UNSUPPORTED, "runs need a == b == 2");
+    if (!d_x || !d_out) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    st = ensure_sum_state(p);
+    if (st != DC_OK) return st;
+    dc::breadth_first_reduce<dc::SumI64, kSumThreads, kSumChunk>
+        <<<p->sum_grid, kSumThreads, 0, p->stream>>>(
+            d_x, p->n, p->sum_state, (unsigned int*)(p->sum_state + p->sum_grid),
+            (long long*)d_out);
+    DC_LAUNCHED(p);
+    return DC_OK;
+}
+
+dc_status dc_run_sum(dc_plan_t p, const int32_t* d_x, int64_t* h_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!h_out) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    st = ensure_sum_state(p);
+    if (st != DC_OK) return st;
+    long long* d_res = p->sum_state + p->sum_grid + 1;
+    st = dc_run_sum_async(p, d_x, (int64_t*)d_res);
+    if (st != DC_OK) return st;
+    DC_CUDA(p, cudaMemcpyAsync(h_out, d_res, 8, cudaMemcpyDeviceToHost, p->stream));
+    DC_CUDA(p, cudaStreamSynchronize(p->stream));
+    return DC_OK;
+}
+
+dc_status dc_run_sum_alg5(dc_plan_t p, int64_t* d_work, int64_t* h_out) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!d_work || !h_out) return fail(DC_ERR_INVALID_ARG, "NULL argument");
+    for (long long len = p->n; len > 1;) {          // one launch per level (Alg 5)
+        const long long m = (len + 1) / 2;
+        dc::alg5_sum_level<<<(unsigned)((m + 255) / 256), 256, 0, p->stream>>>(
+            (long long*)d_work, len, m);
+        DC_LAUNCHED(p);
+        len = m;
+    }
+    DC_CUDA(p, cudaMemcpyAsync(h_out, d_work, 8, cudaMemcpyDeviceToHost, p->stream));
+    DC_CUDA(p, cudaStreamSynchronize(p->stream));
+    return DC_OK;
 }
 
 }  // extern "C"
