@@ -39,6 +39,7 @@ WORKLOADS = {
                 "sort_kv"),
     "sort_u32_small": ("mergesort of 2^20 uniform uint32 keys (configs[0])", 1 << 20, "sort"),
     "maxsub": ("max-subarray-sum D&C on 2^24 int32 values (configs[1])", 1 << 24, "maxsub"),
+    "sum": ("D&C sum (Alg 4, SURVEY f4) of 2^24 int32 values, exact int64", 1 << 24, "sum"),
     "sort_u32_2p30": ("mergesort of 2^30 uint32 keys sharded over N B200 (configs[4])", 1 << 30,
                       "sort"),
 }
@@ -261,6 +262,8 @@ def run_dc(args, wl):
     desc, n, kind = WORKLOADS[wl]
     if kind == "maxsub":
         return run_dc_maxsub(args, wl, desc, n)
+    if kind == "sum":
+        return run_dc_sum(args, wl, desc, n)
 
     kv = kind == "sort_kv"
     pristine_k = dcgen.sort_keys(n, args.dist, seed=3, device=dev)
@@ -479,6 +482,52 @@ def run_dc_maxsub(args, wl, desc, n):
         "e2e": {"value": n / (e2e_ms / 1e3), "unit": "elements/s", "ms_per_step": e2e_ms,
                 "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 24},
         "cpu_baseline": cpu,
+    }), flush=True)
+
+
+def run_dc_sum(args, wl, desc, n):
+    """f4 instance: the D&C sum through the generic O(1)-combine template."""
+    import torch
+
+    import dcgen
+    import paper_conf_ipps_lopez_ortizss13_b200 as dc
+
+    dev = torch.device("cuda", torch.cuda.current_device())
+    x = dcgen.maxsub_input(n, "uniform", seed=2, device=dev)
+    out = torch.empty(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    plan = dc.Plan(n)
+    stream = torch.cuda.current_stream(dev)
+    times = []
+    l0 = None
+    with ClockSampler(dev.index) as clk:
+        for i in range(args.warmup + args.steps):
+            flush.zero_()
+            if i == args.warmup:
+                l0 = plan.launch_count()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            plan.sum_async(x, out)
+            e1.record(stream)
+            if i >= args.warmup:
+                times.append((e0, e1))
+        torch.cuda.synchronize()
+    launches = plan.launch_count() - l0
+    ms = statistics.mean(a.elapsed_time(b) for a, b in times)
+    peak, src = peaks()
+    ach = 4 * n / (ms / 1e3) / 1e9
+    print(json.dumps({
+        "metric": "D&C sum elements/sec (2^24 int32, SURVEY f4)", "value": n / (ms / 1e3),
+        "unit": "elements/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "i32->i64", "data": "synthetic (counter-based splitmix64)",
+        "config": {"workload": wl, "description": desc, "n": n,
+                   "l2": "flushed before every step (512 MiB write)"},
+        "roofline": {"kernel": "breadth_first_reduce<SumI64> (one launch = the step)",
+                     "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
+                     "frac": ach / peak, "traffic": None, "avg_launch_ms": ms,
+                     "algorithmic_bytes_per_launch": 4 * n, "peak_source": src},
+        "gpu_launches": launches, "clocks": clk.summary(), "e2e": None, "cpu_baseline": None,
     }), flush=True)
 
 
