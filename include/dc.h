@@ -183,6 +183,28 @@ dc_status dc_run_sum_async(dc_plan_t plan, const int32_t *d_x, int64_t *d_out);
  * elements) is overwritten; synchronises and returns a[0] in *h_out. */
 dc_status dc_run_sum_alg5(dc_plan_t plan, int64_t *d_work, int64_t *h_out);
 
+/* ------------------------------------- work-division model */
+/* The paper's advanced hybrid work division (Sec. 5.2) for a D&C
+ * with f(m) = m^{log_b a} (mergesort: a = b = 2) on an HPU with p CPU cores,
+ * g GPU cores and CPU/GPU speed ratio gamma (0 < gamma < 1; Sec. 3.2).  A
+ * fraction alpha of the subproblems runs on the CPU; the GPU runs the rest
+ * from the leaves up to level y where both finish together (the closed forms
+ * of Sec. 5.2.2, three cases).  Host-only; INVALID_ARG for a,b < 2, p < 1,
+ * g < 1, gamma outside (0,1), n < 2 or alpha outside [p/n^{log_b a}, 1). */
+
+/* GPU share of the total work n^{log_b a}(log_b n + 1) for a given alpha, the
+ * level y reached by the GPU and the case (1, 2, 3) of Tg that applies. */
+dc_status dc_model_gpu_work(int32_t a, int32_t b, int32_t p, double g, double gamma, double n,
+                            double alpha, double *gpu_work_fraction, double *level_y,
+                            int32_t *model_case);
+
+/* alpha* maximising the GPU work ("numeric methods") and the
+ * corresponding share, level y and case.  The paper's example (a=b=2, p=4,
+ * g=2^12, gamma=1/160, n=2^24) gives alpha* ~ 0.16, ~52 %, y ~ 10. */
+dc_status dc_model_optimise(int32_t a, int32_t b, int32_t p, double g, double gamma, double n,
+                            double *alpha, double *gpu_work_fraction, double *level_y,
+                            int32_t *model_case);
+
 /* ------------------------------------------- multi-GPU building blocks */
 /* The top log2(G) levels of a G-way sharded sort (not in
  * the paper, which notes the method "could easily be extended to multiple gpu

@@ -95,6 +95,36 @@ _SIGS.update({
     "dc_run_sum_alg5": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
 })
 
+_D = ctypes.c_double
+_SIGS.update({
+    "dc_model_gpu_work": ([_I32, _I32, _I32, _D, _D, _D, _D, ctypes.POINTER(_D), ctypes.POINTER(_D),
+                           ctypes.POINTER(_I32)], ctypes.c_int),
+    "dc_model_optimise": ([_I32, _I32, _I32, _D, _D, _D, ctypes.POINTER(_D), ctypes.POINTER(_D),
+                           ctypes.POINTER(_D), ctypes.POINTER(_I32)], ctypes.c_int),
+})
+
+
+def model_gpu_work(a: int, b: int, p: int, g: float, gamma: float, n: float,
+                   alpha: float) -> dict:
+    """Paper Sec. 5.2 model: GPU work share, level y and case for a given alpha."""
+    f, y, c = ctypes.c_double(), ctypes.c_double(), _I32()
+    st = lib().dc_model_gpu_work(a, b, p, g, gamma, n, alpha, ctypes.byref(f), ctypes.byref(y),
+                                 ctypes.byref(c))
+    if st != 0:
+        raise DcError(st, "invalid model parameters")
+    return {"gpu_work_fraction": f.value, "level_y": y.value, "case": c.value}
+
+
+def model_optimise(a: int, b: int, p: int, g: float, gamma: float, n: float) -> dict:
+    """Paper Sec. 5.2 model: alpha* maximising the GPU work."""
+    al, f, y, c = ctypes.c_double(), ctypes.c_double(), ctypes.c_double(), _I32()
+    st = lib().dc_model_optimise(a, b, p, g, gamma, n, ctypes.byref(al), ctypes.byref(f),
+                                 ctypes.byref(y), ctypes.byref(c))
+    if st != 0:
+        raise DcError(st, "invalid model parameters")
+    return {"alpha": al.value, "gpu_work_fraction": f.value, "level_y": y.value, "case": c.value}
+
+
 #: kernel classes of dc_plan_kernel_time
 KERNELS = {"nk1_blocksort": 0, "nk2_partition": 1, "nk3_merge": 2, "nk4_maxsub": 3}
 
