@@ -316,7 +316,47 @@ def bench_main(args, wl, workloads, metric):
     ok = bool((keys[1:].to(torch.int64) & 0xFFFFFFFF >= keys[:-1].to(torch.int64) & 0xFFFFFFFF)
               .all())
     ms = statistics.mean(times)
+
+    # kernel breakdown (rank 0's own kernels): second loop with per-launch events
+    ops.plan.enable_timing(True)
+    for i in range(args.steps):
+        keys.copy_(pristine)
+        flush.zero_()
+        comm.barrier()
+        sort_(keys, None, comm, "u32", ops=ops)
+    torch.cuda.synchronize()
+    kt = ops.plan.kernel_times()
+    ops.plan.enable_timing(False)
+    nk3_ms, nk3_n = kt["nk3_merge"]
+    nk3_avg = nk3_ms / max(nk3_n, 1)
+
+    # end to end through the public API: pinned host shard -> device -> sort -> host
+    host = pristine.cpu().pin_memory()
+    back = torch.empty_like(host).pin_memory()
+    e2e = []
+    for i in range(args.warmup + args.steps):
+        comm.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        keys.copy_(host, non_blocking=True)
+        sort_(keys, None, comm, "u32", ops=ops)
+        back.copy_(keys, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if i >= args.warmup:
+            t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+            tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+            e2e.append(float(t.item()))
+    e2e_ms = statistics.mean(e2e)
+    peak = 6650.0
+    try:
+        peak = float(json.load(open(os.path.join(os.path.dirname(os.path.dirname(
+            os.path.abspath(__file__))), "MEASURED_PEAKS.json")))["hbm_gbs"])
+    except Exception:
+        pass
     if me == 0:
+        ach = 8 * m / (nk3_avg / 1e3) / 1e9 if nk3_n else None
         print(json.dumps({
             "metric": metric, "value": n_total / (ms / 1e3), "unit": "keys/s", "n_gpus": G,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
@@ -325,7 +365,16 @@ def bench_main(args, wl, workloads, metric):
             "config": {"workload": wl, "description": desc, "n": n_total, "per_gpu": m,
                        "dist": args.dist, "parallelism": f"key-range sharding x{G}",
                        "l2": "flushed before every step (512 MiB write)",
-                       "local_sorted_check": ok},
-            "gpu_launches": launches, "e2e": None, "cpu_baseline": None,
+                       "local_sorted_check": ok,
+                       "timing": "per-step CUDA events on every rank, max over ranks"},
+            "roofline": {"kernel": "nk3_merge (rank 0, local merge levels + G-way merge)",
+                         "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
+                         "frac": ach / peak if ach else None, "traffic": None,
+                         "avg_launch_ms": nk3_avg,
+                         "kernels_ms_per_step": {k: v[0] / args.steps for k, v in kt.items()}},
+            "gpu_launches": launches,
+            "e2e": {"value": n_total / (e2e_ms / 1e3), "unit": "keys/s", "ms_per_step": e2e_ms,
+                    "h2d_bytes_per_step": 4 * n_total, "d2h_bytes_per_step": 4 * n_total},
+            "cpu_baseline": None,
         }), flush=True)
     tdist.destroy_process_group()
