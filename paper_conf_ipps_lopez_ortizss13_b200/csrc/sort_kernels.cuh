@@ -282,7 +282,11 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
     const uint32_t SK = smem_addr(sk);
 #pragma unroll 1
     for (int w = IT; w < TILE; w *= 2) {
-        __syncthreads();
+        // Levels whose pairs fit in one warp (2w <= 32*IT) only touch that
+        // warp's own region: a warp barrier suffices and warps drift apart
+        // (search / merge / write phases overlap across warps).
+        const bool warp_local = 2 * w <= 32 * IT;
+        if (warp_local) __syncwarp(); else __syncthreads();
         {   // write this thread's IT ascending keys: A runs ascending, B runs descending
             const int pos = tid * IT;
             const int r = pos / w;                        // run index at width w
@@ -296,7 +300,7 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
                 for (int j = 0; j < IT; ++j) sk[pr + 2 * w - 1 - o - j] = k[j];
             }
         }
-        __syncthreads();
+        if (warp_local) __syncwarp(); else __syncthreads();
         const int tpg = (2 * w) / IT;                     // threads per merged pair
         const int s = (tid / tpg) * (2 * w);              // pair start
         const int diag = (tid % tpg) * IT;
