@@ -116,6 +116,14 @@ dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
  * while per-kernel timing is on.  Results are identical. */
 dc_status dc_plan_set_graphs(dc_plan_t plan, int32_t enable);
 
+/* Chunked pipeline of the one-level schedule (default 8 chunks; 0 or 1 = off):
+ * the array is cut into chunks of tile*2^k keys; each chunk's fused bottom
+ * levels and in-chunk merge levels run on a stream of their own, so chunks
+ * overlap (one chunk's HBM-bound merges with the next one's compute-bound
+ * NK1); the top log2(chunks) levels follow on the plan stream.  Not used
+ * while per-kernel timing is on.  Results are identical. */
+dc_status dc_plan_set_pipeline(dc_plan_t plan, int32_t chunks);
+
 /* Stream all device work of this plan is enqueued on (a cudaStream_t). */
 dc_status dc_plan_set_stream(dc_plan_t plan, void *cuda_stream);
 

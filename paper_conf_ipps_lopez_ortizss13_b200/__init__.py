@@ -59,6 +59,7 @@ _SIGS = {
                           ctypes.POINTER(_I32), ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_graphs": ([_P, _I32], ctypes.c_int),
+    "dc_plan_set_pipeline": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_stream": ([_P, _P], ctypes.c_int),
     "dc_plan_scratch_bytes": ([_P, _I32, ctypes.POINTER(ctypes.c_size_t)], ctypes.c_int),
     "dc_plan_set_scratch": ([_P, _P, ctypes.c_size_t], ctypes.c_int),
@@ -208,6 +209,10 @@ class Plan:
                                       ctypes.byref(h)))
         return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value,
                 "hbm_passes": h.value}
+
+    def set_pipeline(self, chunks: int) -> None:
+        """Chunked multi-stream pipeline of the one-level schedule (0/1 = off, default 8)."""
+        _check(lib().dc_plan_set_pipeline(self._h, chunks))
 
     def set_graphs(self, enable: bool) -> None:
         """CUDA-graph replay of the sort's launch sequence (default on)."""

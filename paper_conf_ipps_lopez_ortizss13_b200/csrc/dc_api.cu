@@ -10,7 +10,9 @@
 
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
+#include <algorithm>
 #include <new>
 #include <string>
 #include <vector>
@@ -140,6 +142,12 @@ struct dc_plan_s {
     bool use_graphs = true;
     std::vector<GraphCache> graphs;
     cudaStream_t cap_stream = nullptr;
+    // chunked pipeline: chunk c's fused bottom levels and in-chunk merge levels
+    // run on their own stream, so one chunk's HBM-bound merges overlap the next
+    // chunk's compute-bound NK1; the top levels follow on the plan stream.
+    int pipe_chunks = 8;
+    std::vector<cudaStream_t> pipe_streams;
+    std::vector<cudaEvent_t> pipe_events;   // [0] fork, [1..] per-chunk joins
     // two levels of the merge tree per HBM pass for keys-only sorts (f1).
     // Off by default: bit-exact, and its 4-way tile merge beats two one-level
     // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
@@ -233,17 +241,19 @@ cudaEvent_t take_event(dc_plan_t p) {
 struct TimedScope {
     dc_plan_t p;
     int kind;
+    cudaStream_t s;
     cudaEvent_t e0 = nullptr;
-    TimedScope(dc_plan_t p_, int kind_) : p(p_), kind(kind_) {
+    TimedScope(dc_plan_t p_, int kind_) : TimedScope(p_, kind_, p_->stream) {}
+    TimedScope(dc_plan_t p_, int kind_, cudaStream_t s_) : p(p_), kind(kind_), s(s_) {
         if (p->timing) {
             e0 = take_event(p);
-            cudaEventRecord(e0, p->stream);
+            cudaEventRecord(e0, s);
         }
     }
     ~TimedScope() {
         if (e0) {
             cudaEvent_t e1 = take_event(p);
-            cudaEventRecord(e1, p->stream);
+            cudaEventRecord(e1, s);
             p->pending.push_back({kind, e0, e1});
         }
     }
@@ -269,6 +279,20 @@ dc_status ensure_scratch(dc_plan_t p, bool vals) {
     p->scratch = ptr;
     p->scratch_bytes = need;
     p->own_scratch = true;
+    return DC_OK;
+}
+
+dc_status ensure_pipeline(dc_plan_t p, int chunks) {
+    while ((int)p->pipe_streams.size() < chunks) {
+        cudaStream_t st = nullptr;
+        DC_CUDA(p, cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+        p->pipe_streams.push_back(st);
+    }
+    while ((int)p->pipe_events.size() < chunks + 1) {
+        cudaEvent_t ev = nullptr;
+        DC_CUDA(p, cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        p->pipe_events.push_back(ev);
+    }
     return DC_OK;
 }
 
@@ -310,33 +334,87 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     uint32_t* oth_k = (passes % 2 == 0) ? sk : keys;
     uint32_t* oth_v = (passes % 2 == 0) ? sv : vals;
 
-    // NK1: base cases + fused bottom levels (reads the caller's buffer).
-    {
+    // One merge level over [org, end) on stream `st` (split region `sp`).
+    auto level = [&](int64_t org, int64_t end, int64_t w, int* sp, cudaStream_t st) -> dc_status {
+        const int tiles = (int)num_tiles(end - org, C.tout());
+        const dc::PairGeom g{org, w, w, end};
+        {
+            TimedScope ts(p, DC_KERNEL_NK2_PARTITION, st);
+            if (SMALL)   // L2-resident: 33-ary warp searches, few dependent rounds
+                dc::nk2_partition_warp<K><<<(tiles + 3) / 4, 128, 0, st>>>(cur_k, g, C.tout(),
+                                                                         tiles, sp);
+            else
+                dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, st>>>(cur_k, g, C.tout(),
+                                                                         tiles, sp);
+            DC_LAUNCHED(p);
+        }
+        {
+            TimedScope ts(p, DC_KERNEL_NK3_MERGE, st);
+            k3<<<tiles, C.nt3, nk3_smem_bytes(C, hv), st>>>(cur_k, cur_v, oth_k, oth_v, sp, g);
+            DC_LAUNCHED(p);
+        }
+        return DC_OK;
+    };
+
+    int64_t w = C.tile();
+    int lv = 0;
+    // Chunked pipeline (one-level schedule, not while timing kernels): the
+    // bottom `lc` levels of every chunk of tile*2^lc keys run on the chunk's
+    // own stream right after its NK1; chunks overlap each other.
+    int lc = 0, chunks = 1;
+    if (!SMALL && !two && !p->timing && p->pipe_chunks > 1) {
+        int lt = 0;
+        while ((1 << lt) < p->pipe_chunks) ++lt;
+        if (single > lt) {
+            lc = single - lt;
+            chunks = (int)num_tiles(n, (int64_t)C.tile() << lc);
+        }
+    }
+    if (chunks > 1) {
+        st = ensure_pipeline(p, chunks);
+        if (st != DC_OK) return st;
+        const int64_t clen = (int64_t)C.tile() << lc;
+        const size_t split_per = (size_t)num_tiles(clen, C.tout()) + 1;
+        DC_CUDA(p, cudaEventRecord(p->pipe_events[0], p->stream));
+        for (int c = 0; c < chunks; ++c) {
+            cudaStream_t cs = p->pipe_streams[c];
+            const int64_t org = c * clen, end = std::min(n, org + clen);
+            DC_CUDA(p, cudaStreamWaitEvent(cs, p->pipe_events[0], 0));
+            {
+                TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT, cs);
+                k1<<<(unsigned)num_tiles(end - org, C.tile()), C.nt1, nk1_smem_bytes(C, hv), cs>>>(
+                    keys + org, vals ? vals + org : nullptr, cur_k + org,
+                    cur_v ? cur_v + org : nullptr, end - org);
+                DC_LAUNCHED(p);
+            }
+            uint32_t *ck = cur_k, *cv = cur_v, *ok = oth_k, *ov = oth_v;
+            for (int l = 0; l < lc; ++l) {
+                st = level(org, end, (int64_t)C.tile() << l, split + c * split_per, cs);
+                if (st != DC_OK) return st;
+                std::swap(cur_k, oth_k);
+                std::swap(cur_v, oth_v);
+            }
+            cur_k = ck; cur_v = cv; oth_k = ok; oth_v = ov;   // same parity for every chunk
+            DC_CUDA(p, cudaEventRecord(p->pipe_events[1 + c], cs));
+        }
+        for (int c = 0; c < chunks; ++c)
+            DC_CUDA(p, cudaStreamWaitEvent(p->stream, p->pipe_events[1 + c], 0));
+        for (int l = 0; l < lc; ++l) {
+            std::swap(cur_k, oth_k);
+            std::swap(cur_v, oth_v);
+        }
+        w = (int64_t)C.tile() << lc;
+        lv = lc;
+    } else {
+        // NK1: base cases + fused bottom levels (reads the caller's buffer).
         TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT);
         k1<<<(unsigned)num_tiles(n, C.tile()), C.nt1, nk1_smem_bytes(C, hv), p->stream>>>(
             keys, vals, cur_k, cur_v, n);
         DC_LAUNCHED(p);
     }
-
-    int64_t w = C.tile();
-    const int tiles = (int)num_tiles(n, C.tout());
-    for (int lv = 0; lv < single; ++lv, w *= 2) {
-        {
-            TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-            if (SMALL)   // L2-resident: 33-ary warp searches, few dependent rounds
-                dc::nk2_partition_warp<K><<<(tiles + 3) / 4, 128, 0, p->stream>>>(
-                    cur_k, dc::PairGeom{0, w, w, n}, C.tout(), tiles, split);
-            else
-                dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
-                    cur_k, dc::PairGeom{0, w, w, n}, C.tout(), tiles, split);
-            DC_LAUNCHED(p);
-        }
-        {
-            TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-            k3<<<tiles, C.nt3, nk3_smem_bytes(C, hv), p->stream>>>(
-                cur_k, cur_v, oth_k, oth_v, split, dc::PairGeom{0, w, w, n});
-            DC_LAUNCHED(p);
-        }
+    for (; lv < single; ++lv, w *= 2) {
+        st = level(0, n, w, split, p->stream);
+        if (st != DC_OK) return st;
         std::swap(cur_k, oth_k);
         std::swap(cur_v, oth_v);
     }
@@ -626,6 +704,7 @@ dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t*
     p->a = a;
     p->b = b;
     p->base_size = base_size;
+    if (const char* e = std::getenv("DC_PIPE_CHUNKS")) p->pipe_chunks = std::atoi(e);  // tuning
     // Level i: a^i nodes of size ceil(n / b^i); stop at the first level whose
     // size is <= base_size (leaves at level log_b n for base 1).
     int64_t nodes = 1, size = n, bpow = 1;
@@ -689,6 +768,14 @@ dc_status dc_plan_set_two_level(dc_plan_t p, int32_t enable) {
     return DC_OK;
 }
 
+dc_status dc_plan_set_pipeline(dc_plan_t p, int32_t chunks) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (chunks < 0 || chunks > 64) return fail(DC_ERR_INVALID_ARG, "chunks must be in [0, 64]");
+    p->pipe_chunks = chunks;
+    drop_graphs(p);
+    return DC_OK;
+}
+
 dc_status dc_plan_set_graphs(dc_plan_t p, int32_t enable) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     p->use_graphs = enable != 0;
@@ -738,6 +825,8 @@ dc_status dc_free(dc_plan_t p) {
         if (gc.graph) cudaGraphDestroy(gc.graph);
     }
     if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
+    for (auto st : p->pipe_streams) cudaStreamDestroy(st);
+    for (auto ev : p->pipe_events) cudaEventDestroy(ev);
     delete p;
     return DC_OK;
 }

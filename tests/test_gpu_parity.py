@@ -143,6 +143,27 @@ def test_sort_graph_replay_same_buffers(dc, oracle_mod, n):
         assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev), seed
 
 
+@pytest.mark.parametrize("chunks", [0, 2, 3, 8, 16])
+@pytest.mark.parametrize("n,with_vals", [((1 << 24) + 12345, False), ((1 << 23) + 77, True)])
+def test_sort_chunked_pipeline(dc, oracle_mod, chunks, n, with_vals):
+    """Chunk streams (each chunk's NK1 + in-chunk levels) then the top levels."""
+    keys = dcgen.sort_keys(n, "few" if with_vals else "uniform", seed=19, device="cuda")
+    vals = dcgen.sort_vals(n, device="cuda") if with_vals else None
+    k_in = _np_keys(keys, "u32")
+    plan = dc.Plan(n)
+    plan.set_pipeline(chunks)
+    for rep in range(3):                 # eager, graph capture, graph replay
+        k = keys.clone()
+        v = vals.clone() if with_vals else None
+        plan.sort_(k, v, key_type="u32")
+        if with_vals:
+            ek, ev = oracle_mod.mergesort(k_in, np.arange(n, dtype=np.uint32))
+            assert np.array_equal(v.cpu().numpy().view(np.uint32), ev), rep
+        else:
+            ek = oracle_mod.mergesort(k_in)
+        assert np.array_equal(_np_keys(k, "u32"), ek), rep
+
+
 def test_sort_repeated_runs_same_plan(dc, oracle_mod):
     n = 50_000
     plan = dc.Plan(n)
