@@ -116,7 +116,8 @@ dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
  * while per-kernel timing is on.  Results are identical. */
 dc_status dc_plan_set_graphs(dc_plan_t plan, int32_t enable);
 
-/* Chunked pipeline of the one-level schedule (default 8 chunks; 0 or 1 = off):
+/* Chunked pipeline of the one-level schedule (default 1 = off; measured slower
+ * on B200):
  * the array is cut into chunks of tile*2^k keys; each chunk's fused bottom
  * levels and in-chunk merge levels run on a stream of their own, so chunks
  * overlap (one chunk's HBM-bound merges with the next one's compute-bound

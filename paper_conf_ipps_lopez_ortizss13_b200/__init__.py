@@ -211,7 +211,7 @@ class Plan:
                 "hbm_passes": h.value}
 
     def set_pipeline(self, chunks: int) -> None:
-        """Chunked multi-stream pipeline of the one-level schedule (0/1 = off, default 8)."""
+        """Chunked multi-stream pipeline of the one-level schedule (0/1 = off, the default)."""
         _check(lib().dc_plan_set_pipeline(self._h, chunks))
 
     def set_graphs(self, enable: bool) -> None:

@@ -143,9 +143,12 @@ struct dc_plan_s {
     std::vector<GraphCache> graphs;
     cudaStream_t cap_stream = nullptr;
     // chunked pipeline: chunk c's fused bottom levels and in-chunk merge levels
-    // run on their own stream, so one chunk's HBM-bound merges overlap the next
-    // chunk's compute-bound NK1; the top levels follow on the plan stream.
-    int pipe_chunks = 8;
+    // run on their own stream, so one chunk's HBM-bound merges could overlap
+    // the next chunk's compute-bound NK1; the top levels follow on the plan
+    // stream.  Off by default: measured slower at 2^28 (2/8/16 chunks: 7.51 /
+    // 7.12 / 6.79 ms vs 6.57) -- NK1 fills an SM's registers and shared memory,
+    // so the kernels split SMs instead of sharing them and NK3 loses bandwidth.
+    int pipe_chunks = 1;
     std::vector<cudaStream_t> pipe_streams;
     std::vector<cudaEvent_t> pipe_events;   // [0] fork, [1..] per-chunk joins
     // two levels of the merge tree per HBM pass for keys-only sorts (f1).
