@@ -254,6 +254,10 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // then fence_proxy_async_smem(); __syncthreads().
 __device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uint32_t* s, int h,
                                            int count) {
+#ifdef DC_NO_TMA_STORE   // sanitizer builds: compute-sanitizer initcheck does not track TMA writes
+    for (int e = threadIdx.x; e < count; e += blockDim.x) dst[e] = s[h + e];
+    return;
+#endif
     const int head = min(count, (4 - h) & 3);              // words before the aligned body
     const int body = (count - head) & ~3;
     if (threadIdx.x == 0 && body > 0) {
