@@ -11,5 +11,5 @@ for tool in memcheck racecheck synccheck initcheck; do
   [ "$tool" = "initcheck" ] && lib="DC_LIB=/tmp/dc_notma.so"
   env $lib timeout 1500 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_run.py $extra \
     > gpurun_out/sanitize_$tool.txt 2>&1
-  echo "$tool rc=$? $(grep -E 'ERROR SUMMARY|sanitize_run ok' gpurun_out/sanitize_$tool.txt | tr '\n' ' ')"
+  echo "$tool rc=$? $(grep -E 'SUMMARY|sanitize_run ok' gpurun_out/sanitize_$tool.txt | tr '\n' ' ')"
 done
