@@ -152,6 +152,21 @@ dc_status dc_run_mergesort(dc_plan_t plan, dc_key_type key_type, void *d_keys,
 dc_status dc_run_mergesort_host(dc_plan_t plan, dc_key_type key_type, void *h_keys,
                                 uint32_t *h_vals);
 
+/* Streaming end-to-end sorts of HOST buffers (pinned for overlap).  Each
+ * submission copies h_in_keys (+h_in_vals) into one of two plan-owned device
+ * slots, sorts there and copies the result to h_out_keys (+h_out_vals); the
+ * host input is not modified.  Work of consecutive submissions overlaps: the
+ * upload of one, the sort of the previous and the download of the one before
+ * run on separate streams (PCIe is full duplex).  A submission starts after
+ * the work already enqueued on the plan stream.  Returns after enqueueing;
+ * the host buffers must stay valid until dc_sort_host_wait returns. */
+dc_status dc_sort_host_submit(dc_plan_t plan, dc_key_type key_type, const void *h_in_keys,
+                              const uint32_t *h_in_vals, void *h_out_keys, uint32_t *h_out_vals);
+
+/* Waits (host) until every submitted host sort has written its output; the
+ * plan stream is also made to wait for them. */
+dc_status dc_sort_host_wait(dc_plan_t plan);
+
 /* ----------------------------------------------------------- max-subarray */
 
 /* Max subarray of d_x[0..n) (device int32).  Synchronises; writes *h_out. */

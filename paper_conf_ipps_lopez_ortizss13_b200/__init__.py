@@ -60,6 +60,8 @@ _SIGS = {
     "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_graphs": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_pipeline": ([_P, _I32], ctypes.c_int),
+    "dc_sort_host_submit": ([_P, ctypes.c_int, _P, _P, _P, _P], ctypes.c_int),
+    "dc_sort_host_wait": ([_P], ctypes.c_int),
     "dc_plan_set_stream": ([_P, _P], ctypes.c_int),
     "dc_plan_scratch_bytes": ([_P, _I32, ctypes.POINTER(ctypes.c_size_t)], ctypes.c_int),
     "dc_plan_set_scratch": ([_P, _P, ctypes.c_size_t], ctypes.c_int),
@@ -276,6 +278,30 @@ class Plan:
         _check(lib().dc_run_mergesort_host(self._h, kt, keys.data_ptr(),
                                            None if vals is None else vals.data_ptr()))
         return keys
+
+    def sort_host_submit(self, keys_in: torch.Tensor, keys_out: torch.Tensor,
+                         vals_in: torch.Tensor | None = None,
+                         vals_out: torch.Tensor | None = None, key_type: str | None = None):
+        """Streaming end-to-end sort of pinned HOST tensors (input unmodified).
+
+        Consecutive submissions overlap (upload / sort / download on separate
+        streams); call :meth:`sort_host_wait` before reading the outputs."""
+        for t in (keys_in, keys_out, vals_in, vals_out):
+            if t is not None and (t.is_cuda or t.numel() != self.n):
+                raise ValueError("host tensors of n elements expected")
+        _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
+        _check(lib().dc_sort_host_submit(self._h, _key_type(keys_in, key_type),
+                                         keys_in.data_ptr(),
+                                         None if vals_in is None else vals_in.data_ptr(),
+                                         keys_out.data_ptr(),
+                                         None if vals_out is None else vals_out.data_ptr()))
+        self._host_refs = getattr(self, "_host_refs", [])[-4:] + [
+            (keys_in, keys_out, vals_in, vals_out)]
+
+    def sort_host_wait(self) -> None:
+        _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
+        _check(lib().dc_sort_host_wait(self._h))
+        self._host_refs = []
 
     def max_subarray(self, x: torch.Tensor) -> tuple[int, int, int]:
         _require_cuda(x, "x")

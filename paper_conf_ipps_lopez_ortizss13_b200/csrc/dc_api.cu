@@ -164,6 +164,16 @@ struct dc_plan_s {
     // host-buffer (end-to-end) staging
     void* d_stage = nullptr;
     size_t d_stage_bytes = 0;
+    // streaming host sorts: two device slots, copy-in / compute / copy-out streams
+    struct HostSlot {
+        void* d = nullptr;              // keys [n] (+ vals [n])
+        size_t bytes = 0;
+        cudaEvent_t in_done = nullptr, sort_done = nullptr, out_done = nullptr;
+    };
+    HostSlot hslot[2];
+    cudaStream_t h2d = nullptr, d2h = nullptr, comp = nullptr;
+    cudaEvent_t join_in = nullptr, join_out = nullptr;   // order against the plan stream
+    int64_t submits = 0;
     // per-kernel CUDA-event timing (instrumentation, off by default)
     bool timing = false;
     struct Timed { int kind; cudaEvent_t e0, e1; };
@@ -821,6 +831,17 @@ dc_status dc_free(dc_plan_t p) {
     if (p->scratch && p->own_scratch) cudaFree(p->scratch);
     if (p->ms_tiles) cudaFree(p->ms_tiles);
     if (p->d_stage) cudaFree(p->d_stage);
+    for (auto& hs : p->hslot) {
+        if (hs.d) cudaFree(hs.d);
+        if (hs.in_done) cudaEventDestroy(hs.in_done);
+        if (hs.sort_done) cudaEventDestroy(hs.sort_done);
+        if (hs.out_done) cudaEventDestroy(hs.out_done);
+    }
+    if (p->join_in) cudaEventDestroy(p->join_in);
+    if (p->join_out) cudaEventDestroy(p->join_out);
+    if (p->h2d) cudaStreamDestroy(p->h2d);
+    if (p->d2h) cudaStreamDestroy(p->d2h);
+    if (p->comp) cudaStreamDestroy(p->comp);
     if (p->mg_state) cudaFree(p->mg_state);
     if (p->sum_state) cudaFree(p->sum_state);
     for (auto& gc : p->graphs) {
@@ -1165,6 +1186,82 @@ dc_status dc_run_sum_alg5(dc_plan_t p, int64_t* d_work, int64_t* h_out) {
     }
     DC_CUDA(p, cudaMemcpyAsync(h_out, d_work, 8, cudaMemcpyDeviceToHost, p->stream));
     DC_CUDA(p, cudaStreamSynchronize(p->stream));
+    return DC_OK;
+}
+
+// ------------------------------------------- streaming end-to-end sorts
+
+dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys,
+                              const uint32_t* h_in_vals, void* h_out_keys, uint32_t* h_out_vals) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (p->a != 2 || p->b != 2) return fail(DC_ERR_UNSUPPORTED, "runs need a == b == 2");
+    if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
+        return fail(DC_ERR_INVALID_ARG, "unknown key type");
+    if (!h_in_keys || !h_out_keys || (h_in_vals == nullptr) != (h_out_vals == nullptr))
+        return fail(DC_ERR_INVALID_ARG, "bad host buffers");
+    if (!p->h2d) {
+        DC_CUDA(p, cudaStreamCreateWithFlags(&p->h2d, cudaStreamNonBlocking));
+        DC_CUDA(p, cudaStreamCreateWithFlags(&p->d2h, cudaStreamNonBlocking));
+        DC_CUDA(p, cudaStreamCreateWithFlags(&p->comp, cudaStreamNonBlocking));
+        DC_CUDA(p, cudaEventCreateWithFlags(&p->join_in, cudaEventDisableTiming));
+        DC_CUDA(p, cudaEventCreateWithFlags(&p->join_out, cudaEventDisableTiming));
+        for (auto& hs : p->hslot) {
+            DC_CUDA(p, cudaEventCreateWithFlags(&hs.in_done, cudaEventDisableTiming));
+            DC_CUDA(p, cudaEventCreateWithFlags(&hs.sort_done, cudaEventDisableTiming));
+            DC_CUDA(p, cudaEventCreateWithFlags(&hs.out_done, cudaEventDisableTiming));
+            DC_CUDA(p, cudaEventRecord(hs.out_done, p->d2h));
+        }
+    }
+    auto& hs = p->hslot[p->submits & 1];
+    const size_t kb = align_up((size_t)p->n * 4, 256);
+    const size_t need = h_in_vals ? 2 * kb : kb;
+    if (hs.bytes < need) {
+        DC_CUDA(p, cudaEventSynchronize(hs.out_done));
+        if (hs.d) cudaFree(hs.d);
+        hs.d = nullptr;
+        if (cudaMalloc(&hs.d, need) != cudaSuccess) {
+            cudaGetLastError();
+            hs.bytes = 0;
+            return fail(DC_ERR_OUT_OF_MEMORY, "host-sort slot cudaMalloc failed");
+        }
+        hs.bytes = need;
+    }
+    uint32_t* dk = (uint32_t*)hs.d;
+    uint32_t* dv = h_in_vals ? (uint32_t*)((char*)hs.d + kb) : nullptr;
+    const size_t bytes = (size_t)p->n * 4;
+    // copy in after the work already queued on the plan stream, and once the
+    // slot's previous result has left
+    DC_CUDA(p, cudaEventRecord(p->join_in, p->stream));
+    DC_CUDA(p, cudaStreamWaitEvent(p->h2d, p->join_in, 0));
+    DC_CUDA(p, cudaStreamWaitEvent(p->h2d, hs.out_done, 0));
+    DC_CUDA(p, cudaMemcpyAsync(dk, h_in_keys, bytes, cudaMemcpyHostToDevice, p->h2d));
+    if (dv) DC_CUDA(p, cudaMemcpyAsync(dv, h_in_vals, bytes, cudaMemcpyHostToDevice, p->h2d));
+    DC_CUDA(p, cudaEventRecord(hs.in_done, p->h2d));
+    // sort on the compute stream (sorts of the two slots serialise: shared scratch)
+    DC_CUDA(p, cudaStreamWaitEvent(p->comp, hs.in_done, 0));
+    cudaStream_t user = p->stream;
+    p->stream = p->comp;
+    st = sort_dispatch(p, kt, dk, dv);
+    p->stream = user;
+    if (st != DC_OK) return st;
+    DC_CUDA(p, cudaEventRecord(hs.sort_done, p->comp));
+    // copy out
+    DC_CUDA(p, cudaStreamWaitEvent(p->d2h, hs.sort_done, 0));
+    DC_CUDA(p, cudaMemcpyAsync(h_out_keys, dk, bytes, cudaMemcpyDeviceToHost, p->d2h));
+    if (dv) DC_CUDA(p, cudaMemcpyAsync(h_out_vals, dv, bytes, cudaMemcpyDeviceToHost, p->d2h));
+    DC_CUDA(p, cudaEventRecord(hs.out_done, p->d2h));
+    p->submits++;
+    return DC_OK;
+}
+
+dc_status dc_sort_host_wait(dc_plan_t p) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    if (!p->d2h) return DC_OK;
+    DC_CUDA(p, cudaEventRecord(p->join_out, p->d2h));
+    DC_CUDA(p, cudaStreamWaitEvent(p->stream, p->join_out, 0));   // the plan stream joins
+    DC_CUDA(p, cudaStreamSynchronize(p->d2h));
     return DC_OK;
 }
 

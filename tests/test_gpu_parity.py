@@ -185,6 +185,29 @@ def test_sort_host_buffers(dc, oracle_mod):
     assert np.array_equal(vals.numpy().view(np.uint32), ev)
 
 
+@pytest.mark.parametrize("with_vals", [False, True])
+def test_sort_host_streaming(dc, oracle_mod, with_vals):
+    """Streaming submissions (two device slots, overlapped copies) of several
+    distinct inputs; the inputs stay unmodified, each output is its own sort."""
+    n = 3 * 8192 + 1001 if not with_vals else (1 << 23) + 77
+    plan = dc.Plan(n)
+    ins = [dcgen.sort_keys(n, d, seed=s).pin_memory()
+           for s, d in enumerate(["uniform", "few", "reverse", "paper", "uniform"])]
+    keep = [t.clone() for t in ins]
+    outs = [torch.empty_like(t).pin_memory() for t in ins]
+    vin = dcgen.sort_vals(n).pin_memory() if with_vals else None
+    vouts = [torch.empty_like(vin).pin_memory() if with_vals else None for _ in ins]
+    for t, o, vo in zip(ins, outs, vouts):
+        plan.sort_host_submit(t, o, vin, vo, key_type="u32")
+    plan.sort_host_wait()
+    for t, k, o, vo in zip(ins, keep, outs, vouts):
+        assert torch.equal(t, k)
+        ek, ev = oracle_mod.mergesort(_np_keys(k, "u32"), np.arange(n, dtype=np.uint32))
+        assert np.array_equal(_np_keys(o, "u32"), ek)
+        if with_vals:
+            assert np.array_equal(vo.numpy().view(np.uint32), ev)
+
+
 def test_sort_2pow24_against_oracle(dc, oracle_mod):
     n = 1 << 24
     k_in, k_out, v_out = run_sort(dc, n, "uniform", with_vals=True, seed=3)
