@@ -253,7 +253,7 @@ def run_dc(args, wl):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
+    if world > 1 or os.environ.get("DC_BENCH_DIST"):   # DC_BENCH_DIST=1: that path at N=1
         from paper_conf_ipps_lopez_ortizss13_b200 import dist as dcdist
 
         return dcdist.bench_main(args, wl, WORKLOADS, METRIC)

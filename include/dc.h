@@ -47,7 +47,7 @@ typedef enum {
     DC_ERR_UNSUPPORTED = 2,   /* valid request this build cannot run (a!=2) */
     DC_ERR_OUT_OF_MEMORY = 3, /* scratch allocation failed                    */
     DC_ERR_CUDA = 4,          /* a CUDA runtime call or kernel failed        */
-    DC_ERR_NCCL = 5,          /* reserved: collectives run in torch.distributed */
+    DC_ERR_NCCL = 5,          /* NCCL missing or a collective failed         */
     DC_ERR_BAD_STATE = 6      /* plan poisoned by an earlier CUDA error       */
 } dc_status;
 
@@ -229,13 +229,69 @@ dc_status dc_model_optimise(int32_t a, int32_t b, int32_t p, double g, double ga
                             double *alpha, double *gpu_work_fraction, double *level_y,
                             int32_t *model_case);
 
+/* ------------------------------------------------ multi-GPU (rows a7-a10) */
+/* One process (or, for tests, one thread) per GPU.  With a communicator set,
+ * the plan's n is the GLOBAL problem size; every rank passes its shard of
+ * m = n/world elements, the global positions [rank*m, (rank+1)*m):
+ *   dc_run_mergesort   sorts the shard locally (levels >= log2 world), then
+ *                      runs the top log2(world) levels of the merge tree as
+ *                      ONE exchange ("could easily be extended to
+ *                      multiple gpu cards"; the single-transfer principle of
+ *                      P:L474-478): exact composite-order splitters from an
+ *                      all-gather of samples, an all-reduce of their counts and
+ *                      an all-gather of bracketing windows; one host sync for
+ *                      the split sizes; one all-to-all of keys (+ values); a
+ *                      local stable G-way merge.  On exit rank r holds global
+ *                      positions [r*m, (r+1)*m) of the stable sorted order.
+ *   dc_run_maxsubarray returns the global result (indices are global
+ *                      positions): per-rank summary tuple -> all-gather ->
+ *                      ordered combine.
+ * Collectives are enqueued on the plan stream.  All ranks must make the same
+ * calls in the same order.  Host-buffer entry points are single-GPU only
+ * (DC_ERR_UNSUPPORTED with a communicator). */
+
+/* 128 opaque bytes identifying a new NCCL communicator; create on one rank and
+ * broadcast (e.g. torch.distributed.broadcast_object_list).  NCCL is loaded
+ * at run time (the copy already in the process, else libnccl.so.2, else
+ * $DC_NCCL_LIB); DC_ERR_NCCL if it cannot be. */
+dc_status dc_get_unique_id(uint8_t id[128]);
+
+/* Joins the NCCL communicator `id` as `rank` of `world` (collective: blocks
+ * until every rank has joined; call with the plan's device current).  Must
+ * precede the plan's first run; n % world == 0 required (DC_ERR_INVALID_ARG).
+ * world == 1 is allowed (the single-GPU path). */
+dc_status dc_plan_set_comm(dc_plan_t plan, const uint8_t id[128], int32_t rank, int32_t world);
+
+/* In-process loopback group: `world` ranks that are threads of one process
+ * sharing one GPU, with the collectives done by device copies between their
+ * buffers.  Same protocol and kernels as NCCL; used to test the multi-GPU path
+ * on a single GPU.  Free after every member plan has been freed. */
+typedef struct dc_loopback_s *dc_loopback_t;
+dc_status dc_loopback_create(int32_t world, dc_loopback_t *out);
+dc_status dc_loopback_free(dc_loopback_t group);
+/* Joins `group` as `rank` (not collective).  Same preconditions as
+ * dc_plan_set_comm.  A member that fails aborts the group: the others then
+ * return DC_ERR_NCCL instead of waiting (and after 120 s in any case). */
+dc_status dc_plan_set_loopback(dc_plan_t plan, dc_loopback_t group, int32_t rank);
+
+/* Communicator of a plan: rank, world and shard size m (1, 0, n without). */
+dc_status dc_plan_comm_info(dc_plan_t plan, int32_t *rank, int32_t *world, int64_t *shard_n);
+
+/* Sample stride S of the splitter search (default 4096; windows hold < S keys;
+ * world*S*4 <= 200 KiB).  Set before a run, the same on every rank. */
+dc_status dc_plan_set_mg_stride(dc_plan_t plan, int64_t stride);
+
+/* Split matrix of the last multi-GPU sort: h_cmat[r*(world+1) + d] = number of
+ * rank-r elements among the first d*m of the global stable order. */
+dc_status dc_plan_last_splits(dc_plan_t plan, int64_t *h_cmat);
+
 /* ------------------------------------------- multi-GPU building blocks */
 /* The top log2(G) levels of a G-way sharded sort (not in
  * the paper, which notes the method "could easily be extended to multiple gpu
  * cards").  Rank r holds global positions [r*m, (r+1)*m) and has
- * sorted them with dc_run_mergesort.  The collectives between these steps
- * run in torch.distributed (NCCL over NVLink); these calls are the per-rank
- * device work.  All are enqueue-only on the plan stream unless stated.
+ * sorted them with dc_run_mergesort.  These are the per-rank device steps
+ * of the protocol above, exposed for callers that run the collectives
+ * themselves (e.g. in torch.distributed; dist.py).  All are enqueue-only on the plan stream unless stated.
  * Composite order: element (key, rank, position) -- the global stable order.
  */
 

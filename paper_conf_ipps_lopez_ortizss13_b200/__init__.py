@@ -10,13 +10,18 @@ if the library is missing or no CUDA device is present, calls raise.
     dc.max_subarray(x) -> (sum, start, end)
     dc.Plan(n)                            # explicit plan: level table, schedule, runs
 
-Multi-GPU (one process per GPU, torch.distributed/NCCL): see :mod:`.dist`.
+Multi-GPU (one process per GPU): ``plan = dc.init_dist(n)`` binds a plan of
+global size n to a library-owned NCCL communicator; ``plan.sort_(shard)`` then
+runs the whole distributed sort in the library.  :mod:`.dist` composes the
+same per-rank steps over any torch.distributed group (gloo tests).
 """
 from __future__ import annotations
 
+import atexit
 import ctypes
 import os
 import subprocess
+import weakref
 
 import torch
 
@@ -24,7 +29,7 @@ from . import build as _build
 
 __all__ = [
     "DcError", "Plan", "sort_", "max_subarray", "lib", "KEY_U32", "KEY_I32", "KEY_F32",
-    "MaxsubResult", "MaxsubTuple",
+    "MaxsubResult", "MaxsubTuple", "get_unique_id", "init_dist", "LoopbackGroup",
 ]
 
 KEY_U32, KEY_I32, KEY_F32 = 0, 1, 2
@@ -90,6 +95,18 @@ _SIGS.update({
     "dc_mg_split_matrix": ([_P, ctypes.c_int, _P, _I32, _I64, _I64, _P], ctypes.c_int),
     "dc_mg_error": ([_P, ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_mg_merge_runs": ([_P, ctypes.c_int, _P, _P, _P, _P, _P, _I32], ctypes.c_int),
+})
+
+_SIGS.update({
+    "dc_get_unique_id": ([_P], ctypes.c_int),
+    "dc_plan_set_comm": ([_P, _P, _I32, _I32], ctypes.c_int),
+    "dc_loopback_create": ([_I32, ctypes.POINTER(_P)], ctypes.c_int),
+    "dc_loopback_free": ([_P], ctypes.c_int),
+    "dc_plan_set_loopback": ([_P, _P, _I32], ctypes.c_int),
+    "dc_plan_comm_info": ([_P, ctypes.POINTER(_I32), ctypes.POINTER(_I32), ctypes.POINTER(_I64)],
+                          ctypes.c_int),
+    "dc_plan_set_mg_stride": ([_P, _I64], ctypes.c_int),
+    "dc_plan_last_splits": ([_P, _P], ctypes.c_int),
 })
 
 _SIGS.update({
@@ -188,12 +205,17 @@ class Plan:
         _check(lib().dc_plan(n, a, b, base_size, ctypes.byref(h)))
         self._h = h
         self.n, self.a, self.b, self.base_size = n, a, b, base_size
+        _live_plans.add(self)
 
-    def __del__(self):
+    def close(self) -> None:
+        """Free the plan's device state now (idempotent; also done by GC / at exit)."""
         h = getattr(self, "_h", None)
         if h is not None and _lib is not None:
             _lib.dc_free(h)
-            self._h = None
+        self._h = None
+
+    def __del__(self):
+        self.close()
 
     def levels(self) -> list[tuple[int, int]]:
         """[(nodes a^i, size ceil(n/b^i)) for each level i]."""
@@ -211,6 +233,38 @@ class Plan:
                                       ctypes.byref(h)))
         return {"tile": t.value, "fused_levels": f.value, "global_passes": p.value,
                 "hbm_passes": h.value}
+
+    # ------------------------------------------------ library communicator
+    def _attached(self) -> None:
+        r, w, m = _I32(), _I32(), _I64()
+        _check(lib().dc_plan_comm_info(self._h, ctypes.byref(r), ctypes.byref(w), ctypes.byref(m)))
+        self.rank, self.world, self.n_global, self.n = r.value, w.value, self.n, m.value
+
+    def set_comm(self, uid: bytes, rank: int, world: int) -> None:
+        """Join the NCCL communicator ``uid`` (from :func:`get_unique_id`) as
+        ``rank`` of ``world``; afterwards ``self.n`` is this rank's shard size
+        and sort_ / max_subarray run the multi-GPU method (include/dc.h)."""
+        if len(uid) != 128:
+            raise ValueError("unique id must be 128 bytes")
+        buf = ctypes.create_string_buffer(bytes(uid), 128)
+        _check(lib().dc_plan_set_comm(self._h, buf, rank, world))
+        self._attached()
+
+    def set_loopback(self, group: "LoopbackGroup", rank: int) -> None:
+        """Join an in-process loopback group (threads sharing one GPU; tests)."""
+        _check(lib().dc_plan_set_loopback(self._h, group._h, rank))
+        self._group = group            # the group outlives its member plans
+        self._attached()
+
+    def set_mg_stride(self, stride: int) -> None:
+        _check(lib().dc_plan_set_mg_stride(self._h, stride))
+
+    def last_splits(self) -> list[list[int]]:
+        """Split matrix c[r][d] of the last multi-GPU sort (world x (world+1))."""
+        w = getattr(self, "world", 1)
+        buf = (_I64 * (w * (w + 1)))()
+        _check(lib().dc_plan_last_splits(self._h, buf))
+        return [list(buf[r * (w + 1):(r + 1) * (w + 1)]) for r in range(w)]
 
     def set_pipeline(self, chunks: int) -> None:
         """Chunked multi-stream pipeline of the one-level schedule (0/1 = off, the default)."""
@@ -423,6 +477,61 @@ class Plan:
                                       None if out_vals is None else out_vals.data_ptr(),
                                       lens, len(run_len)))
         return out_keys
+
+
+# Plans (then groups) still alive at interpreter exit -- e.g. held by a
+# traceback cycle -- are freed before the CUDA runtime is torn down.
+_live_plans: "weakref.WeakSet[Plan]" = weakref.WeakSet()
+_live_groups: "weakref.WeakSet[LoopbackGroup]" = weakref.WeakSet()
+
+
+@atexit.register
+def _free_at_exit() -> None:
+    for p in list(_live_plans):
+        p.close()
+    for g in list(_live_groups):
+        g.close()
+
+
+def get_unique_id() -> bytes:
+    """128-byte NCCL unique id for :meth:`Plan.set_comm` (create on one rank)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().dc_get_unique_id(buf))
+    return buf.raw
+
+
+class LoopbackGroup:
+    """``world`` ranks as threads of this process sharing one GPU (dc_loopback_*)."""
+
+    def __init__(self, world: int):
+        h = _P()
+        _check(lib().dc_loopback_create(world, ctypes.byref(h)))
+        self._h, self.world = h, world
+        _live_groups.add(self)
+
+    def close(self) -> None:
+        h = getattr(self, "_h", None)
+        if h is not None and _lib is not None:
+            _lib.dc_loopback_free(h)
+        self._h = None
+
+    def __del__(self):
+        self.close()
+
+
+def init_dist(n: int, group=None) -> Plan:
+    """Plan of global size n bound to a library-owned NCCL communicator over
+    the torch.distributed group (rank 0 creates the id, broadcast by torch).
+    Set the CUDA device of this rank first."""
+    import torch.distributed as tdist
+
+    rank, world = tdist.get_rank(group), tdist.get_world_size(group)
+    obj = [get_unique_id() if rank == 0 else None]
+    tdist.broadcast_object_list(obj, src=tdist.get_global_rank(group, 0) if group else 0,
+                                group=group)
+    plan = Plan(n)
+    plan.set_comm(obj[0], rank, world)
+    return plan
 
 
 _plans: dict = {}

@@ -18,6 +18,7 @@
 #include <vector>
 
 #include "dc.h"
+#include "plan.h"
 #include "dc_reduce.cuh"
 #include "maxsub_kernels.cuh"
 #include "mg_kernels.cuh"
@@ -114,74 +115,6 @@ int nk3_smem_bytes(SortCfg c, bool vals) {
 
 }  // namespace
 
-struct dc_plan_s {
-    int64_t n = 0;
-    int32_t a = 2, b = 2;
-    int64_t base_size = 1;
-    std::vector<int64_t> nodes, sizes;
-    cudaStream_t stream = nullptr;
-    bool bad = false;
-    int64_t launches = 0;
-    // scratch (keys ping-pong, values ping-pong, partition array)
-    void* scratch = nullptr;
-    size_t scratch_bytes = 0;
-    bool own_scratch = false;
-    // max-subarray state
-    dc_maxsub_tuple* ms_tiles = nullptr;
-    unsigned int* ms_ticket = nullptr;
-    dc_maxsub_result* ms_res = nullptr;
-    // CUDA graphs of the sort's launch sequence, per (keys, vals, key type)
-    struct GraphCache {
-        uint32_t* keys;
-        uint32_t* vals;
-        dc_key_type kt;
-        cudaGraph_t graph;
-        cudaGraphExec_t exec;
-        int64_t launches;
-    };
-    bool use_graphs = true;
-    std::vector<GraphCache> graphs;
-    cudaStream_t cap_stream = nullptr;
-    // chunked pipeline: chunk c's fused bottom levels and in-chunk merge levels
-    // run on their own stream, so one chunk's HBM-bound merges could overlap
-    // the next chunk's compute-bound NK1; the top levels follow on the plan
-    // stream.  Off by default: measured slower at 2^28 (2/8/16 chunks: 7.51 /
-    // 7.12 / 6.79 ms vs 6.57) -- NK1 fills an SM's registers and shared memory,
-    // so the kernels split SMs instead of sharing them and NK3 loses bandwidth.
-    int pipe_chunks = 1;
-    std::vector<cudaStream_t> pipe_streams;
-    std::vector<cudaEvent_t> pipe_events;   // [0] fork, [1..] per-chunk joins
-    // two levels of the merge tree per HBM pass for keys-only sorts (f1).
-    // Off by default: bit-exact, and its 4-way tile merge beats two one-level
-    // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
-    // two-level partition costs 0.21 ms per pass vs 2 x 0.03.
-    bool two_level = false;
-    // D&C sum (f4): per-CTA parts + ticket + result
-    long long* sum_state = nullptr;
-    int sum_grid = 0;
-    // multi-GPU splitter state: bracket packs [64] lo, [64] hi, error flag
-    unsigned long long* mg_state = nullptr;
-    // host-buffer (end-to-end) staging
-    void* d_stage = nullptr;
-    size_t d_stage_bytes = 0;
-    // streaming host sorts: two device slots, copy-in / compute / copy-out streams
-    struct HostSlot {
-        void* d = nullptr;              // keys [n] (+ vals [n])
-        size_t bytes = 0;
-        cudaEvent_t in_done = nullptr, sort_done = nullptr, out_done = nullptr;
-    };
-    HostSlot hslot[2];
-    cudaStream_t h2d = nullptr, d2h = nullptr, comp = nullptr;
-    cudaEvent_t join_in = nullptr, join_out = nullptr;   // order against the plan stream
-    int64_t submits = 0;
-    // per-kernel CUDA-event timing (instrumentation, off by default)
-    bool timing = false;
-    struct Timed { int kind; cudaEvent_t e0, e1; };
-    std::vector<Timed> pending;
-    std::vector<cudaEvent_t> event_pool;
-    double acc_ms[DC_KERNEL_COUNT] = {0};
-    int64_t acc_n[DC_KERNEL_COUNT] = {0};
-};
 
 namespace {
 
@@ -682,6 +615,14 @@ dc_status ensure_sum_state(dc_plan_t p) {
 
 }  // namespace
 
+namespace dcx {
+dc_status fail(dc_status s, const std::string& msg) { return ::fail(s, msg); }
+dc_status cuda_fail(dc_plan_t p, cudaError_t e, const char* what) { return ::cuda_fail(p, e, what); }
+dc_status local_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
+    return sort_dispatch(p, kt, keys, vals);
+}
+}  // namespace dcx
+
 // =================================================================== ABI
 
 extern "C" {
@@ -714,6 +655,7 @@ dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t*
     dc_plan_s* p = new (std::nothrow) dc_plan_s();
     if (!p) return fail(DC_ERR_OUT_OF_MEMORY, "plan allocation failed");
     p->n = n;
+    p->n_global = n;
     p->a = a;
     p->b = b;
     p->base_size = base_size;
@@ -823,6 +765,7 @@ dc_status dc_plan_set_scratch(dc_plan_t p, void* d, size_t bytes) {
 
 dc_status dc_free(dc_plan_t p) {
     if (!p) return DC_OK;
+    if (p->mg) dcx::mg_destroy(p->mg);
     for (auto& t : p->pending) {
         cudaEventDestroy(t.e0);
         cudaEventDestroy(t.e1);
@@ -891,7 +834,15 @@ dc_status dc_plan_kernel_time(dc_plan_t p, int32_t kernel, double* total_ms, int
     return DC_OK;
 }
 
+static dc_status run_mergesort(dc_plan_t p, dc_key_type kt, void* d_keys, uint32_t* d_vals);
+
 dc_status dc_run_mergesort(dc_plan_t p, dc_key_type kt, void* d_keys, uint32_t* d_vals) {
+    const dc_status st = run_mergesort(p, kt, d_keys, d_vals);
+    if (st != DC_OK && p && p->mg) dcx::mg_abort(p->mg);   // release the other ranks
+    return st;
+}
+
+static dc_status run_mergesort(dc_plan_t p, dc_key_type kt, void* d_keys, uint32_t* d_vals) {
     dc_status st = check_plan(p);
     if (st != DC_OK) return st;
     if (p->a != 2 || p->b != 2)
@@ -900,6 +851,7 @@ dc_status dc_run_mergesort(dc_plan_t p, dc_key_type kt, void* d_keys, uint32_t* 
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
     if (!d_keys || !aligned16(d_keys)) return fail(DC_ERR_INVALID_ARG, "keys NULL or misaligned");
     if (d_vals && !aligned16(d_vals)) return fail(DC_ERR_INVALID_ARG, "vals misaligned");
+    if (p->mg) return dcx::mg_sort(p, kt, (uint32_t*)d_keys, d_vals);
     return sort_dispatch(p, kt, (uint32_t*)d_keys, d_vals);
 }
 
@@ -911,6 +863,7 @@ dc_status dc_run_mergesort_host(dc_plan_t p, dc_key_type kt, void* h_keys, uint3
     if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
     if (!h_keys) return fail(DC_ERR_INVALID_ARG, "keys NULL");
+    if (p->mg) return fail(DC_ERR_UNSUPPORTED, "host-buffer sorts are single-GPU");
     size_t kb = align_up((size_t)p->n * 4, 256);
     st = ensure_stage(p, h_vals ? 2 * kb : kb);
     if (st != DC_OK) return st;
@@ -949,8 +902,14 @@ dc_status dc_run_maxsubarray_tuple_async(dc_plan_t p, const int32_t* d_x, int64_
 
 dc_status dc_run_maxsubarray(dc_plan_t p, const int32_t* d_x, dc_maxsub_result* h_out) {
     dc_status st = check_plan(p);
-    if (st != DC_OK) return st;
-    if (!h_out) return fail(DC_ERR_INVALID_ARG, "out NULL");
+    if (st == DC_OK && !h_out) st = fail(DC_ERR_INVALID_ARG, "out NULL");
+    if (st == DC_OK && p->mg && (!d_x || !aligned16(d_x)))
+        st = fail(DC_ERR_INVALID_ARG, "x NULL or misaligned");
+    if (st != DC_OK) {
+        if (p && p->mg) dcx::mg_abort(p->mg);
+        return st;
+    }
+    if (p->mg) return dcx::mg_maxsub(p, d_x, h_out);
     st = ensure_ms_state(p);
     if (st != DC_OK) return st;
     st = dc_run_maxsubarray_async(p, d_x, 0, p->ms_res);
@@ -1200,6 +1159,7 @@ dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
     if (!h_in_keys || !h_out_keys || (h_in_vals == nullptr) != (h_out_vals == nullptr))
         return fail(DC_ERR_INVALID_ARG, "bad host buffers");
+    if (p->mg) return fail(DC_ERR_UNSUPPORTED, "host-buffer sorts are single-GPU");
     if (!p->h2d) {
         DC_CUDA(p, cudaStreamCreateWithFlags(&p->h2d, cudaStreamNonBlocking));
         DC_CUDA(p, cudaStreamCreateWithFlags(&p->d2h, cudaStreamNonBlocking));

@@ -12,7 +12,11 @@ log2(G) levels become one exchange step:
   a9  local stable G-way merge of the received runs (kernels);
   a10 max-subarray: per-rank summary tuple -> all-gather -> ordered combine.
 
-Collectives go through a tiny interface (:class:`Comm`): :class:`TorchComm`
+The product path for N GPUs is the library-owned runtime (``init_dist`` /
+dc_plan_set_comm: the same steps in C++ over NCCL); this module composes the
+per-rank steps over any torch.distributed group, which is how the protocol's
+host logic is tested on CPU with gloo.  Collectives go through a tiny
+interface (:class:`Comm`): :class:`TorchComm`
 wraps a torch.distributed process group (NCCL on GPUs; gloo in the CPU tests)
 and :class:`LoopbackComm` runs G virtual ranks as threads in one process on
 one GPU (the 1-GPU test of the whole protocol).  Every step on the data runs
@@ -270,7 +274,11 @@ def max_subarray(x: torch.Tensor, comm: Comm | None = None, ops=None):
 # ------------------------------------------------------------ N>1 bench
 
 def bench_main(args, wl, workloads, metric):
-    """bench.py under torchrun: 2^30 keys sharded over WORLD_SIZE GPUs (configs[4])."""
+    """bench.py under torchrun: 2^30 keys sharded over WORLD_SIZE GPUs (configs[4]).
+
+    The product path: a plan of the global size bound to a library-owned NCCL
+    communicator (``init_dist``); every step is one ``dc_run_mergesort`` per
+    rank -- local levels, splitters, all-to-all and G-way merge in the library."""
     import json
     import os
     import statistics
@@ -279,54 +287,68 @@ def bench_main(args, wl, workloads, metric):
 
     import dcgen
 
+    from . import init_dist
+
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
-    tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    comm = TorchComm()
-    G, me = comm.world, comm.rank
+    dev = torch.device("cuda", local)
+    tdist.init_process_group("nccl", device_id=dev)
+    G, me = tdist.get_world_size(), tdist.get_rank()
     desc, n_total, kind = workloads[wl]
     if n_total % G:
         raise SystemExit("n must be divisible by the number of GPUs")
-    m = n_total // G
-    dev = torch.device("cuda", local)
+    plan = init_dist(n_total)
+    m = plan.n
     pristine = dcgen.sort_keys(n_total, args.dist, seed=5, start=me * m, count=m, device=dev)
     keys = torch.empty_like(pristine)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-    ops = DcOps(m)
     stream = torch.cuda.current_stream(dev)
+
+    def max_over_ranks(ms):
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        return float(t.item())
+
     times = []
     l0 = None
     for i in range(args.warmup + args.steps):
         keys.copy_(pristine)
         flush.zero_()
         if i == args.warmup:
-            l0 = ops.launches()
-        comm.barrier()
+            l0 = plan.launch_count()
+        tdist.barrier()
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        sort_(keys, None, comm, "u32", ops=ops)
+        plan.sort_(keys, key_type="u32")
         e1.record(stream)
         torch.cuda.synchronize()
         if i >= args.warmup:
-            t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-            tdist.all_reduce(t, op=tdist.ReduceOp.MAX)                # max over ranks
-            times.append(float(t.item()))
-    launches = ops.launches() - l0
-    ok = bool((keys[1:].to(torch.int64) & 0xFFFFFFFF >= keys[:-1].to(torch.int64) & 0xFFFFFFFF)
-              .all())
+            times.append(max_over_ranks(e0.elapsed_time(e1)))
+    launches = plan.launch_count() - l0
+    u = keys.to(torch.int64) & 0xFFFFFFFF
+    desc_at = torch.nonzero(u[1:] < u[:-1]).flatten()
+    unsorted = int(desc_at.numel())
+    first_desc = desc_at[:4].tolist()
+    ends = torch.stack([u[0], u[-1]])                  # rank boundaries: last(r) <= first(r+1)
+    allends = torch.empty(2 * G, dtype=ends.dtype, device=dev)
+    tdist.all_gather_into_tensor(allends, ends)
+    e = allends.view(G, 2).cpu()
+    boundaries_ok = bool(all(e[r, 1] <= e[r + 1, 0] for r in range(G - 1)))
+    del u, desc_at
     ms = statistics.mean(times)
+    splits = plan.last_splits() if G > 1 else [[0, m]]
 
     # kernel breakdown (rank 0's own kernels): second loop with per-launch events
-    ops.plan.enable_timing(True)
+    plan.enable_timing(True)
     for i in range(args.steps):
         keys.copy_(pristine)
         flush.zero_()
-        comm.barrier()
-        sort_(keys, None, comm, "u32", ops=ops)
+        tdist.barrier()
+        plan.sort_(keys, key_type="u32")
     torch.cuda.synchronize()
-    kt = ops.plan.kernel_times()
-    ops.plan.enable_timing(False)
+    kt = plan.kernel_times()
+    plan.enable_timing(False)
     nk3_ms, nk3_n = kt["nk3_merge"]
     nk3_avg = nk3_ms / max(nk3_n, 1)
 
@@ -335,19 +357,17 @@ def bench_main(args, wl, workloads, metric):
     back = torch.empty_like(host).pin_memory()
     e2e = []
     for i in range(args.warmup + args.steps):
-        comm.barrier()
+        tdist.barrier()
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         keys.copy_(host, non_blocking=True)
-        sort_(keys, None, comm, "u32", ops=ops)
+        plan.sort_(keys, key_type="u32")
         back.copy_(keys, non_blocking=True)
         e1.record(stream)
         torch.cuda.synchronize()
         if i >= args.warmup:
-            t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-            tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
-            e2e.append(float(t.item()))
+            e2e.append(max_over_ranks(e0.elapsed_time(e1)))
     e2e_ms = statistics.mean(e2e)
     peak = 6650.0
     try:
@@ -355,6 +375,7 @@ def bench_main(args, wl, workloads, metric):
             os.path.abspath(__file__))), "MEASURED_PEAKS.json")))["hbm_gbs"])
     except Exception:
         pass
+    moved = sum(splits[me][d + 1] - splits[me][d] for d in range(G) if d != me)
     if me == 0:
         ach = 8 * m / (nk3_avg / 1e3) / 1e9 if nk3_n else None
         print(json.dumps({
@@ -364,8 +385,10 @@ def bench_main(args, wl, workloads, metric):
             "data": "synthetic (counter-based splitmix64)",
             "config": {"workload": wl, "description": desc, "n": n_total, "per_gpu": m,
                        "dist": args.dist, "parallelism": f"key-range sharding x{G}",
+                       "runtime": "library-owned NCCL communicator (dc_plan_set_comm)",
                        "l2": "flushed before every step (512 MiB write)",
-                       "local_sorted_check": ok,
+                       "local_descents": unsorted, "first_descents": first_desc,
+                       "rank_boundaries_ordered": boundaries_ok, "rank0_keys_sent": moved,
                        "timing": "per-step CUDA events on every rank, max over ranks"},
             "roofline": {"kernel": "nk3_merge (rank 0, local merge levels + G-way merge)",
                          "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
@@ -377,4 +400,5 @@ def bench_main(args, wl, workloads, metric):
                     "h2d_bytes_per_step": 4 * n_total, "d2h_bytes_per_step": 4 * n_total},
             "cpu_baseline": None,
         }), flush=True)
+    plan.close()
     tdist.destroy_process_group()

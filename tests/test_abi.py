@@ -131,3 +131,44 @@ def test_scratch_is_the_papers_2n_working_space():
     assert n * 4 + n * 4 <= n * 4 + extra             # input + scratch >= 2n ints
     assert (n * 4 + extra) - ws["bytes"] < 0.01 * ws["bytes"]   # ... and not much more
     assert p.scratch_bytes(True) >= 2 * n * 4
+
+
+# ------------------------------------------------ library communicator (host side)
+
+def test_unique_id_is_128_bytes():
+    a, b = dc.get_unique_id(), dc.get_unique_id()
+    assert len(a) == 128 and len(b) == 128 and a != b
+
+
+def test_comm_info_without_communicator():
+    p = dc.Plan(12345)
+    r, w, m = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int64()
+    assert dc.lib().dc_plan_comm_info(p._h, ctypes.byref(r), ctypes.byref(w), ctypes.byref(m)) == 0
+    assert (r.value, w.value, m.value) == (0, 1, 12345)
+    buf = (ctypes.c_int64 * 4)()
+    assert dc.lib().dc_plan_last_splits(p._h, buf) == 1          # no multi-GPU sort yet
+
+
+@pytest.mark.parametrize("rank,world,n", [(0, 0, 1000), (-1, 2, 1000), (2, 2, 1000),
+                                          (0, 3, 1000)])
+def test_set_comm_validates_before_joining(rank, world, n):
+    """Invalid rank / world / divisibility is rejected before NCCL is touched
+    (a valid call would block in ncclCommInitRank waiting for the peers)."""
+    p = dc.Plan(n)
+    uid = ctypes.create_string_buffer(dc.get_unique_id(), 128)
+    assert dc.lib().dc_plan_set_comm(p._h, uid, rank, world) == 1
+    assert dc.lib().dc_plan_set_comm(p._h, None, 0, 1) == 1
+
+
+def test_set_comm_rejects_non_binary_plans():
+    p = dc.Plan(1024, 4, 4, 1)
+    uid = ctypes.create_string_buffer(dc.get_unique_id(), 128)
+    assert dc.lib().dc_plan_set_comm(p._h, uid, 0, 2) == 2
+
+
+def test_mg_stride_range():
+    p = dc.Plan(1000)
+    assert dc.lib().dc_plan_set_mg_stride(p._h, 0) == 1
+    assert dc.lib().dc_plan_set_mg_stride(p._h, 1 << 21) == 1
+    assert dc.lib().dc_plan_set_mg_stride(p._h, 1024) == 0
+    assert dc.lib().dc_loopback_free(None) == 0

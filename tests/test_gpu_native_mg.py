@@ -1,0 +1,198 @@
+"""The library-owned multi-GPU runtime (dc_plan_set_comm / dc_plan_set_loopback,
+rows a7-a10 + b) on one GPU.
+
+A loopback group runs G ranks as threads of this process, each with its own
+plan and CUDA stream; the collectives are device copies between their buffers,
+the protocol and kernels are the ones NCCL runs use.  The rank outputs,
+concatenated in rank order, must equal the CPU oracle's stable sort /
+max-subarray of the whole input, bit for bit.  NCCL itself is exercised at
+world 1 (one GPU per gpurun box).
+"""
+import threading
+
+import numpy as np
+import pytest
+import torch
+
+import dcgen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def dc():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_lopez_ortizss13_b200 as m
+    return m
+
+
+def run_ranks(dc, n, world, fn, stride=None):
+    """fn(plan, rank, m) on `world` threads joined to one loopback group."""
+    group = dc.LoopbackGroup(world)
+    plans = []
+    for r in range(world):
+        p = dc.Plan(n)
+        if stride:
+            p.set_mg_stride(stride)
+        p.set_loopback(group, r)
+        plans.append(p)
+    results, errors = [None] * world, [None] * world
+
+    def body(r):
+        try:
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                results[r] = fn(plans[r], r, plans[r].n)
+                s.synchronize()
+        except BaseException as e:   # noqa: BLE001 - surfaced by the caller
+            errors[r] = e.with_traceback(None)   # no frame cycle keeping plans alive
+
+    threads = [threading.Thread(target=body, args=(r,)) for r in range(world)]
+    for t in threads:
+        t.start()
+    for t in threads:
+        t.join(timeout=300)
+    return results, errors, plans
+
+
+def _view(a, key_type):
+    return a.view({"u32": np.uint32, "i32": np.int32, "f32": np.float32}[key_type])
+
+
+def sort_case(dc, oracle_mod, n, world, dist_name, key_type, with_vals, stride=None, seed=31):
+    def fn(plan, r, m):
+        keys = dcgen.sort_keys(n, dist_name, seed=seed, key_type=key_type, start=r * m, count=m,
+                               device="cuda")
+        vals = dcgen.sort_vals(n, start=r * m, count=m, device="cuda") if with_vals else None
+        plan.sort_(keys, vals, key_type=key_type)
+        return keys.cpu(), (vals.cpu() if with_vals else None), plan.last_splits()
+
+    res, errs, plans = run_ranks(dc, n, world, fn, stride)
+    for e in errs:
+        if e is not None:
+            raise e
+    full = dcgen.sort_keys(n, dist_name, seed=seed, key_type=key_type).numpy()
+    ek, ev = oracle_mod.mergesort(_view(full, key_type), np.arange(n, dtype=np.uint32),
+                                  key_type=key_type)
+    got = torch.cat([r[0] for r in res]).numpy()
+    assert np.array_equal(got.view(np.uint32), ek.view(np.uint32))
+    if with_vals:
+        assert np.array_equal(torch.cat([r[1] for r in res]).numpy().view(np.uint32), ev)
+    # every rank computed the same split matrix; its columns partition [0, n)
+    cm = np.array(res[0][2])
+    for r in res[1:]:
+        assert np.array_equal(np.array(r[2]), cm)
+    m = n // world
+    assert np.array_equal(cm.sum(axis=0), np.arange(world + 1) * m)
+    assert np.all(np.diff(cm, axis=1) >= 0)
+    return cm
+
+
+@pytest.mark.parametrize("world", [2, 3, 4, 8])
+@pytest.mark.parametrize("dist_name", ["uniform", "few", "sorted", "reverse", "equal"])
+def test_loopback_kv(dc, oracle_mod, world, dist_name):
+    sort_case(dc, oracle_mod, world * 100_003, world, dist_name, "u32", True)
+
+
+@pytest.mark.parametrize("key_type", ["u32", "i32", "f32"])
+@pytest.mark.parametrize("stride", [64, 1000, 4096])
+def test_loopback_keys_only(dc, oracle_mod, key_type, stride):
+    sort_case(dc, oracle_mod, 4 * 250_001, 4, "paper", key_type, False, stride)
+
+
+def test_loopback_large_shards(dc, oracle_mod):
+    """2^24 keys over 4 ranks: 4M-key shards use the full-size tile config."""
+    sort_case(dc, oracle_mod, 1 << 24, 4, "uniform", "u32", False)
+
+
+def test_loopback_equal_keys_split_exactly(dc, oracle_mod):
+    """All keys equal: the stable order is (rank, position), so rank r keeps its
+    own shard and nothing moves."""
+    world = 4
+    cm = sort_case(dc, oracle_mod, world * 70_001, world, "equal", "u32", True)
+    m = 70_001
+    for r in range(world):
+        assert cm[r][r + 1] - cm[r][r] == m
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 8])
+@pytest.mark.parametrize("kind", ["uniform", "negative", "small"])
+def test_loopback_maxsub(dc, oracle_mod, world, kind):
+    n = world * 300_007
+
+    def fn(plan, r, m):
+        x = dcgen.maxsub_input(n, kind, seed=5, start=r * m, count=m, device="cuda")
+        return plan.max_subarray(x)
+
+    res, errs, _ = run_ranks(dc, n, world, fn)
+    for e in errs:
+        if e is not None:
+            raise e
+    full = dcgen.maxsub_input(n, kind, seed=5).numpy()
+    expect = tuple(int(v) for v in oracle_mod.maxsub(full))
+    for r in res:
+        assert tuple(r) == expect
+
+
+def test_loopback_failing_member_releases_others(dc):
+    """A rank whose call fails validation aborts the group: the other rank gets
+    DC_ERR_NCCL promptly instead of waiting in a barrier."""
+    n = 2 * 50_000
+    lib = dc.lib()
+
+    def fn(plan, r, m):
+        keys = dcgen.sort_keys(n, "uniform", seed=1, start=r * m, count=m, device="cuda")
+        if r == 1:
+            st = lib.dc_run_mergesort(plan._h, 7, keys.data_ptr(), None)   # bad key type
+            assert st == 1
+            return "failed"
+        plan.sort_(keys)
+        return "sorted"
+
+    import time
+    t0 = time.time()
+    res, errs, _ = run_ranks(dc, n, 2, fn)
+    assert time.time() - t0 < 60
+    assert res[1] == "failed"
+    assert isinstance(errs[0], dc.DcError) and errs[0].status == 5
+
+
+def test_comm_validation(dc):
+    g = dc.LoopbackGroup(2)
+    p = dc.Plan(1001)
+    with pytest.raises(dc.DcError):              # n % world != 0
+        p.set_loopback(g, 0)
+    p = dc.Plan(1000)
+    with pytest.raises(dc.DcError):
+        p.set_loopback(g, 2)                     # rank out of range
+    p.set_loopback(g, 0)
+    assert (p.rank, p.world, p.n, p.n_global) == (0, 2, 500, 1000)
+    q = dc.Plan(1000)
+    with pytest.raises(dc.DcError):              # rank already joined
+        q.set_loopback(g, 0)
+    with pytest.raises(dc.DcError):              # second communicator
+        p.set_loopback(g, 1)
+    r = dc.Plan(1024)
+    r.sort_(dcgen.sort_keys(1024, "uniform", seed=1, device="cuda"))
+    with pytest.raises(dc.DcError):              # after the first run
+        r.set_loopback(g, 1)
+    with pytest.raises(dc.DcError):              # host-buffer paths are single-GPU
+        p.sort_host_(torch.zeros(500, dtype=torch.int32).pin_memory())
+
+
+def test_nccl_world1_sort_and_maxsub(dc, oracle_mod):
+    """NCCL communicator of one rank: dlopen, unique id, init, collectives."""
+    n = 3 * 8192 + 101
+    p = dc.Plan(n)
+    p.set_comm(dc.get_unique_id(), 0, 1)
+    assert (p.rank, p.world, p.n) == (0, 1, n)
+    keys = dcgen.sort_keys(n, "few", seed=4, device="cuda")
+    vals = dcgen.sort_vals(n, device="cuda")
+    k_in = keys.cpu().numpy().view(np.uint32)
+    p.sort_(keys, vals)
+    ek, ev = oracle_mod.mergesort(k_in, np.arange(n, dtype=np.uint32))
+    assert np.array_equal(keys.cpu().numpy().view(np.uint32), ek)
+    assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)
+    x = dcgen.maxsub_input(n, "uniform", seed=8, device="cuda")
+    assert p.max_subarray(x) == tuple(int(v) for v in oracle_mod.maxsub(x.cpu().numpy()))
