@@ -281,6 +281,20 @@ dc_status dc_plan_comm_info(dc_plan_t plan, int32_t *rank, int32_t *world, int64
  * world*S*4 <= 200 KiB).  Set before a run, the same on every rank. */
 dc_status dc_plan_set_mg_stride(dc_plan_t plan, int64_t stride);
 
+/* Exchange of the multi-GPU sort.  enable != 0 (default): FUSED -- every
+ * rank sorts its shard into a plan-owned buffer that all peers map (CUDA IPC
+ * over NVLink/NVSwitch; plain pointers in a loopback group), and the first
+ * round of the G-way merge reads the runs straight from the peers' buffers
+ * (dc_mg_merge_peers), then a stream-ordered barrier; no all-to-all, no
+ * receive buffer write.  enable == 0: NCCL all-to-all, then the local merge.
+ * Set before the first sort, the same on every rank; if any rank cannot map
+ * every peer, all ranks fall back to the all-to-all (decided collectively at
+ * the first sort).  $DC_MG_P2P=0/1 overrides. */
+dc_status dc_plan_set_mg_p2p(dc_plan_t plan, int32_t enable);
+
+/* Exchange in use: 1 fused, -1 all-to-all, 0 not decided yet / no communicator. */
+dc_status dc_plan_mg_exchange_mode(dc_plan_t plan, int32_t *mode);
+
 /* Split matrix of the last multi-GPU sort: h_cmat[r*(world+1) + d] = number of
  * rank-r elements among the first d*m of the global stable order. */
 dc_status dc_plan_last_splits(dc_plan_t plan, int64_t *h_cmat);
@@ -344,6 +358,22 @@ dc_status dc_mg_error(dc_plan_t plan, int32_t *h_err);
 dc_status dc_mg_merge_runs(dc_plan_t plan, dc_key_type key_type, uint32_t *d_in_keys,
                            uint32_t *d_in_vals, uint32_t *d_out_keys, uint32_t *d_out_vals,
                            const int64_t *h_run_len, int32_t runs);
+
+/* a8+a9 fused: stable merge of `runs` sorted runs that live in separate
+ * buffers -- in the multi-GPU sort, the sorted shards of the peer GPUs, read
+ * directly over NVLink, so the exchange overlaps the merge tile by tile and
+ * no receive buffer is written.  Run r is h_len[r] elements at offset
+ * h_off[r] of the buffer h_run_keys[r] (+ h_run_vals[r]; host arrays of
+ * device pointers, 16-byte aligned, readable for h_bound[r] elements; the
+ * pointers may be peer mappings).  Earlier runs win ties.  Output:
+ * d_out_keys (+ d_out_vals), sum(h_len) <= plan n elements.  With more than
+ * two runs the first round writes d_tmp_* (n elements each) and later rounds
+ * are local.  Enqueue-only. */
+dc_status dc_mg_merge_peers(dc_plan_t plan, dc_key_type key_type,
+                            const uint32_t *const *h_run_keys, const uint32_t *const *h_run_vals,
+                            const int64_t *h_bound, const int64_t *h_off, const int64_t *h_len,
+                            int32_t runs, uint32_t *d_tmp_keys, uint32_t *d_tmp_vals,
+                            uint32_t *d_out_keys, uint32_t *d_out_vals);
 
 /* ------------------------------------------------------ instrumentation */
 

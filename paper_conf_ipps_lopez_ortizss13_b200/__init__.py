@@ -107,6 +107,10 @@ _SIGS.update({
                           ctypes.c_int),
     "dc_plan_set_mg_stride": ([_P, _I64], ctypes.c_int),
     "dc_plan_last_splits": ([_P, _P], ctypes.c_int),
+    "dc_plan_set_mg_p2p": ([_P, _I32], ctypes.c_int),
+    "dc_plan_mg_exchange_mode": ([_P, ctypes.POINTER(_I32)], ctypes.c_int),
+    "dc_mg_merge_peers": ([_P, ctypes.c_int, _P, _P, _P, _P, _P, _I32, _P, _P, _P, _P],
+                          ctypes.c_int),
 })
 
 _SIGS.update({
@@ -258,6 +262,15 @@ class Plan:
 
     def set_mg_stride(self, stride: int) -> None:
         _check(lib().dc_plan_set_mg_stride(self._h, stride))
+
+    def set_mg_p2p(self, enable: bool) -> None:
+        """Fused exchange (merge reads the peers' shards) vs NCCL all-to-all."""
+        _check(lib().dc_plan_set_mg_p2p(self._h, int(enable)))
+
+    def exchange_mode(self) -> str:
+        m = _I32()
+        _check(lib().dc_plan_mg_exchange_mode(self._h, ctypes.byref(m)))
+        return {1: "fused", -1: "all_to_all", 0: "undecided"}[m.value]
 
     def last_splits(self) -> list[list[int]]:
         """Split matrix c[r][d] of the last multi-GPU sort (world x (world+1))."""
@@ -464,6 +477,25 @@ class Plan:
         e = _I32()
         _check(lib().dc_mg_error(self._h, ctypes.byref(e)))
         return e.value
+
+    def mg_merge_peers(self, runs: list, out_keys: torch.Tensor,
+                       out_vals: torch.Tensor | None = None, tmp_keys: torch.Tensor | None = None,
+                       tmp_vals: torch.Tensor | None = None, key_type: str | None = None):
+        """Stable merge of runs stored in separate buffers: runs = [(keys_buf,
+        vals_buf or None, offset, length), ...] (earlier runs win ties)."""
+        r = len(runs)
+        kp = (_P * r)(*[t[0].data_ptr() for t in runs])
+        vp = (_P * r)(*[t[1].data_ptr() for t in runs]) if out_vals is not None else None
+        bound = (_I64 * r)(*[t[0].numel() for t in runs])
+        off = (_I64 * r)(*[t[2] for t in runs])
+        ln = (_I64 * r)(*[t[3] for t in runs])
+        self._bind_stream(out_keys)
+        _check(lib().dc_mg_merge_peers(
+            self._h, _key_type(out_keys, key_type), kp, vp, bound, off, ln, r,
+            None if tmp_keys is None else tmp_keys.data_ptr(),
+            None if tmp_vals is None else tmp_vals.data_ptr(), out_keys.data_ptr(),
+            None if out_vals is None else out_vals.data_ptr()))
+        return out_keys
 
     def mg_merge_runs(self, in_keys: torch.Tensor, in_vals: torch.Tensor | None,
                       out_keys: torch.Tensor, out_vals: torch.Tensor | None, run_len: list[int],

@@ -242,8 +242,12 @@ dc_status ensure_pipeline(dc_plan_t p, int chunks) {
     return DC_OK;
 }
 
+// Sorts keys[0..n) (+ vals) into out_k (+ out_v); out may equal the input
+// (in place).  NK1 reads the input; the passes ping-pong between scratch and
+// the output buffer.
 template <class K, bool V, bool SMALL>
-dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
+dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_k,
+                     uint32_t* out_v) {
     const int64_t n = p->n;
     const bool hv = V;
     dc_status st = ensure_scratch(p, hv);
@@ -273,12 +277,12 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
     const bool two = kTwoCapable && p->two_level && P >= 2;
     const int single = two ? (P % 2) : P;
     const int passes = two ? single + (P - single) / 2 : P;
-    // Ping-pong parity: the last pass must write the caller's buffer, so NK1
-    // writes the caller's buffer iff the number of passes is even.
-    uint32_t* cur_k = (passes % 2 == 0) ? keys : sk;
-    uint32_t* cur_v = (passes % 2 == 0) ? vals : sv;
-    uint32_t* oth_k = (passes % 2 == 0) ? sk : keys;
-    uint32_t* oth_v = (passes % 2 == 0) ? sv : vals;
+    // Ping-pong parity: the last pass must write the output buffer, so NK1
+    // writes the output buffer iff the number of passes is even.
+    uint32_t* cur_k = (passes % 2 == 0) ? out_k : sk;
+    uint32_t* cur_v = (passes % 2 == 0) ? out_v : sv;
+    uint32_t* oth_k = (passes % 2 == 0) ? sk : out_k;
+    uint32_t* oth_v = (passes % 2 == 0) ? sv : out_v;
 
     // One merge level over [org, end) on stream `st` (split region `sp`).
     auto level = [&](int64_t org, int64_t end, int64_t w, int* sp, cudaStream_t st) -> dc_status {
@@ -402,19 +406,21 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
 }
 
 template <class K>
-dc_status sort_kv_dispatch(dc_plan_t p, uint32_t* keys, uint32_t* vals) {
+dc_status sort_kv_dispatch(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* ok,
+                           uint32_t* ov) {
     const bool small = p->n < kSmallN;
-    if (vals) return small ? sort_typed<K, true, true>(p, keys, vals)
-                           : sort_typed<K, true, false>(p, keys, vals);
-    return small ? sort_typed<K, false, true>(p, keys, nullptr)
-                 : sort_typed<K, false, false>(p, keys, nullptr);
+    if (vals) return small ? sort_typed<K, true, true>(p, keys, vals, ok, ov)
+                           : sort_typed<K, true, false>(p, keys, vals, ok, ov);
+    return small ? sort_typed<K, false, true>(p, keys, nullptr, ok, nullptr)
+                 : sort_typed<K, false, false>(p, keys, nullptr, ok, nullptr);
 }
 
-dc_status sort_direct(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
+dc_status sort_direct(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals, uint32_t* ok,
+                      uint32_t* ov) {
     switch (kt) {
-        case DC_KEY_U32: return sort_kv_dispatch<dc::KeyU32>(p, keys, vals);
-        case DC_KEY_I32: return sort_kv_dispatch<dc::KeyI32>(p, keys, vals);
-        case DC_KEY_F32: return sort_kv_dispatch<dc::KeyF32>(p, keys, vals);
+        case DC_KEY_U32: return sort_kv_dispatch<dc::KeyU32>(p, keys, vals, ok, ov);
+        case DC_KEY_I32: return sort_kv_dispatch<dc::KeyI32>(p, keys, vals, ok, ov);
+        case DC_KEY_F32: return sort_kv_dispatch<dc::KeyF32>(p, keys, vals, ok, ov);
     }
     return fail(DC_ERR_INVALID_ARG, "unknown key type");
 }
@@ -424,10 +430,15 @@ dc_status sort_direct(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* val
 // allocates scratch and sets kernel attributes); the second captures the
 // launches on a plan-owned stream and instantiates a graph; later runs
 // replay it on the plan stream.  Off while per-kernel timing is enabled.
-dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
-    if (!p->use_graphs || p->timing) return sort_direct(p, kt, keys, vals);
+dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals,
+                        uint32_t* ok = nullptr, uint32_t* ov = nullptr) {
+    if (!ok) {                                   // in place
+        ok = keys;
+        ov = vals;
+    }
+    if (!p->use_graphs || p->timing) return sort_direct(p, kt, keys, vals, ok, ov);
     for (auto& gc : p->graphs) {
-        if (gc.keys == keys && gc.vals == vals && gc.kt == kt) {
+        if (gc.keys == keys && gc.vals == vals && gc.out == ok && gc.kt == kt) {
             if (!gc.exec) {                                   // second sighting: capture
                 if (!p->cap_stream)
                     DC_CUDA(p, cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking));
@@ -435,7 +446,7 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
                 p->stream = p->cap_stream;
                 DC_CUDA(p, cudaStreamBeginCapture(p->cap_stream, cudaStreamCaptureModeThreadLocal));
                 const int64_t l0 = p->launches;
-                dc_status st = sort_direct(p, kt, keys, vals);
+                dc_status st = sort_direct(p, kt, keys, vals, ok, ov);
                 cudaGraph_t graph = nullptr;
                 cudaError_t e = cudaStreamEndCapture(p->cap_stream, &graph);
                 p->stream = user;
@@ -451,9 +462,9 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
             return DC_OK;
         }
     }
-    if (p->graphs.size() >= 8) return sort_direct(p, kt, keys, vals);
-    p->graphs.push_back({keys, vals, kt, nullptr, nullptr, 0});   // first sighting: eager
-    return sort_direct(p, kt, keys, vals);
+    if (p->graphs.size() >= 8) return sort_direct(p, kt, keys, vals, ok, ov);
+    p->graphs.push_back({keys, vals, ok, kt, nullptr, nullptr, 0});   // first sighting: eager
+    return sort_direct(p, kt, keys, vals, ok, ov);
 }
 
 // Max-subarray grid: about one wave of resident CTAs (occupancy x SMs),
@@ -575,6 +586,59 @@ dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* 
     return DC_OK;
 }
 
+// a8+a9 fused: the first round of the G-way merge reads its runs where they
+// lie (peer shards over NVLink); later rounds are local (mg_merge_typed).
+template <class K, bool V>
+dc_status mg_merge_peers_typed(dc_plan_t p, const uint32_t* const* rk, const uint32_t* const* rv,
+                               const int64_t* bound, const int64_t* off, const int64_t* len,
+                               int runs, uint32_t* tmp_k, uint32_t* tmp_v, uint32_t* out_k,
+                               uint32_t* out_v) {
+    int64_t total = 0;
+    for (int r = 0; r < runs; ++r) total += len[r];
+    if (total > p->n) return fail(DC_ERR_INVALID_ARG, "runs exceed the plan size");
+    dc_status st = ensure_scratch(p, V);
+    if (st != DC_OK) return st;
+    const size_t kb = align_up((size_t)p->n * 4, 256);
+    int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
+    constexpr SortCfg C = cfg_for<K, V, false>();
+    auto* k3 = dc::nk3_merge_ab<C.nt3, C.it, K, V>;
+    static bool attr_done = false;
+    if (!attr_done) {
+        DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        nk3_smem_bytes(C, V)));
+        attr_done = true;
+    }
+    const bool one_round = runs <= 2;
+    uint32_t* dk = one_round ? out_k : tmp_k;
+    uint32_t* dv = one_round ? out_v : tmp_v;
+    std::vector<int64_t> next;
+    int64_t org = 0;
+    for (int r = 0; r < runs; r += 2) {
+        const int rb = r + 1 < runs ? r + 1 : r;          // odd tail: B empty (a copy)
+        const int64_t la = len[r], lb = r + 1 < runs ? len[r + 1] : 0;
+        if (la + lb > 0) {
+            const int tiles = (int)num_tiles(la + lb, C.tout());
+            {
+                TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
+                dc::nk2_partition_ab<K><<<(tiles + 3) / 4, 128, 0, p->stream>>>(
+                    rk[r] + off[r], la, rk[rb] + off[rb], lb, C.tout(), tiles, split);
+                DC_LAUNCHED(p);
+            }
+            {
+                TimedScope ts(p, DC_KERNEL_NK3_MERGE);
+                k3<<<tiles, C.nt3, nk3_smem_bytes(C, V), p->stream>>>(
+                    rk[r], V ? rv[r] : nullptr, bound[r], off[r], la, rk[rb],
+                    V ? rv[rb] : nullptr, bound[rb], off[rb], lb, dk, dv, org, split);
+                DC_LAUNCHED(p);
+            }
+        }
+        next.push_back(la + lb);
+        org += la + lb;
+    }
+    if (one_round) return DC_OK;
+    return mg_merge_typed<K, V>(p, tmp_k, tmp_v, out_k, out_v, next);
+}
+
 dc_status ensure_mg_state(dc_plan_t p) {
     if (p->mg_state) return DC_OK;
     void* ptr = nullptr;
@@ -618,8 +682,9 @@ dc_status ensure_sum_state(dc_plan_t p) {
 namespace dcx {
 dc_status fail(dc_status s, const std::string& msg) { return ::fail(s, msg); }
 dc_status cuda_fail(dc_plan_t p, cudaError_t e, const char* what) { return ::cuda_fail(p, e, what); }
-dc_status local_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
-    return sort_dispatch(p, kt, keys, vals);
+dc_status local_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals,
+                     uint32_t* out_k, uint32_t* out_v) {
+    return sort_dispatch(p, kt, keys, vals, out_k, out_v);
 }
 }  // namespace dcx
 
@@ -1098,6 +1163,42 @@ dc_status dc_mg_merge_runs(dc_plan_t p, dc_key_type kt, uint32_t* d_in_keys, uin
                      : mg_merge_typed<dc::KeyF32, false>(p, d_in_keys, nullptr, d_out_keys,
                                                          nullptr, lens);
     }
+    return fail(DC_ERR_INVALID_ARG, "unknown key type");
+}
+
+dc_status dc_mg_merge_peers(dc_plan_t p, dc_key_type kt, const uint32_t* const* h_run_keys,
+                            const uint32_t* const* h_run_vals, const int64_t* h_bound,
+                            const int64_t* h_off, const int64_t* h_len, int32_t runs,
+                            uint32_t* d_tmp_keys, uint32_t* d_tmp_vals, uint32_t* d_out_keys,
+                            uint32_t* d_out_vals) {
+    dc_status st = check_plan(p);
+    if (st != DC_OK) return st;
+    const bool v = d_out_vals != nullptr;
+    if (!h_run_keys || !h_bound || !h_off || !h_len || runs < 1 || !d_out_keys ||
+        (v && !h_run_vals) || (runs > 2 && (!d_tmp_keys || (v && !d_tmp_vals))))
+        return fail(DC_ERR_INVALID_ARG, "bad peer-merge arguments");
+    for (int r = 0; r < runs; ++r) {
+        if (!h_run_keys[r] || !aligned16(h_run_keys[r]) ||
+            (v && (!h_run_vals[r] || !aligned16(h_run_vals[r]))))
+            return fail(DC_ERR_INVALID_ARG, "run buffers must be 16-byte aligned");
+        if (h_off[r] < 0 || h_len[r] < 0 || h_off[r] + h_len[r] > h_bound[r])
+            return fail(DC_ERR_INVALID_ARG, "run outside its buffer");
+    }
+    if (!aligned16(d_out_keys) || (v && !aligned16(d_out_vals)) ||
+        (d_tmp_keys && !aligned16(d_tmp_keys)) || (d_tmp_vals && !aligned16(d_tmp_vals)))
+        return fail(DC_ERR_INVALID_ARG, "buffers must be 16-byte aligned");
+#define DC_PEERS(KT)                                                                         \
+    return v ? mg_merge_peers_typed<KT, true>(p, h_run_keys, h_run_vals, h_bound, h_off, h_len, \
+                                              runs, d_tmp_keys, d_tmp_vals, d_out_keys,       \
+                                              d_out_vals)                                     \
+             : mg_merge_peers_typed<KT, false>(p, h_run_keys, nullptr, h_bound, h_off, h_len,  \
+                                               runs, d_tmp_keys, nullptr, d_out_keys, nullptr)
+    switch (kt) {
+        case DC_KEY_U32: DC_PEERS(dc::KeyU32);
+        case DC_KEY_I32: DC_PEERS(dc::KeyI32);
+        case DC_KEY_F32: DC_PEERS(dc::KeyF32);
+    }
+#undef DC_PEERS
     return fail(DC_ERR_INVALID_ARG, "unknown key type");
 }
 

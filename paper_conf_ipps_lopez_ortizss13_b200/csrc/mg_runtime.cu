@@ -142,12 +142,70 @@ struct Coll {
                                   const int64_t* scnt, const int64_t* soff, const int64_t* rcnt,
                                   const int64_t* roff, cudaStream_t s) = 0;
     virtual void abort() {}
+    // Stream-ordered barrier: work after it on any rank's stream follows every
+    // rank's work before it.
+    virtual dc_status barrier(cudaStream_t s) = 0;
+    // Peer access: every rank's `mine` (a cudaMalloc base) mapped into this
+    // process (peers[rank] = mine); *ok = 0 if this rank cannot map them all.
+    virtual dc_status share_buffer(void* mine, std::vector<void*>& peers, int* ok,
+                                   cudaStream_t s) = 0;
+    virtual void unshare(std::vector<void*>& peers) { (void)peers; }
 };
 
 struct NcclColl final : Coll {
     ncclComm_t comm = nullptr;
+    char* stage = nullptr;   // device staging for barrier words and IPC handles
     ~NcclColl() override {
         if (comm) nccl().CommDestroy(comm);
+        if (stage) cudaFree(stage);
+    }
+    dc_status ensure_stage() {
+        if (!stage) MG_CU(cudaMalloc(&stage, 256 + (size_t)(world + 1) * 64));
+        return DC_OK;
+    }
+    dc_status barrier(cudaStream_t s) override {
+        MG_TRY(ensure_stage());
+        return nccl_check(nccl().AllReduce(stage, stage, 1, ncclInt64, ncclSum, comm, s),
+                          "ncclAllReduce(barrier)");
+    }
+    // CUDA IPC over the node's NVLink/NVSwitch fabric: all-gather the 64-byte
+    // handles, open every peer's (lazy peer access).
+    dc_status share_buffer(void* mine, std::vector<void*>& peers, int* ok,
+                           cudaStream_t s) override {
+        MG_TRY(ensure_stage());
+        peers.assign(world, nullptr);
+        peers[rank] = mine;
+        *ok = 1;
+        cudaIpcMemHandle_t h;
+        std::memset(&h, 0, sizeof h);
+        if (!mine || cudaIpcGetMemHandle(&h, mine) != cudaSuccess) {
+            cudaGetLastError();
+            *ok = 0;
+        }
+        static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+        char* mine_d = stage + 256;
+        char* all_d = stage + 256 + 64;
+        MG_CU(cudaMemcpyAsync(mine_d, &h, 64, cudaMemcpyHostToDevice, s));
+        MG_TRY(all_gather(mine_d, all_d, 64, s));
+        std::vector<cudaIpcMemHandle_t> hs(world);
+        MG_CU(cudaMemcpyAsync(hs.data(), all_d, (size_t)world * 64, cudaMemcpyDeviceToHost, s));
+        MG_CU(cudaStreamSynchronize(s));
+        for (int q = 0; q < world && *ok; ++q) {
+            if (q == rank) continue;
+            void* ptr = nullptr;
+            if (cudaIpcOpenMemHandle(&ptr, hs[q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+                cudaGetLastError();
+                *ok = 0;
+                break;
+            }
+            peers[q] = ptr;
+        }
+        return DC_OK;
+    }
+    void unshare(std::vector<void*>& peers) override {
+        for (int q = 0; q < (int)peers.size(); ++q)
+            if (q != rank && peers[q]) cudaIpcCloseMemHandle(peers[q]);
+        peers.clear();
     }
     dc_status all_gather(const void* send, void* recv, size_t bytes, cudaStream_t s) override {
         return nccl_check(nccl().AllGather(send, recv, bytes, ncclUint8, comm, s), "ncclAllGather");
@@ -222,6 +280,23 @@ struct LoopColl final : Coll {
         std::lock_guard<std::mutex> lk(g->mu);
         g->aborted = true;
         g->cv.notify_all();
+    }
+    dc_status barrier(cudaStream_t s) override {
+        MG_CU(cudaEventRecord(g->ready[rank], s));
+        MG_TRY(lb_barrier(g));
+        for (int r = 0; r < world; ++r) MG_CU(cudaStreamWaitEvent(s, g->ready[r], 0));
+        return lb_barrier(g);
+    }
+    // One process, one device: the peers' buffers are directly addressable.
+    dc_status share_buffer(void* mine, std::vector<void*>& peers, int* ok,
+                           cudaStream_t s) override {
+        (void)s;
+        g->ptr[rank] = mine;
+        MG_TRY(lb_barrier(g));
+        peers.resize(world);
+        for (int r = 0; r < world; ++r) peers[r] = const_cast<void*>(g->ptr[r]);
+        *ok = 1;
+        return lb_barrier(g);
     }
     // Second half of every collective: signal that this rank's reads are
     // enqueued, and order this stream after every rank's reads of our buffers.
@@ -307,7 +382,14 @@ struct MgCtx {
     int64_t* h_pin = nullptr;   // pinned: split matrix, then the max-subarray result
     size_t h_pin_words = 0;
     std::vector<int64_t> last_cmat;
+    // fused exchange: the sorted shard lives in xbuf (keys, then values),
+    // mapped by every peer; peers[q] = rank q's xbuf in this address space
+    int p2p = 0;                // 0 undecided, 1 fused, -1 NCCL all-to-all
+    char* xbuf = nullptr;
+    std::vector<void*> peers;
     ~MgCtx() {
+        if (coll) coll->unshare(peers);
+        if (xbuf) cudaFree(xbuf);
         delete coll;
         if (ws) cudaFree(ws);
         if (recv) cudaFree(recv);
@@ -383,7 +465,47 @@ dc_status ensure_recv(MgCtx* c, bool vals) {
     return DC_OK;
 }
 
-dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
+// The fused exchange needs every rank to map every peer's shard buffer;
+// decided once, collectively (all ranks agree or all use the all-to-all).
+dc_status setup_p2p(dc_plan_t p, MgCtx* c) {
+    if (c->p2p) return DC_OK;
+    int want = p->mg_p2p ? 1 : 0;
+    if (const char* e = std::getenv("DC_MG_P2P")) want = std::atoi(e) != 0;
+    if (!want) {
+        c->p2p = -1;
+        return DC_OK;
+    }
+    const size_t kb = al256((size_t)c->m * 4);
+    int ok = 1;
+    if (cudaMalloc(&c->xbuf, 2 * kb) != cudaSuccess) {
+        cudaGetLastError();
+        c->xbuf = nullptr;
+        ok = 0;
+    }
+    int mapped = 0;   // every rank joins the (collective) exchange, even without a buffer
+    MG_TRY(c->coll->share_buffer(c->xbuf, c->peers, &mapped, p->stream));
+    ok = ok && mapped;
+    // agree: the number of ranks that cannot map everything, summed
+    MG_TRY(ensure_ws(p, c, c->ws_stride ? c->ws_stride : p->mg_stride));
+    c->h_pin[0] = ok ? 0 : 1;
+    MG_CU(cudaMemcpyAsync(c->counts, c->h_pin, 8, cudaMemcpyHostToDevice, p->stream));
+    MG_TRY(c->coll->all_reduce_sum_i64(c->counts, 1, p->stream));
+    MG_CU(cudaMemcpyAsync(c->h_pin, c->counts, 8, cudaMemcpyDeviceToHost, p->stream));
+    MG_CU(cudaStreamSynchronize(p->stream));
+    if (c->h_pin[0] == 0) {
+        c->p2p = 1;
+        return DC_OK;
+    }
+    c->coll->unshare(c->peers);
+    if (c->xbuf) cudaFree(c->xbuf);
+    c->xbuf = nullptr;
+    c->p2p = -1;
+    return DC_OK;
+}
+
+// keys/vals: this rank's sorted shard (in xbuf when fused); out: the caller's buffers.
+dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, uint32_t* vals,
+                        uint32_t* out_k, uint32_t* out_v) {
     const int G = c->world, me = c->rank;
     const int64_t m = c->m, S = p->mg_stride, q = (m + S - 1) / S, wcap = S;
     if ((int64_t)G * wcap * 4 > 200 * 1024)
@@ -421,16 +543,34 @@ dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, u
         if (scnt[d] < 0 || rcnt[d] < 0) return fail(DC_ERR_BAD_STATE, "negative split size");
     }
     if (tot != m) return fail(DC_ERR_BAD_STATE, "received element count != shard size");
+    const size_t kb = al256((size_t)m * 4);
+    if (c->p2p == 1) {
+        // a8+a9 fused: merge straight from the peers' shards (NVLink reads)
+        if (G > 2) MG_TRY(ensure_recv(c, vals != nullptr));
+        std::vector<const uint32_t*> rk(G), rv(G);
+        std::vector<int64_t> bound(G, m), off(G);
+        for (int d = 0; d < G; ++d) {
+            rk[d] = (const uint32_t*)c->peers[d];
+            rv[d] = (const uint32_t*)((const char*)c->peers[d] + kb);
+            off[d] = cm[d * (G + 1) + me];
+        }
+        uint32_t* tk = G > 2 ? c->recv : nullptr;
+        uint32_t* tv = (G > 2 && vals) ? (uint32_t*)((char*)c->recv + kb) : nullptr;
+        MG_TRY(dc_mg_merge_peers(p, kt, rk.data(), vals ? rv.data() : nullptr, bound.data(),
+                                 off.data(), rcnt.data(), G, tk, tv, out_k, out_v));
+        // nobody rewrites its shard (next sort) while a peer may still read it
+        return c->coll->barrier(s);
+    }
     // a8: all-to-all of the ranges (keys and values in one group)
     MG_TRY(ensure_recv(c, vals != nullptr));
     uint32_t* rk = c->recv;
-    uint32_t* rv = vals ? (uint32_t*)((char*)c->recv + al256((size_t)m * 4)) : nullptr;
+    uint32_t* rv = vals ? (uint32_t*)((char*)c->recv + kb) : nullptr;
     const uint32_t* send[2] = {keys, vals};
     uint32_t* recv[2] = {rk, rv};
     MG_TRY(c->coll->all_to_allv(vals ? 2 : 1, send, recv, scnt.data(), soff.data(), rcnt.data(),
                                 roff.data(), s));
     // a9: local stable G-way merge (earlier ranks win ties) into the caller's buffers
-    return dc_mg_merge_runs(p, kt, rk, rv, keys, vals, rcnt.data(), G);
+    return dc_mg_merge_runs(p, kt, rk, rv, out_k, out_v, rcnt.data(), G);
 }
 
 dc_status attach(dc_plan_t p, Coll* coll, int rank, int world) {
@@ -466,8 +606,20 @@ dc_status can_attach(dc_plan_t p, int32_t rank, int32_t world) {
 
 dc_status mg_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
     MgCtx* c = p->mg;
-    dc_status st = local_sort(p, kt, keys, vals);     // levels >= log2 G: no communication
-    if (st == DC_OK && c->world > 1) st = sort_exchange(p, c, kt, keys, vals);
+    auto run = [&]() -> dc_status {
+        if (c->world == 1) return local_sort(p, kt, keys, vals);
+        MG_TRY(setup_p2p(p, c));
+        if (c->p2p == 1) {   // levels >= log2 G into the shared shard buffer
+            const size_t kb = al256((size_t)c->m * 4);
+            uint32_t* xk = (uint32_t*)c->xbuf;
+            uint32_t* xv = vals ? (uint32_t*)(c->xbuf + kb) : nullptr;
+            MG_TRY(local_sort(p, kt, keys, vals, xk, xv));
+            return sort_exchange(p, c, kt, xk, xv, keys, vals);
+        }
+        MG_TRY(local_sort(p, kt, keys, vals));        // levels >= log2 G: no communication
+        return sort_exchange(p, c, kt, keys, vals, keys, vals);
+    };
+    const dc_status st = run();
     if (st != DC_OK) c->coll->abort();
     return st;
 }
@@ -588,6 +740,20 @@ dc_status dc_plan_set_mg_stride(dc_plan_t p, int64_t stride) {
     if (!p) return dcx::fail(DC_ERR_INVALID_ARG, "plan is NULL");
     if (stride < 1 || stride > (1 << 20)) return dcx::fail(DC_ERR_INVALID_ARG, "stride out of range");
     p->mg_stride = stride;
+    return DC_OK;
+}
+
+dc_status dc_plan_set_mg_p2p(dc_plan_t p, int32_t enable) {
+    if (!p) return dcx::fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (p->mg && p->mg->p2p != 0)
+        return dcx::fail(DC_ERR_INVALID_ARG, "exchange mode is fixed after the first sort");
+    p->mg_p2p = enable != 0;
+    return DC_OK;
+}
+
+dc_status dc_plan_mg_exchange_mode(dc_plan_t p, int32_t* mode) {
+    if (!p || !mode) return dcx::fail(DC_ERR_INVALID_ARG, "NULL argument");
+    *mode = p->mg ? p->mg->p2p : 0;
     return DC_OK;
 }
 

@@ -15,7 +15,9 @@ struct MgCtx;   // multi-GPU runtime state (mg_runtime.cu)
 // Internal entry points shared between dc_api.cu and mg_runtime.cu.
 dc_status fail(dc_status s, const std::string& msg);                 // sets dc_last_error
 dc_status cuda_fail(dc_plan_t p, cudaError_t e, const char* what);   // poisons the plan
-dc_status local_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals);
+// sorts keys (+vals) into out_k (+out_v); nullptr outputs = in place
+dc_status local_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals,
+                     uint32_t* out_k = nullptr, uint32_t* out_v = nullptr);
 dc_status mg_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals);
 dc_status mg_maxsub(dc_plan_t p, const int32_t* x, dc_maxsub_result* h_out);
 void mg_destroy(MgCtx* c);
@@ -42,6 +44,7 @@ struct dc_plan_s {
     struct GraphCache {
         uint32_t* keys;
         uint32_t* vals;
+        uint32_t* out;
         dc_key_type kt;
         cudaGraph_t graph;
         cudaGraphExec_t exec;
@@ -87,6 +90,7 @@ struct dc_plan_s {
     dcx::MgCtx* mg = nullptr;
     int64_t n_global = 0;
     int64_t mg_stride = 4096;   // splitter sample stride S
+    bool mg_p2p = true;         // fused exchange (peer reads) when every rank can map every peer
     // per-kernel CUDA-event timing (instrumentation, off by default)
     bool timing = false;
     struct Timed { int kind; cudaEvent_t e0, e1; };

@@ -530,14 +530,20 @@ __device__ __forceinline__ void stage_piece(const uint32_t* __restrict__ g, long
 // pieces are staged in shared memory by TMA, each thread finds its own
 // IT-output diagonal there and merges serially, and the tile leaves by one
 // TMA bulk store.  n bounds the readable part of src.
+//
+// A and B may live in different buffers (e.g. a peer GPU's memory, read over
+// NVLink by the multi-GPU merge): src_a / src_b are 16-byte-aligned buffer
+// bases, na_bound / nb_bound their readable lengths, a0 / b0 offsets in them.
 template <int NT, int IT, class K, bool V>
-__device__ __forceinline__ void merge_tile(const uint32_t* __restrict__ src_k,
-                                           const uint32_t* __restrict__ src_v,
+__device__ __forceinline__ void merge_tile(const uint32_t* __restrict__ src_ka,
+                                           const uint32_t* __restrict__ src_va, long long n_a,
+                                           long long a0, int na,
+                                           const uint32_t* __restrict__ src_kb,
+                                           const uint32_t* __restrict__ src_vb, long long n_b,
+                                           long long b0, int nb,
                                            uint32_t* __restrict__ dst_k,
-                                           uint32_t* __restrict__ dst_v, long long n,
-                                           long long a0, int na, long long b0, int nb,
-                                           long long o0, uint32_t* sk, uint32_t* sv,
-                                           uint32_t BAR) {
+                                           uint32_t* __restrict__ dst_v, long long o0,
+                                           uint32_t* sk, uint32_t* sv, uint32_t BAR) {
     constexpr int TOUT = NT * IT;
     constexpr int TW = tile_words(TOUT, IT + 16);
     constexpr uint32_t SV_OFF = TW * 4;
@@ -547,30 +553,30 @@ __device__ __forceinline__ void merge_tile(const uint32_t* __restrict__ src_k,
     const int fa = (int)(a0 & 3), fb = (int)(b0 & 3);
     const int ob = (fa + na + 1 + 3) & ~3;             // B region word offset (16 B aligned)
     const uint32_t A = SK + 4u * fa, B = SK + 4u * (ob + fb);
-    const long long n4 = n & ~3LL;
+    const long long a4 = n_a & ~3LL, b4 = n_b & ~3LL;
 
     if (tid == 0) {
         mbar_init(BAR, 1);
-        const uint32_t bytes = piece_bytes(a0, a0 + na, n4) + piece_bytes(b0, b0 + nb, n4);
+        const uint32_t bytes = piece_bytes(a0, a0 + na, a4) + piece_bytes(b0, b0 + nb, b4);
         mbar_arrive_expect_tx(BAR, bytes * (V ? 2 : 1));
-        stage_piece(src_k, a0, a0 + na, n4, 0, SK, BAR);
-        stage_piece(src_k, b0, b0 + nb, n4, ob, SK, BAR);
+        stage_piece(src_ka, a0, a0 + na, a4, 0, SK, BAR);
+        stage_piece(src_kb, b0, b0 + nb, b4, ob, SK, BAR);
         if (V) {
-            stage_piece(src_v, a0, a0 + na, n4, 0, SV, BAR);
-            stage_piece(src_v, b0, b0 + nb, n4, ob, SV, BAR);
+            stage_piece(src_va, a0, a0 + na, a4, 0, SV, BAR);
+            stage_piece(src_vb, b0, b0 + nb, b4, ob, SV, BAR);
         }
     }
-    // elements at or beyond n4 (only in the last pieces of the array)
-    if (a0 + na > n4) {
-        for (long long g = max(a0, n4) + tid; g < a0 + na; g += NT) {
-            sk[fa + (g - a0)] = src_k[g];
-            if (V) sv[fa + (g - a0)] = src_v[g];
+    // elements at or beyond the aligned bound (only in the last pieces of a buffer)
+    if (a0 + na > a4) {
+        for (long long g = max(a0, a4) + tid; g < a0 + na; g += NT) {
+            sk[fa + (g - a0)] = src_ka[g];
+            if (V) sv[fa + (g - a0)] = src_va[g];
         }
     }
-    if (b0 + nb > n4) {
-        for (long long g = max(b0, n4) + tid; g < b0 + nb; g += NT) {
-            sk[ob + fb + (g - b0)] = src_k[g];
-            if (V) sv[ob + fb + (g - b0)] = src_v[g];
+    if (b0 + nb > b4) {
+        for (long long g = max(b0, b4) + tid; g < b0 + nb; g += NT) {
+            sk[ob + fb + (g - b0)] = src_kb[g];
+            if (V) sv[ob + fb + (g - b0)] = src_vb[g];
         }
     }
     __syncthreads();
@@ -624,8 +630,53 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
     const int i1 = (dd1 == a_len + b_len) ? (int)a_len : split[j + 1];
     const int na = i1 - i0;
     const int nb = (int)(dd1 - dd0) - na;
-    merge_tile<NT, IT, K, V>(src_k, src_v, dst_k, dst_v, g.end, s + i0, na,
-                             s + a_len + (dd0 - i0), nb, g.org + d0, smem, smem + TW,
+    merge_tile<NT, IT, K, V>(src_k, src_v, g.end, s + i0, na, src_k, src_v, g.end,
+                             s + a_len + (dd0 - i0), nb, dst_k, dst_v, g.org + d0, smem,
+                             smem + TW, smem_addr(&bar));
+}
+
+// ------------------------------------------- merges of separately stored runs
+// The first round of the multi-GPU G-way merge reads its two runs straight
+// from the sorted shards of two (peer) GPUs -- the exchange fused into the
+// merge, the NVLink reads overlapping the merge tile by tile.  A run is
+// (buffer base, readable length, offset, length); bases are 16-byte aligned.
+
+// Co-rank of every output tile of merge(A, B), one warp per tile (33-ary
+// search: ~log33 of the run length dependent rounds of remote latency).
+template <class K>
+__global__ void nk2_partition_ab(const uint32_t* __restrict__ A, long long a_len,
+                                 const uint32_t* __restrict__ B, long long b_len, int tout,
+                                 int num_tiles, int* __restrict__ split) {
+    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    if (j >= num_tiles) return;                       // warp-uniform
+    const long long diag = (long long)j * tout;
+    const long long lo = max(0LL, diag - b_len), hi = min(diag, a_len);
+    const long long c = warp_first_false(lo, hi, [&](long long m) {
+        return !K::lt(__ldg(B + (diag - 1 - m)), __ldg(A + m));
+    });
+    if ((threadIdx.x & 31) == 0) split[j] = (int)c;
+}
+
+// Output tile j of merge(A, B) -> dst[o_off + j*TOUT, ...).
+template <int NT, int IT, class K, bool V>
+__global__ void __launch_bounds__(NT)
+nk3_merge_ab(const uint32_t* __restrict__ ka, const uint32_t* __restrict__ va, long long a_bound,
+             long long a_off, long long a_len, const uint32_t* __restrict__ kb,
+             const uint32_t* __restrict__ vb, long long b_bound, long long b_off, long long b_len,
+             uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v, long long o_off,
+             const int* __restrict__ split) {
+    constexpr int TOUT = NT * IT;
+    constexpr int TW = tile_words(TOUT, IT + 16);
+    extern __shared__ __align__(16) uint32_t smem[];
+    __shared__ __align__(8) uint64_t bar;
+    const long long d0 = (long long)blockIdx.x * TOUT;
+    const long long d1 = min(d0 + TOUT, a_len + b_len);
+    const int i0 = split[blockIdx.x];
+    const int i1 = (d1 == a_len + b_len) ? (int)a_len : split[blockIdx.x + 1];
+    const int na = i1 - i0;
+    const int nb = (int)(d1 - d0) - na;
+    merge_tile<NT, IT, K, V>(ka, va, a_bound, a_off + i0, na, kb, vb, b_bound,
+                             b_off + (d0 - i0), nb, dst_k, dst_v, o_off + d0, smem, smem + TW,
                              smem_addr(&bar));
 }
 

@@ -27,12 +27,13 @@ def dc():
     return m
 
 
-def run_ranks(dc, n, world, fn, stride=None):
+def run_ranks(dc, n, world, fn, stride=None, p2p=True):
     """fn(plan, rank, m) on `world` threads joined to one loopback group."""
     group = dc.LoopbackGroup(world)
     plans = []
     for r in range(world):
         p = dc.Plan(n)
+        p.set_mg_p2p(p2p)
         if stride:
             p.set_mg_stride(stride)
         p.set_loopback(group, r)
@@ -60,15 +61,22 @@ def _view(a, key_type):
     return a.view({"u32": np.uint32, "i32": np.int32, "f32": np.float32}[key_type])
 
 
-def sort_case(dc, oracle_mod, n, world, dist_name, key_type, with_vals, stride=None, seed=31):
+def sort_case(dc, oracle_mod, n, world, dist_name, key_type, with_vals, stride=None, seed=31,
+              p2p=True, reps=1):
     def fn(plan, r, m):
-        keys = dcgen.sort_keys(n, dist_name, seed=seed, key_type=key_type, start=r * m, count=m,
-                               device="cuda")
-        vals = dcgen.sort_vals(n, start=r * m, count=m, device="cuda") if with_vals else None
-        plan.sort_(keys, vals, key_type=key_type)
-        return keys.cpu(), (vals.cpu() if with_vals else None), plan.last_splits()
+        src = dcgen.sort_keys(n, dist_name, seed=seed, key_type=key_type, start=r * m, count=m,
+                              device="cuda")
+        keys = torch.empty_like(src)
+        vals = torch.empty(m, dtype=torch.int32, device="cuda") if with_vals else None
+        for _ in range(reps):              # repeated sorts reuse the shared shard buffers
+            keys.copy_(src)
+            if with_vals:
+                vals.copy_(dcgen.sort_vals(n, start=r * m, count=m, device="cuda"))
+            plan.sort_(keys, vals, key_type=key_type)
+        return (keys.cpu(), (vals.cpu() if with_vals else None), plan.last_splits(),
+                plan.exchange_mode())
 
-    res, errs, plans = run_ranks(dc, n, world, fn, stride)
+    res, errs, plans = run_ranks(dc, n, world, fn, stride, p2p)
     for e in errs:
         if e is not None:
             raise e
@@ -86,13 +94,23 @@ def sort_case(dc, oracle_mod, n, world, dist_name, key_type, with_vals, stride=N
     m = n // world
     assert np.array_equal(cm.sum(axis=0), np.arange(world + 1) * m)
     assert np.all(np.diff(cm, axis=1) >= 0)
+    assert all(r[3] == ("fused" if p2p else "all_to_all") for r in res)
     return cm
 
 
+@pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
 @pytest.mark.parametrize("world", [2, 3, 4, 8])
 @pytest.mark.parametrize("dist_name", ["uniform", "few", "sorted", "reverse", "equal"])
-def test_loopback_kv(dc, oracle_mod, world, dist_name):
-    sort_case(dc, oracle_mod, world * 100_003, world, dist_name, "u32", True)
+def test_loopback_kv(dc, oracle_mod, world, dist_name, p2p):
+    sort_case(dc, oracle_mod, world * 100_003, world, dist_name, "u32", True, p2p=p2p)
+
+
+@pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
+@pytest.mark.parametrize("world", [2, 5])
+def test_loopback_repeated_sorts(dc, oracle_mod, world, p2p):
+    """Three sorts back to back per rank (graph replay of the local levels,
+    the shard buffers rewritten while peers have just read them)."""
+    sort_case(dc, oracle_mod, world * 200_001, world, "paper", "u32", True, p2p=p2p, reps=3)
 
 
 @pytest.mark.parametrize("key_type", ["u32", "i32", "f32"])
@@ -101,9 +119,10 @@ def test_loopback_keys_only(dc, oracle_mod, key_type, stride):
     sort_case(dc, oracle_mod, 4 * 250_001, 4, "paper", key_type, False, stride)
 
 
-def test_loopback_large_shards(dc, oracle_mod):
-    """2^24 keys over 4 ranks: 4M-key shards use the full-size tile config."""
-    sort_case(dc, oracle_mod, 1 << 24, 4, "uniform", "u32", False)
+@pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
+def test_loopback_large_shards(dc, oracle_mod, p2p):
+    """2^25 keys over 2 ranks: 16M-key shards use the full-size tile config."""
+    sort_case(dc, oracle_mod, 1 << 25, 2, "uniform", "u32", False, p2p=p2p)
 
 
 def test_loopback_equal_keys_split_exactly(dc, oracle_mod):
@@ -196,3 +215,44 @@ def test_nccl_world1_sort_and_maxsub(dc, oracle_mod):
     assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)
     x = dcgen.maxsub_input(n, "uniform", seed=8, device="cuda")
     assert p.max_subarray(x) == tuple(int(v) for v in oracle_mod.maxsub(x.cpu().numpy()))
+
+
+@pytest.mark.parametrize("key_type", ["u32", "i32", "f32"])
+@pytest.mark.parametrize("runs", [1, 2, 3, 4, 7])
+def test_merge_peers_separate_buffers(dc, oracle_mod, key_type, runs):
+    """dc_mg_merge_peers on runs that each live in their own buffer at an
+    arbitrary offset (unaligned starts, ragged lengths, empty runs)."""
+    rng = np.random.default_rng(runs)
+    lens = [int(rng.integers(0, 40_000)) for _ in range(runs)]
+    if runs > 2:
+        lens[1] = 0
+    total = sum(lens)
+    plan = dc.Plan(max(total, 1))
+    bufs, vbufs, offs, allk, allv, pos = [], [], [], [], [], 0
+    view = {"u32": np.uint32, "i32": np.int32, "f32": np.float32}[key_type]
+    for r, ln in enumerate(lens):
+        off = int(rng.integers(0, 37))
+        k = dcgen.sort_keys(off + ln + 11, "few", seed=r, key_type=key_type)
+        seg = k[off:off + ln].numpy().view(view)
+        srt = np.sort(seg, kind="stable")
+        k[off:off + ln] = torch.from_numpy(srt.copy().view(np.int32)
+                                           if key_type != "f32" else srt.copy())
+        v = torch.arange(pos - off, pos - off + k.numel(), dtype=torch.int32)
+        bufs.append(k.cuda())
+        vbufs.append(v.cuda())
+        offs.append(off)
+        allk.append(k[off:off + ln].numpy().view(view))
+        allv.append(v[off:off + ln].numpy().view(np.uint32))
+        pos += ln
+    out_k = torch.empty(max(total, 1), dtype=bufs[0].dtype, device="cuda")
+    out_v = torch.empty(max(total, 1), dtype=torch.int32, device="cuda")
+    tk = torch.empty_like(out_k)
+    tv = torch.empty_like(out_v)
+    plan.mg_merge_peers([(bufs[r], vbufs[r], offs[r], lens[r]) for r in range(runs)],
+                        out_k, out_v, tk, tv, key_type=key_type)
+    cat_k = np.concatenate(allk)
+    cat_v = np.concatenate(allv)
+    ek, ev = oracle_mod.mergesort(cat_k, cat_v, key_type=key_type)   # stable: earlier run wins
+    got = out_k[:total].cpu().numpy().view(view)
+    assert np.array_equal(got.view(np.uint32), ek.view(np.uint32))
+    assert np.array_equal(out_v[:total].cpu().numpy().view(np.uint32), ev)
