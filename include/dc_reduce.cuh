@@ -21,6 +21,9 @@
 // and the caller provides `parts` (one T per CTA) and a zero-initialised
 // `ticket`; the result is written to *out by the last CTA.  Launch with a grid
 // of at most a few waves; NT threads per CTA (multiple of 32, <= 1024).
+// Two kernels: breadth_first_reduce (plain loads, any element type) and
+// breadth_first_reduce_tma (TMA-streamed warp segments, 4-byte elements;
+// the library's dc_run_sum uses it).
 #pragma once
 #include <cstdint>
 
@@ -113,6 +116,162 @@ breadth_first_reduce(const typename M::In* __restrict__ x, long long n,
     if (tid == 0) {
         *out = a;
         *ticket = 0u;   // re-arm for the next launch
+    }
+}
+
+// ------------------------------------------------------------------------
+// breadth_first_reduce_tma: the same D&C with the data streamed by TMA.
+// Every WARP owns one contiguous range of RW elements (RW a multiple of
+// 32*L) and streams it in segments of 32*L elements, one 1-D bulk copy per
+// segment into an S-stage shared-memory ring (mbarrier per warp and stage);
+// lane l folds the L contiguous elements [l*L, (l+1)*L) of each segment
+// (128-bit shared reads, bank-conflict free because L/4 is odd), an ordered
+// shuffle tree combines the 32 lane summaries, lane 0 keeps the warp's running
+// summary; warps, then CTAs (last CTA, atomic ticket), combine in order.
+// Requirements: sizeof(In) == 4, x 16-byte aligned; launch with NT threads,
+// breadth_first_reduce_tma_smem<NT, L, S>() bytes of dynamic shared memory
+// (raise cudaFuncAttributeMaxDynamicSharedMemorySize above 48 KB) and a grid
+// of at most one wave; RW = breadth_first_reduce_tma_rw<NT, L>(n, grid).
+namespace rtma {
+__device__ __forceinline__ uint32_t saddr(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void bar_init(uint32_t bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void bar_expect(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bar_wait(uint32_t bar, uint32_t phase) {
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(bar), "r"(phase)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void copy(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+        ::"r"(dst), "l"(src), "r"(bytes), "r"(bar)
+        : "memory");
+}
+__device__ __forceinline__ void fence_async() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+}  // namespace rtma
+
+template <int NT, int L, int S>
+constexpr size_t breadth_first_reduce_tma_smem() {
+    return (size_t)S * NT * L * 4;
+}
+template <int NT, int L>
+inline long long breadth_first_reduce_tma_rw(long long n, int grid) {
+    const long long warps = (long long)grid * (NT / 32), seg = 32LL * L;
+    return ((n + warps - 1) / warps + seg - 1) / seg * seg;
+}
+
+template <class M, int NT, int L, int S>
+__global__ void __launch_bounds__(NT)
+breadth_first_reduce_tma(const typename M::In* __restrict__ x, long long n, long long RW,
+                         typename M::T* __restrict__ parts, unsigned int* __restrict__ ticket,
+                         typename M::T* __restrict__ out) {
+    using T = typename M::T;
+    using In = typename M::In;
+    static_assert(sizeof(In) == 4, "4-byte elements");
+    static_assert(L % 4 == 0 && ((L / 4) & 1) == 1, "L/4 odd: conflict-free 128-bit reads");
+    constexpr int NW = NT / 32, SEG = 32 * L;
+    extern __shared__ __align__(16) unsigned char rtma_smem[];
+    In* ring = reinterpret_cast<In*>(rtma_smem);               // [S][NW][SEG]
+    __shared__ __align__(8) uint64_t bars[S][NW];
+    __shared__ T red[NW];
+    __shared__ bool am_last;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const long long wbeg = min(n, ((long long)blockIdx.x * NW + warp) * RW);
+    const long long wend = min(n, wbeg + RW);
+    const int nseg = (int)((wend - wbeg + SEG - 1) / SEG);
+    if (lane == 0)
+        for (int s = 0; s < S; ++s) rtma::bar_init(rtma::saddr(&bars[s][warp]));
+    __syncwarp();
+    auto seg_ptr = [&](int s) { return ring + (s * NW + warp) * SEG; };
+    auto issue = [&](int k) {
+        const int s = k % S;
+        const long long g0 = wbeg + (long long)k * SEG;
+        const int body = (int)min((long long)SEG, wend - g0) & ~3;
+        const uint32_t bar = rtma::saddr(&bars[s][warp]);
+        rtma::bar_expect(bar, 4u * body);
+        if (body) rtma::copy(rtma::saddr(seg_ptr(s)), x + g0, 4u * body, bar);
+    };
+    if (lane == 0)
+        for (int k = 0; k < S && k < nseg; ++k) issue(k);
+    T acc = M::identity();                                      // lane 0: warp summary
+    for (int k = 0; k < nseg; ++k) {
+        const int s = k % S;
+        rtma::bar_wait(rtma::saddr(&bars[s][warp]), (uint32_t)((k / S) & 1));
+        const long long g0 = wbeg + (long long)k * SEG;
+        const int cnt = (int)min((long long)SEG, wend - g0);
+        const In* sl = seg_ptr(s) + lane * L;
+        const long long i0 = g0 + (long long)lane * L;
+        T f = M::identity();
+        if (cnt == SEG) {
+#pragma unroll
+            for (int q = 0; q < L / 4; ++q) {
+                const int4 v = *reinterpret_cast<const int4*>(sl + 4 * q);
+                const In* e = reinterpret_cast<const In*>(&v);
+                f = M::combine(f, M::leaf(e[0], i0 + 4 * q));
+                f = M::combine(f, M::leaf(e[1], i0 + 4 * q + 1));
+                f = M::combine(f, M::leaf(e[2], i0 + 4 * q + 2));
+                f = M::combine(f, M::leaf(e[3], i0 + 4 * q + 3));
+            }
+        } else {                                                // last, partial segment
+            const int body = cnt & ~3;
+            for (int e = lane * L; e < min(cnt, lane * L + L); ++e)
+                f = M::combine(f, M::leaf(e < body ? seg_ptr(s)[e] : x[g0 + e], g0 + e));
+        }
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {                      // ordered warp tree
+            const T r = reduce_shfl_down(f, o);
+            if ((lane & (2 * o - 1)) == 0) f = M::combine(f, r);
+        }
+        if (lane == 0) acc = M::combine(acc, f);
+        __syncwarp();
+        if (lane == 0 && k + S < nseg) {
+            rtma::fence_async();
+            issue(k + S);
+        }
+    }
+    if (lane == 0) red[warp] = acc;
+    __syncthreads();
+    if (tid == 0) {
+        T c = M::identity();
+        for (int w = 0; w < NW; ++w) c = M::combine(c, red[w]);
+        parts[blockIdx.x] = c;
+        __threadfence();
+        am_last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!am_last) return;
+    __threadfence();
+    const int np = gridDim.x, per = (np + NT - 1) / NT;
+    T a = M::identity();
+    for (int q = tid * per; q < min(np, tid * per + per); ++q) {
+        T v;
+        const volatile int* src = reinterpret_cast<const volatile int*>(parts + q);
+        int* dst = reinterpret_cast<int*>(&v);
+#pragma unroll
+        for (int w = 0; w < (int)(sizeof(T) / 4); ++w) dst[w] = src[w];   // L2-coherent
+        a = M::combine(a, v);
+    }
+    a = reduce_block<M, NT>(a, red);
+    if (tid == 0) {
+        *out = a;
+        *ticket = 0u;
     }
 }
 

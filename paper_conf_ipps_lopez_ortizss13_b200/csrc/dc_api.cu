@@ -24,6 +24,7 @@
 #include "mg_kernels.cuh"
 #include "sort_kernels.cuh"
 #include "sort2_kernels.cuh"
+#include "maxsub_tma.cuh"
 
 namespace {
 
@@ -290,7 +291,10 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         const dc::PairGeom g{org, w, w, end};
         {
             TimedScope ts(p, DC_KERNEL_NK2_PARTITION, st);
-            if (SMALL)   // L2-resident: 33-ary warp searches, few dependent rounds
+#ifndef DC_NK2_WARP_ALL
+#define DC_NK2_WARP_ALL 0
+#endif
+            if (SMALL || DC_NK2_WARP_ALL)   // L2-resident: 33-ary warp searches, few dependent rounds
                 dc::nk2_partition_warp<K><<<(tiles + 3) / 4, 128, 0, st>>>(cur_k, g, C.tout(),
                                                                          tiles, sp);
             else
@@ -362,6 +366,9 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
             keys, vals, cur_k, cur_v, n);
         DC_LAUNCHED(p);
     }
+#ifdef DC_ONLY_NK1   // measurement builds only: time the fused kernel alone
+    return DC_OK;
+#endif
     for (; lv < single; ++lv, w *= 2) {
         st = level(0, n, w, split, p->stream);
         if (st != DC_OK) return st;
@@ -467,20 +474,47 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
     return sort_direct(p, kt, keys, vals, ok, ov);
 }
 
+// Max-subarray kernel: DC_MS_TMA = 1 (default) streams every lane's range by
+// TMA (maxsub_tma.cuh, one CTA per SM); 0 is the register-load version.
+#ifndef DC_MS_TMA
+#define DC_MS_TMA 1
+#endif
+#ifndef DC_MS_P            // L: elements per lane per warp segment (L/4 odd)
+#define DC_MS_P 68
+#endif
+#ifndef DC_MS_S
+#define DC_MS_S 2
+#endif
+#ifndef DC_MS_TNT
+#define DC_MS_TNT 256
+#endif
+#ifndef DC_MS_J
+#define DC_MS_J 2
+#endif
+constexpr int kMsP = DC_MS_P, kMsS = DC_MS_S, kMsTNT = DC_MS_TNT, kMsJ = DC_MS_J;
+constexpr int ms_tma_smem() { return kMsS * kMsTNT * kMsP * 4; }   // S x NW x 32*L words
+
 // Max-subarray grid: about one wave of resident CTAs (occupancy x SMs),
-// never more CTAs than tiles.
+// never more CTAs than there is work for.
 int ms_grid(dc_plan_t p) {
     static int grid = 0;
     if (!grid) {
-        int dev = 0, sms = 148, occ = 4;
+        int dev = 0, sms = 148, occ = 1;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, dc::nk4_maxsub<kNK4Threads, kNK4Chunk>,
-                                                      kNK4Threads, 0);
+        if (DC_MS_TMA) {
+            auto* k = dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ>;
+            cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, ms_tma_smem());
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kMsTNT, ms_tma_smem());
+        } else {
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                &occ, dc::nk4_maxsub<kNK4Threads, kNK4Chunk>, kNK4Threads, 0);
+        }
         grid = sms * (occ > 0 ? occ : 1);
     }
-    const int64_t tiles = num_tiles(p->n, kMsTile);
-    return (int)(tiles < grid ? tiles : grid);
+    const int64_t units = DC_MS_TMA ? num_tiles(p->n, (int64_t)kMsTNT * kMsP)   // >= 1 segment/warp
+                                    : num_tiles(p->n, kMsTile);
+    return (int)(units < grid ? units : grid);
 }
 
 dc_status ensure_ms_state(dc_plan_t p) {
@@ -504,8 +538,17 @@ dc_status maxsub_launch(dc_plan_t p, const int32_t* d_x, int64_t off, int mode,
     dc_status st = ensure_ms_state(p);
     if (st != DC_OK) return st;
     TimedScope ts(p, DC_KERNEL_NK4_MAXSUB);
-    dc::nk4_maxsub<kNK4Threads, kNK4Chunk><<<ms_grid(p), kNK4Threads, 0, p->stream>>>(
-        d_x, p->n, p->ms_tiles, p->ms_ticket, off, mode, out_res, out_tup);
+    const int grid = ms_grid(p);
+    if (DC_MS_TMA) {
+        // warp ranges of RW elements, a multiple of the 32*L-element segment
+        const int64_t warps = (int64_t)grid * (kMsTNT / 32), seg = 32LL * kMsP;
+        const int64_t R = ((p->n + warps - 1) / warps + seg - 1) / seg * seg;
+        dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ><<<grid, kMsTNT, ms_tma_smem(), p->stream>>>(
+            d_x, p->n, R, p->ms_tiles, p->ms_ticket, off, mode, out_res, out_tup);
+    } else {
+        dc::nk4_maxsub<kNK4Threads, kNK4Chunk><<<grid, kNK4Threads, 0, p->stream>>>(
+            d_x, p->n, p->ms_tiles, p->ms_ticket, off, mode, out_res, out_tup);
+    }
     DC_LAUNCHED(p);
     return DC_OK;
 }
@@ -652,20 +695,24 @@ dc_status ensure_mg_state(dc_plan_t p) {
 }
 
 
-// f4: the D&C sum through the generic O(1)-combine template (dc_reduce.cuh).
+// f4: the D&C sum through the generic O(1)-combine template (dc_reduce.cuh),
+// TMA-streamed warp segments of 32 x kSumL elements, one CTA per SM.
 constexpr int kSumThreads = 256;
-constexpr int kSumChunk = 64;
+constexpr int kSumL = 68;
+constexpr int kSumS = 2;
+constexpr size_t kSumSmem = dc::breadth_first_reduce_tma_smem<kSumThreads, kSumL, kSumS>();
 
 dc_status ensure_sum_state(dc_plan_t p) {
     if (p->sum_state) return DC_OK;
-    int dev = 0, sms = 148, occ = 4;
+    int dev = 0, sms = 148, occ = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &occ, dc::breadth_first_reduce<dc::SumI64, kSumThreads, kSumChunk>, kSumThreads, 0);
-    const int64_t tiles = num_tiles(p->n, (int64_t)kSumThreads * kSumChunk);
+    auto* k = dc::breadth_first_reduce_tma<dc::SumI64, kSumThreads, kSumL, kSumS>;
+    DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSumSmem));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kSumThreads, kSumSmem);
+    const int64_t units = num_tiles(p->n, (int64_t)kSumThreads * kSumL);   // >= 1 segment/warp
     const int64_t grid = (int64_t)sms * (occ > 0 ? occ : 1);
-    p->sum_grid = (int)(tiles < grid ? tiles : grid);
+    p->sum_grid = (int)(units < grid ? units : grid);
     void* ptr = nullptr;
     // parts[grid] | ticket (8 B) | result (8 B)
     if (cudaMalloc(&ptr, (size_t)(p->sum_grid + 2) * 8) != cudaSuccess) {
@@ -1211,10 +1258,11 @@ dc_status dc_run_sum_async(dc_plan_t p, const int32_t* d_x, int64_t* d_out) {
     if (!d_x || !d_out) return fail(DC_ERR_INVALID_ARG, "NULL argument");
     st = ensure_sum_state(p);
     if (st != DC_OK) return st;
-    dc::breadth_first_reduce<dc::SumI64, kSumThreads, kSumChunk>
-        <<<p->sum_grid, kSumThreads, 0, p->stream>>>(
-            d_x, p->n, p->sum_state, (unsigned int*)(p->sum_state + p->sum_grid),
-            (long long*)d_out);
+    if (!aligned16(d_x)) return fail(DC_ERR_INVALID_ARG, "x must be 16-byte aligned");
+    dc::breadth_first_reduce_tma<dc::SumI64, kSumThreads, kSumL, kSumS>
+        <<<p->sum_grid, kSumThreads, kSumSmem, p->stream>>>(
+            d_x, p->n, dc::breadth_first_reduce_tma_rw<kSumThreads, kSumL>(p->n, p->sum_grid),
+            p->sum_state, (unsigned int*)(p->sum_state + p->sum_grid), (long long*)d_out);
     DC_LAUNCHED(p);
     return DC_OK;
 }

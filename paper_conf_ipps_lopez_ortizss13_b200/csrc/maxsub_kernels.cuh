@@ -65,9 +65,9 @@ __device__ __forceinline__ MsTupT<I> ms_combine(const MsTupT<I>& L, const MsTupT
 
 // Left-to-right fold of one element x at index i: combine(T, leaf(x, i)),
 // which is Kadane's step with the tie rules above.  The running values are
-// kept in FP64: a thread folds at most 2^8 int32 elements, so every value is
-// an integer of magnitude < 2^40 (sentinel -2^62 is a power of two) and FP64
-// adds and compares are EXACT.  This moves the adds and compares onto the
+// kept in FP64: a thread folds at most 2^16 int32 elements, so every real
+// value is an integer of magnitude < 2^47 and FP64 adds and compares are
+// EXACT (the sentinel -2^62 absorbs rounding and stays below every real value).  This moves the adds and compares onto the
 // FP64 pipe and leaves only the selects on the integer ALU pipe, which the
 // int64 version saturated.  tup() converts back to int64.
 struct MsFold {
@@ -90,6 +90,22 @@ struct MsFold {
         best = better ? suf : best;
         bs = better ? ss : bs;
         be = better ? i : be;
+    }
+    // this = combine(this, R), R immediately right of this (ms_combine's rules
+    // on the FP64 fields; exact for real values, the sentinel stays below all)
+    __device__ __forceinline__ void absorb(const MsFold& R) {
+        const double lp = tot + R.pre;
+        const bool keep_pre = pre >= lp;
+        const double rs = R.tot + suf;
+        const bool left_suf = rs >= R.suf;
+        const double cross = suf + R.pre;
+        if (cross > best) { best = cross; bs = ss; be = R.pe; }
+        if (R.best > best) { best = R.best; bs = R.bs; be = R.be; }
+        pre = keep_pre ? pre : lp;
+        pe = keep_pre ? pe : R.pe;
+        suf = left_suf ? rs : R.suf;
+        ss = left_suf ? ss : R.ss;
+        tot += R.tot;
     }
     __device__ __forceinline__ MsTup tup() const {
         MsTup t;

@@ -1,0 +1,171 @@
+// maxsub_tma.cuh -- NK4 with TMA-streamed warp segments (the default NK4).
+//
+// Same method as nk4_maxsub (maxsub_kernels.cuh): contiguous pieces are
+// folded left to right (leaves + bottom levels), then combined in order
+// (top levels).  What changes is how the data arrives.  Loading a private
+// contiguous chunk per lane with 128-bit loads makes every warp load touch
+// 32 lines (32 L1 requests per instruction; the L1/TEX pipe bounded that
+// kernel), and one TMA copy per lane costs a request per 256 bytes.  Here
+// every WARP owns one contiguous range and streams it in segments of 32*L
+// elements, one 1-D TMA bulk copy per segment (S-stage ring, one mbarrier per
+// warp and stage); lane l folds the L contiguous elements [l*L, (l+1)*L) of
+// the segment from shared memory (L/4 odd: the 128-bit reads of a warp are
+// bank-conflict free) as J interleaved chains, and an ordered FP64 warp tree
+// folds the 32 lane summaries into the warp's running summary.  Warps, then
+// CTAs (atomic ticket, last CTA), are combined in order as before.
+#pragma once
+#include <cstdint>
+
+#include "maxsub_kernels.cuh"
+#include "sort_kernels.cuh"
+
+namespace dc {
+
+__device__ __forceinline__ MsFold ms_fold_shfl_down(const MsFold& t, int off) {
+    MsFold r;
+    r.tot = __shfl_down_sync(0xffffffffu, t.tot, off);
+    r.pre = __shfl_down_sync(0xffffffffu, t.pre, off);
+    r.suf = __shfl_down_sync(0xffffffffu, t.suf, off);
+    r.best = __shfl_down_sync(0xffffffffu, t.best, off);
+    r.pe = __shfl_down_sync(0xffffffffu, t.pe, off);
+    r.ss = __shfl_down_sync(0xffffffffu, t.ss, off);
+    r.bs = __shfl_down_sync(0xffffffffu, t.bs, off);
+    r.be = __shfl_down_sync(0xffffffffu, t.be, off);
+    return r;
+}
+
+// Ordered combine of the 32 lanes' folds (lane order = segment order); lane 0.
+__device__ __forceinline__ MsFold ms_fold_warp(MsFold t) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const MsFold r = ms_fold_shfl_down(t, off);
+        if ((lane & (2 * off - 1)) == 0) t.absorb(r);
+    }
+    return t;
+}
+
+template <int NT, int L, int S, int J>
+__global__ void __launch_bounds__(NT, 1)
+nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
+               dc_maxsub_tuple* __restrict__ parts, unsigned int* __restrict__ ticket,
+               long long off, int mode, dc_maxsub_result* __restrict__ out_res,
+               dc_maxsub_tuple* __restrict__ out_tup) {
+    static_assert(L % 4 == 0 && ((L / 4) & 1) == 1, "lane stride: 4 x odd words");
+    constexpr int NW = NT / 32;
+    constexpr int SEG = 32 * L;                                // elements per segment
+    constexpr int V = L / 4;                                   // 16-byte vectors per lane
+    constexpr int VJ = (V + J - 1) / J;                        // chain j: vectors [j*VJ, ...)
+    extern __shared__ __align__(16) int ms_smem[];            // [S][NW][SEG]
+    __shared__ __align__(8) uint64_t bars[S][NW];
+    __shared__ MsTup red[NW];
+    __shared__ MsTupG redg[NW];
+    __shared__ bool am_last;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+
+    // this warp's range [wbeg, wend) (RW is a multiple of SEG); CTA-local indices
+    const long long cbase = min(n, (long long)blockIdx.x * NW * RW);
+    const long long wbeg = min(n, ((long long)blockIdx.x * NW + warp) * RW);
+    const long long wend = min(n, wbeg + RW);
+    const int nseg = (int)((wend - wbeg + SEG - 1) / SEG);
+
+    if (lane == 0) {
+#pragma unroll
+        for (int s = 0; s < S; ++s) mbar_init(smem_addr(&bars[s][warp]), 1);
+    }
+    __syncwarp();
+    auto seg_ptr = [&](int s) { return ms_smem + (s * NW + warp) * SEG; };
+    auto issue = [&](int k) {          // lane 0: segment k -> stage k % S
+        const int s = k % S;
+        const uint32_t bar = smem_addr(&bars[s][warp]);
+        const long long g0 = wbeg + (long long)k * SEG;
+        const int cnt = (int)min((long long)SEG, wend - g0);
+        const int body = cnt & ~3;    // 16-byte part (g0 is 16-byte aligned)
+        mbar_arrive_expect_tx(bar, 4u * body);
+        if (body) bulk_g2s(smem_addr(seg_ptr(s)), x + g0, 4u * body, bar);
+    };
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < S; ++k)
+            if (k < nseg) issue(k);
+    }
+
+    MsFold acc;                        // lane 0: the warp's running summary
+    acc.init();
+    for (int k = 0; k < nseg; ++k) {
+        const int s = k % S;
+        mbar_wait(smem_addr(&bars[s][warp]), (uint32_t)((k / S) & 1));
+        const long long g0 = wbeg + (long long)k * SEG;
+        const int cnt = (int)min((long long)SEG, wend - g0);
+        const int* sl = seg_ptr(s) + lane * L;
+        const int e0 = lane * L;                     // first element of this lane
+        const int i0 = (int)(g0 - cbase) + e0;
+        MsFold f;
+        f.init();
+        if (cnt == SEG) {
+            MsFold g[J];
+#pragma unroll
+            for (int j = 0; j < J; ++j) g[j].init();
+#pragma unroll
+            for (int q = 0; q < VJ; ++q) {
+#pragma unroll
+                for (int j = 0; j < J; ++j) {
+                    if (j * VJ + q < V && q < VJ) {          // compile-time after unrolling
+                        const int o = 4 * (j * VJ + q);
+                        const int4 v = *reinterpret_cast<const int4*>(sl + o);
+                        g[j].step(v.x, i0 + o);
+                        g[j].step(v.y, i0 + o + 1);
+                        g[j].step(v.z, i0 + o + 2);
+                        g[j].step(v.w, i0 + o + 3);
+                    }
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < J; ++j) f.absorb(g[j]);
+        } else {                                     // the warp's last, partial segment
+            const int body = cnt & ~3;
+            for (int e = e0; e < min(cnt, e0 + L); ++e)
+                f.step(e < body ? sl[e - e0] : x[g0 + e], i0 + (e - e0));
+        }
+        f = ms_fold_warp(f);
+        if (lane == 0) acc.absorb(f);
+        __syncwarp();                                // every lane is done with stage s
+        if (lane == 0 && k + S < nseg) {
+            fence_proxy_async_smem();
+            issue(k + S);
+        }
+    }
+
+    // ---- warps -> CTA summary (thread 0), in order
+    if (lane == 0) red[warp] = acc.tup();
+    __syncthreads();
+    if (tid == 0) {
+        MsTupG c = ms_empty<long long>();
+        for (int w = 0; w < NW; ++w) c = ms_combine(c, ms_widen(red[w], cbase));
+        ms_store(&parts[blockIdx.x], c, 0);
+        __threadfence();
+        am_last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!am_last) return;
+
+    // ---- NK5: ordered combine of the per-CTA summaries (top levels)
+    __threadfence();
+    const int np = gridDim.x;
+    const int per = (np + NT - 1) / NT;
+    MsTupG a = ms_empty<long long>();
+    for (int q = tid * per; q < min(np, tid * per + per); ++q) a = ms_combine(a, ms_load_cg(parts + q));
+    a = ms_block_combine<NT>(a, redg);
+    if (tid == 0) {
+        if (mode == 0) {
+            out_res->sum = a.best;
+            out_res->start = a.bs + off;
+            out_res->end = a.be + off;
+        } else {
+            ms_store(out_tup, a, off);
+        }
+        *ticket = 0u;
+    }
+}
+
+}  // namespace dc

@@ -284,8 +284,11 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
     constexpr int TILE = NT * IT;
     const int tid = threadIdx.x;
     const uint32_t SK = smem_addr(sk);
+#ifndef DC_NK1_STOPW   // measurement knob only: stop the merge levels below this width
+#define DC_NK1_STOPW (1 << 30)
+#endif
 #pragma unroll 1
-    for (int w = IT; w < TILE; w *= 2) {
+    for (int w = IT; w < TILE && w < DC_NK1_STOPW; w *= 2) {
         // Levels whose pairs fit in one warp (2w <= 32*IT) only touch that
         // warp's own region: a warp barrier suffices and warps drift apart
         // (search / merge / write phases overlap across warps).
@@ -391,7 +394,9 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     }
 
     // ---- 2. leaves + in-thread levels
+#ifndef DC_NK1_NOREG   // measurement knob only
     thread_sort<K, IT, V>(k, ix);
+#endif
 
     // ---- 3. shared-memory merge levels: run width w -> 2w
     if constexpr (!V && !K::kNeedStable) {

@@ -52,6 +52,28 @@ static int run(const int32_t* x, long long n, void* parts, void* ticket, void* o
     return (int)cudaDeviceSynchronize();
 }
 
+// The TMA-streamed variant (warp segments of 32 x 36 elements, 3 stages).
+template <class M>
+static int run_tma(const int32_t* x, long long n, void* parts, void* ticket, void* out) {
+    constexpr int NT = 128, L = 36, S = 3;
+    constexpr size_t smem = dc::breadth_first_reduce_tma_smem<NT, L, S>();
+    auto* k = dc::breadth_first_reduce_tma<M, NT, L, S>;
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const long long units = (n + NT * L - 1) / (NT * L);
+    const int grid = (int)(units < 300 ? (units > 0 ? units : 1) : 300);
+    k<<<grid, NT, smem>>>(x, n, dc::breadth_first_reduce_tma_rw<NT, L>(n, grid),
+                          (typename M::T*)parts, (unsigned int*)ticket, (typename M::T*)out);
+    return (int)cudaDeviceSynchronize();
+}
+
+extern "C" int demo_maxsub_tma(const int32_t* x, long long n, void* parts, void* ticket,
+                               void* out) {
+    return run_tma<MaxsubMonoid>(x, n, parts, ticket, out);
+}
+extern "C" int demo_hash_tma(const int32_t* x, long long n, void* parts, void* ticket, void* out) {
+    return run_tma<HashMonoid>(x, n, parts, ticket, out);
+}
+
 extern "C" int demo_maxsub(const int32_t* x, long long n, void* parts, void* ticket, void* out) {
     return run<MaxsubMonoid>(x, n, parts, ticket, out);
 }

@@ -29,7 +29,8 @@ def dc():
     return m
 
 
-SUM_SIZES = [1, 2, 3, 7, 1000, 8191, 8192, 8193, 100_003, 1 << 20, (1 << 24) + 17]
+SUM_SIZES = [1, 2, 3, 7, 1000, 8191, 8192, 8193, 17407, 17408, 17409, 100_003, 1 << 20,
+             (1 << 24) + 17]
 
 
 @pytest.mark.parametrize("n", SUM_SIZES)
@@ -54,7 +55,7 @@ def demo():
                            "-std=c++17", "-shared", "-Xcompiler", "-fPIC", "-I",
                            os.path.join(ROOT, "include"), "-o", out, src])
     lib = ctypes.CDLL(out)
-    for f in (lib.demo_maxsub, lib.demo_hash):
+    for f in (lib.demo_maxsub, lib.demo_hash, lib.demo_maxsub_tma, lib.demo_hash_tma):
         f.argtypes = [ctypes.c_void_p, ctypes.c_longlong, ctypes.c_void_p, ctypes.c_void_p,
                       ctypes.c_void_p]
         f.restype = ctypes.c_int
@@ -68,22 +69,24 @@ def _bufs(words_per_t):
     return parts, ticket, out
 
 
-@pytest.mark.parametrize("n", [1, 5, 2047, 2048, 2049, 100_003, 1 << 20])
-def test_generic_template_maxsub_monoid(oracle_mod, demo, n):
+@pytest.mark.parametrize("kernel", ["plain", "tma"])
+@pytest.mark.parametrize("n", [1, 5, 2047, 2048, 2049, 4607, 4608, 4609, 100_003, 1 << 20])
+def test_generic_template_maxsub_monoid(oracle_mod, demo, n, kernel):
     x = dcgen.maxsub_input(n, "small", seed=9, device="cuda")
     parts, ticket, out = _bufs(8)
-    assert demo.demo_maxsub(x.data_ptr(), n, parts.data_ptr(), ticket.data_ptr(),
-                            out.data_ptr()) == 0
+    f = demo.demo_maxsub if kernel == "plain" else demo.demo_maxsub_tma
+    assert f(x.data_ptr(), n, parts.data_ptr(), ticket.data_ptr(), out.data_ptr()) == 0
     t = out.cpu().tolist()
     assert (t[3], t[6], t[7]) == oracle_mod.maxsub(x.cpu().numpy())
 
 
+@pytest.mark.parametrize("kernel", ["plain", "tma"])
 @pytest.mark.parametrize("n", [1, 33, 4096, 77_777, 1 << 20])
-def test_generic_template_hash_monoid(demo, n):
+def test_generic_template_hash_monoid(demo, n, kernel):
     x = dcgen.maxsub_input(n, "uniform", seed=10, device="cuda")
     parts, ticket, out = _bufs(2)
-    assert demo.demo_hash(x.data_ptr(), n, parts.data_ptr(), ticket.data_ptr(),
-                          out.data_ptr()) == 0
+    f = demo.demo_hash if kernel == "plain" else demo.demo_hash_tma
+    assert f(x.data_ptr(), n, parts.data_ptr(), ticket.data_ptr(), out.data_ptr()) == 0
     got = int(out.cpu()[0]) & ((1 << 64) - 1)
     m = (1 << 64) - 1
     h = 0
