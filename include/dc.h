@@ -295,6 +295,15 @@ dc_status dc_plan_set_mg_p2p(dc_plan_t plan, int32_t enable);
 /* Exchange in use: 1 fused, -1 all-to-all, 0 not decided yet / no communicator. */
 dc_status dc_plan_mg_exchange_mode(dc_plan_t plan, int32_t *mode);
 
+/* Phase times of the multi-GPU sorts run while dc_plan_enable_timing is on
+ * (CUDA events on the plan stream; each timed sort waits for itself):
+ * h_ms3[0] local sort (levels >= log2 G), [1] splitters incl. the host sync,
+ * [2] exchange + G-way merge (fused, or all-to-all + merge), summed over
+ * *sorts sorts; *keys_received = keys this rank took from peers (summed). */
+dc_status dc_plan_mg_phase_times(dc_plan_t plan, double *h_ms3, int64_t *sorts,
+                                 int64_t *keys_received);
+dc_status dc_plan_mg_reset_phases(dc_plan_t plan);
+
 /* Split matrix of the last multi-GPU sort: h_cmat[r*(world+1) + d] = number of
  * rank-r elements among the first d*m of the global stable order. */
 dc_status dc_plan_last_splits(dc_plan_t plan, int64_t *h_cmat);

@@ -108,6 +108,8 @@ _SIGS.update({
     "dc_plan_set_mg_stride": ([_P, _I64], ctypes.c_int),
     "dc_plan_last_splits": ([_P, _P], ctypes.c_int),
     "dc_plan_set_mg_p2p": ([_P, _I32], ctypes.c_int),
+    "dc_plan_mg_phase_times": ([_P, _P, ctypes.POINTER(_I64), ctypes.POINTER(_I64)], ctypes.c_int),
+    "dc_plan_mg_reset_phases": ([_P], ctypes.c_int),
     "dc_plan_mg_exchange_mode": ([_P, ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_mg_merge_peers": ([_P, ctypes.c_int, _P, _P, _P, _P, _P, _I32, _P, _P, _P, _P],
                           ctypes.c_int),
@@ -266,6 +268,18 @@ class Plan:
     def set_mg_p2p(self, enable: bool) -> None:
         """Fused exchange (merge reads the peers' shards) vs NCCL all-to-all."""
         _check(lib().dc_plan_set_mg_p2p(self._h, int(enable)))
+
+    def mg_phase_times(self) -> dict:
+        """{'local_sort','splitters','exchange_merge'} ms summed over timed sorts,
+        'sorts', 'keys_received' (dc_plan_mg_phase_times)."""
+        ms = (ctypes.c_double * 3)()
+        n, k = _I64(), _I64()
+        _check(lib().dc_plan_mg_phase_times(self._h, ms, ctypes.byref(n), ctypes.byref(k)))
+        return {"local_sort": ms[0], "splitters": ms[1], "exchange_merge": ms[2],
+                "sorts": n.value, "keys_received": k.value}
+
+    def mg_reset_phases(self) -> None:
+        _check(lib().dc_plan_mg_reset_phases(self._h))
 
     def exchange_mode(self) -> str:
         m = _I32()

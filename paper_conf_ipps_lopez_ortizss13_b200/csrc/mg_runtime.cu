@@ -387,7 +387,15 @@ struct MgCtx {
     int p2p = 0;                // 0 undecided, 1 fused, -1 NCCL all-to-all
     char* xbuf = nullptr;
     std::vector<void*> peers;
+    // phase timing (while the plan's kernel timing is on): events around
+    // [local sort | splitters | exchange + merge], accumulated per phase
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    double phase_ms[3] = {0, 0, 0};
+    int64_t phase_n = 0;
+    int64_t moved = 0, moved_total = 0;   // keys this rank received from peers (last / sum)
     ~MgCtx() {
+        for (auto e : ev)
+            if (e) cudaEventDestroy(e);
         if (coll) coll->unshare(peers);
         if (xbuf) cudaFree(xbuf);
         delete coll;
@@ -503,6 +511,13 @@ dc_status setup_p2p(dc_plan_t p, MgCtx* c) {
     return DC_OK;
 }
 
+dc_status mark(dc_plan_t p, MgCtx* c, int i) {
+    if (!p->timing) return DC_OK;
+    if (!c->ev[i]) MG_CU(cudaEventCreate(&c->ev[i]));
+    MG_CU(cudaEventRecord(c->ev[i], p->stream));
+    return DC_OK;
+}
+
 // keys/vals: this rank's sorted shard (in xbuf when fused); out: the caller's buffers.
 dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, uint32_t* vals,
                         uint32_t* out_k, uint32_t* out_v) {
@@ -543,6 +558,9 @@ dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, u
         if (scnt[d] < 0 || rcnt[d] < 0) return fail(DC_ERR_BAD_STATE, "negative split size");
     }
     if (tot != m) return fail(DC_ERR_BAD_STATE, "received element count != shard size");
+    c->moved = m - rcnt[me];
+    c->moved_total += c->moved;
+    MG_TRY(mark(p, c, 2));                 // splitters done (host-synchronised above)
     const size_t kb = al256((size_t)m * 4);
     if (c->p2p == 1) {
         // a8+a9 fused: merge straight from the peers' shards (NVLink reads)
@@ -609,15 +627,30 @@ dc_status mg_sort(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals) {
     auto run = [&]() -> dc_status {
         if (c->world == 1) return local_sort(p, kt, keys, vals);
         MG_TRY(setup_p2p(p, c));
+        MG_TRY(mark(p, c, 0));
         if (c->p2p == 1) {   // levels >= log2 G into the shared shard buffer
             const size_t kb = al256((size_t)c->m * 4);
             uint32_t* xk = (uint32_t*)c->xbuf;
             uint32_t* xv = vals ? (uint32_t*)(c->xbuf + kb) : nullptr;
             MG_TRY(local_sort(p, kt, keys, vals, xk, xv));
-            return sort_exchange(p, c, kt, xk, xv, keys, vals);
+            MG_TRY(mark(p, c, 1));
+            MG_TRY(sort_exchange(p, c, kt, xk, xv, keys, vals));
+        } else {
+            MG_TRY(local_sort(p, kt, keys, vals));    // levels >= log2 G: no communication
+            MG_TRY(mark(p, c, 1));
+            MG_TRY(sort_exchange(p, c, kt, keys, vals, keys, vals));
         }
-        MG_TRY(local_sort(p, kt, keys, vals));        // levels >= log2 G: no communication
-        return sort_exchange(p, c, kt, keys, vals, keys, vals);
+        MG_TRY(mark(p, c, 3));
+        if (p->timing) {                               // accumulate (waits for this sort)
+            MG_CU(cudaEventSynchronize(c->ev[3]));
+            for (int i = 0; i < 3; ++i) {
+                float ms = 0.f;
+                MG_CU(cudaEventElapsedTime(&ms, c->ev[i], c->ev[i + 1]));
+                c->phase_ms[i] += ms;
+            }
+            c->phase_n += 1;
+        }
+        return DC_OK;
     };
     const dc_status st = run();
     if (st != DC_OK) c->coll->abort();
@@ -754,6 +787,24 @@ dc_status dc_plan_set_mg_p2p(dc_plan_t p, int32_t enable) {
 dc_status dc_plan_mg_exchange_mode(dc_plan_t p, int32_t* mode) {
     if (!p || !mode) return dcx::fail(DC_ERR_INVALID_ARG, "NULL argument");
     *mode = p->mg ? p->mg->p2p : 0;
+    return DC_OK;
+}
+
+dc_status dc_plan_mg_phase_times(dc_plan_t p, double* h_ms3, int64_t* sorts,
+                                 int64_t* keys_received) {
+    if (!p || !h_ms3) return dcx::fail(DC_ERR_INVALID_ARG, "NULL argument");
+    if (!p->mg) return dcx::fail(DC_ERR_INVALID_ARG, "plan has no communicator");
+    for (int i = 0; i < 3; ++i) h_ms3[i] = p->mg->phase_ms[i];
+    if (sorts) *sorts = p->mg->phase_n;
+    if (keys_received) *keys_received = p->mg->moved_total;
+    return DC_OK;
+}
+
+dc_status dc_plan_mg_reset_phases(dc_plan_t p) {
+    if (!p || !p->mg) return dcx::fail(DC_ERR_INVALID_ARG, "plan has no communicator");
+    for (double& v : p->mg->phase_ms) v = 0;
+    p->mg->phase_n = 0;
+    p->mg->moved_total = 0;
     return DC_OK;
 }
 

@@ -339,8 +339,10 @@ def bench_main(args, wl, workloads, metric):
     ms = statistics.mean(times)
     splits = plan.last_splits() if G > 1 else [[0, m]]
 
-    # kernel breakdown (rank 0's own kernels): second loop with per-launch events
+    # kernel + phase breakdown (rank 0): second loop with per-launch events
     plan.enable_timing(True)
+    if G > 1:
+        plan.mg_reset_phases()
     for i in range(args.steps):
         keys.copy_(pristine)
         flush.zero_()
@@ -348,7 +350,22 @@ def bench_main(args, wl, workloads, metric):
         plan.sort_(keys, key_type="u32")
     torch.cuda.synchronize()
     kt = plan.kernel_times()
+    phases = plan.mg_phase_times() if G > 1 else None
     plan.enable_timing(False)
+    exchange = None
+    if phases and phases["sorts"]:
+        ns = phases["sorts"]
+        xms = phases["exchange_merge"] / ns
+        recv_b = 4 * phases["keys_received"] / ns          # bytes in over NVLink per step
+        exchange = {"mode": plan.exchange_mode(),
+                    "local_sort_ms": phases["local_sort"] / ns,
+                    "splitters_ms": phases["splitters"] / ns,
+                    "exchange_merge_ms": xms,
+                    "nvlink_bytes_in_per_rank": recv_b,
+                    "nvlink_gbs_in": recv_b / (xms / 1e3) / 1e9 if xms else None,
+                    "nvlink_frac_of_900": recv_b / (xms / 1e3) / 900e9 if xms else None,
+                    "note": "exchange_merge overlaps the NVLink reads with the first merge "
+                            "round when fused, so its GB/s is a lower bound on link use"}
     nk3_ms, nk3_n = kt["nk3_merge"]
     nk3_avg = nk3_ms / max(nk3_n, 1)
 
@@ -396,6 +413,7 @@ def bench_main(args, wl, workloads, metric):
                          "avg_launch_ms": nk3_avg,
                          "kernels_ms_per_step": {k: v[0] / args.steps for k, v in kt.items()}},
             "gpu_launches": launches,
+            "multi_gpu_phases": exchange,
             "e2e": {"value": n_total / (e2e_ms / 1e3), "unit": "keys/s", "ms_per_step": e2e_ms,
                     "h2d_bytes_per_step": 4 * n_total, "d2h_bytes_per_step": 4 * n_total},
             "cpu_baseline": None,

@@ -256,3 +256,29 @@ def test_merge_peers_separate_buffers(dc, oracle_mod, key_type, runs):
     got = out_k[:total].cpu().numpy().view(view)
     assert np.array_equal(got.view(np.uint32), ek.view(np.uint32))
     assert np.array_equal(out_v[:total].cpu().numpy().view(np.uint32), ev)
+
+
+@pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
+def test_loopback_phase_times(dc, p2p):
+    """Phase accounting with timing on: one entry per sort, keys received from
+    peers = shard size minus the rank's own part of its output slice."""
+    world, n = 3, 3 * 150_001
+
+    def fn(plan, r, m):
+        plan.enable_timing(True)
+        keys = dcgen.sort_keys(n, "uniform", seed=3, start=r * m, count=m, device="cuda")
+        plan.sort_(keys, key_type="u32")
+        ph = plan.mg_phase_times()
+        cm = plan.last_splits()
+        plan.enable_timing(False)
+        return ph, cm
+
+    res, errs, _ = run_ranks(dc, n, world, fn, p2p=p2p)
+    for e in errs:
+        if e is not None:
+            raise e
+    m = n // world
+    for r, (ph, cm) in enumerate(res):
+        assert ph["sorts"] == 1
+        assert ph["keys_received"] == m - (cm[r][r + 1] - cm[r][r])
+        assert ph["local_sort"] > 0 and ph["splitters"] > 0 and ph["exchange_merge"] > 0
