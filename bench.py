@@ -528,7 +528,8 @@ def run_dc_sum(args, wl, desc, n):
                    "l2": "flushed before every step (512 MiB write)"},
         "roofline": {"kernel": "breadth_first_reduce<SumI64> (one launch = the step)",
                      "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
-                     "frac": ach / peak, "traffic": None, "avg_launch_ms": ms,
+                     "frac": ach / peak, "traffic": ncu_traffic("breadth_first_reduce", wl),
+                     "avg_launch_ms": ms,
                      "algorithmic_bytes_per_launch": 4 * n, "peak_source": src},
         "gpu_launches": launches, "clocks": clk.summary(), "e2e": None, "cpu_baseline": None,
     }), flush=True)

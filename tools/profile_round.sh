@@ -3,7 +3,7 @@
 # of the default bench command, ncu --set full of the top kernels.
 mkdir -p gpurun_out
 timeout 600 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
-for w in sort_kv sort_u32_small maxsub; do
+for w in sort_kv sort_u32_small maxsub sum; do
   timeout 300 python bench.py --workload $w --steps 10 --warmup 3 > gpurun_out/bench_$w.json 2>&1
 done
 timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2>&1
@@ -19,4 +19,8 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk3_
   -o gpurun_out/prof_nk3_kv python bench.py --workload sort_kv --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk4_maxsub -s 3 -c 1 \
   -o gpurun_out/prof_nk4 python bench.py --workload maxsub --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk1_blocksort -s 1 -c 1 \
+  -o gpurun_out/prof_nk1_kv python bench.py --workload sort_kv --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > /dev/null 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:breadth_first_reduce -s 3 -c 1 \
+  -o gpurun_out/prof_sum python bench.py --workload sum --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 ls -la gpurun_out
