@@ -246,14 +246,50 @@ def test_full_size_2pow28_key_value(dc, dist):
     torch.cuda.empty_cache()
 
 
+def _assert_sorted_permutation_u32(k_in, k_out, samples=12, seed=0):
+    """Properties that hold at any size, checked without another sort:
+    the output is non-decreasing; it is a permutation of the input (histogram
+    of the top 16 key bits and the exact key sum agree); and sampled outputs
+    have the right rank -- out[i] = o satisfies #(in < o) <= i < #(in <= o),
+    counted over the input (the definition of the i-th smallest key)."""
+    n = k_in.numel()
+    kin = k_in.to(torch.int64) & 0xFFFFFFFF
+    kout = k_out.to(torch.int64) & 0xFFFFFFFF
+    assert bool((kout[1:] >= kout[:-1]).all())
+    assert int(kin.sum()) == int(kout.sum())
+    assert torch.equal(torch.bincount(kin >> 16, minlength=1 << 16),
+                       torch.bincount(kout >> 16, minlength=1 << 16))
+    g = torch.Generator().manual_seed(seed)
+    idx = [0, n - 1] + torch.randint(0, n, (samples,), generator=g).tolist()
+    for i in idx:
+        o = int(kout[i])
+        assert int((kin < o).sum()) <= i < int((kin <= o).sum())
+
+
 @pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "few"])
 def test_full_size_2pow28_keys(dc, dist):
     n = 1 << 28
     keys = dcgen.sort_keys(n, dist, seed=3, device="cuda")
-    ref = torch.sort(keys.view(torch.uint32).to(torch.int64) & 0xFFFFFFFF, stable=True).values
+    k_in = keys.clone()
     dc.Plan(n).sort_(keys, key_type="u32")
     torch.cuda.synchronize()
-    assert torch.equal(keys.to(torch.int64) & 0xFFFFFFFF, ref)
+    _assert_sorted_permutation_u32(k_in, keys)
+
+
+def test_max_size_keys(dc):
+    """n = 2^31 - 1, the largest per-GPU size of the ABI (17 global passes,
+    int32 co-ranks at their limit)."""
+    n = (1 << 31) - 1
+    keys = dcgen.sort_keys(n, "uniform", seed=7, device="cuda")
+    k_in = keys.clone()
+    plan = dc.Plan(n)
+    assert plan.schedule("u32")["global_passes"] == 17
+    plan.sort_(keys, key_type="u32")
+    torch.cuda.synchronize()
+    del plan
+    _assert_sorted_permutation_u32(k_in, keys, samples=6)
+    del keys, k_in
+    torch.cuda.empty_cache()
 
 
 # ------------------------------------------------------------ max-subarray
