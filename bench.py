@@ -333,8 +333,12 @@ def run_dc(args, wl):
     nk3_avg = nk3_ms / max(nk3_n, 1)
     achieved = bytes_per_key * n / (nk3_avg / 1e3) / 1e9 if nk3_n else None
     nk1_avg = nk1_ms / max(nk1_n, 1)
+    two = sched["hbm_passes"] < sched["global_passes"]
     roofline = {
-        "kernel": "nk3_merge (one global merge level)",
+        "kernel": ("nk3_merge4 (one HBM pass = two merge levels: 4-way tile merge; the pass's "
+                   "exact 4-run selection is nk2_partition)") if two
+                  else "nk3_merge (one global merge level)",
+        "levels_per_launch": 2 if two else 1,
         "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
         "frac": achieved / peak if achieved else None,
         "traffic": ncu_traffic("nk3_merge", wl),
@@ -374,6 +378,7 @@ def run_dc(args, wl):
         "config": {"workload": wl, "description": desc, "n": n, "dist": args.dist,
                    "key_type": "u32", "values": kv, "tile": sched["tile"],
                    "fused_levels": sched["fused_levels"], "global_passes": sched["global_passes"],
+                   "hbm_passes": sched["hbm_passes"],
                    "l2": "flushed before every step (512 MiB write); input 1 GiB > L2",
                    "step_ms_min": min(step_ms), "step_ms_max": max(step_ms),
                    "instrumented_step_ms": ms_instr,

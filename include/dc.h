@@ -100,14 +100,17 @@ dc_status dc_plan_levels(dc_plan_t plan, int32_t *num_levels, int64_t *nodes,
  * values): the fused bottom kernel sorts tiles of `tile` keys (the leaves plus
  * fused_levels = ceil(log2(tile)) levels of the binary tree, entirely on
  * chip); global_passes = ceil(log2(ceil(n/tile))) levels remain, executed in
- * hbm_passes passes over HBM (keys-only sorts fold two levels per pass when
- * enabled with dc_plan_set_two_level).  Any output pointer may be NULL. */
+ * hbm_passes passes over HBM (keys-only u32/i32 sorts of n >= 2^23 fold two
+ * levels per pass unless disabled with dc_plan_set_two_level).  Any output
+ * pointer may be NULL. */
 dc_status dc_plan_schedule(dc_plan_t plan, dc_key_type key_type, int32_t with_vals,
                            int32_t *tile, int32_t *fused_levels, int32_t *global_passes,
                            int32_t *hbm_passes);
 
-/* Enable or disable (default) the two-levels-per-pass schedule of keys-only
- * sorts (a 4-way merge per HBM pass).  Results are identical. */
+/* Enable (default) or disable the two-levels-per-pass schedule of keys-only
+ * u32/i32 sorts with n >= 2^23 (every pass merges groups of four
+ * runs -- an exact 4-run selection per output tile, then a 4-way tile merge;
+ * sort4_kernels.cuh).  Results are identical either way. */
 dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
 
 /* Enable (default) or disable CUDA-graph replay of the sort's launch sequence:

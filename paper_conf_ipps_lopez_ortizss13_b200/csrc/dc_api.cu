@@ -23,7 +23,7 @@
 #include "maxsub_kernels.cuh"
 #include "mg_kernels.cuh"
 #include "sort_kernels.cuh"
-#include "sort2_kernels.cuh"
+#include "sort4_kernels.cuh"
 #include "maxsub_tma.cuh"
 
 namespace {
@@ -129,19 +129,27 @@ int global_passes(int64_t n, int64_t tile) {
 
 size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kMinTout) + 1; }
 
-// Two-level passes (keys-only): granule g = T/4 of the 4-way output tile T.
-constexpr int kTwoT = kCfgFast.tout();
-int nk3_2l_smem_bytes() { return dc::nk3_2l_words(kCfgFast.tout(), kCfgFast.it) * 4; }
-constexpr int kTwoG = kTwoT / 4;
-static_assert(kTwoT % 4 == 0 && (4 * kCfgFast.tile()) % kTwoT == 0, "two-level tiling");
+// Two-level passes (keys-only): 4-way output tiles of kTwoT keys, one cut
+// vector (4 ints) per tile; every group of 4 runs is cut into ceil(4w/kTwoT)
+// tiles (at most one more per group than n / kTwoT in total).
+#ifndef DC_TWO_NT
+#define DC_TWO_NT 768
+#endif
+#ifndef DC_TWO_IT
+#define DC_TWO_IT 33
+#endif
+constexpr int kTwoNT = DC_TWO_NT;
+constexpr int kTwoIT = DC_TWO_IT;
+constexpr int kTwoT = kTwoNT * kTwoIT;
+int nk3_2l_smem_bytes() { return dc::m4_smem_bytes(kTwoT, kTwoIT); }
 
-size_t two_level_tab_entries(int64_t n) {
-    // pairs at the smallest width (w = tile): 2*ceil(n/4w), (2w/g + 1) entries each
+size_t two_level_tab_entries(int64_t) { return 0; }
+size_t two_level_bnd_entries(int64_t n) {
+    // groups at the smallest width (w = tile) have the most tiles
     const int64_t w = kCfgFast.tile();
-    const int64_t pairs = 2 * ((n + 4 * w - 1) / (4 * w));
-    return (size_t)(pairs * (2 * w / kTwoG + 1));
+    const int64_t groups = (n + 4 * w - 1) / (4 * w);
+    return 4 * ((size_t)(groups * num_tiles(4 * w, kTwoT)) + 2);
 }
-size_t two_level_bnd_entries(int64_t n) { return 3 * ((size_t)num_tiles(n, kTwoT) + 2); }
 
 size_t scratch_needed(int64_t n, bool vals) {
     size_t kb = align_up((size_t)n * 4, 256);
@@ -271,7 +279,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     }
 
     // Levels over HBM: P = ceil(log2(ceil(n/tile))).  Keys-only sorts fold
-    // two levels into one pass (4-way groups, sort2_kernels.cuh); with P odd
+    // two levels into one pass (4-way groups, sort4_kernels.cuh); with P odd
     // one single-level pass goes first.
     const int P = global_passes(n, C.tile());
     constexpr bool kTwoCapable = !V && !K::kNeedStable && !SMALL;
@@ -378,31 +386,32 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     if constexpr (kTwoCapable) {
         if (two) {
             int* tab = split + align_up(split_entries(n) * 4, 256) / 4;
-            int* bnd = tab + align_up(two_level_tab_entries(n) * 4, 256) / 4;
-            auto* k32 = dc::nk3_merge2<C.nt3, C.it, K>;
+            dc::Cut4* cuts = (dc::Cut4*)(tab + align_up(two_level_tab_entries(n) * 4, 256) / 4);
+            auto* k32 = dc::nk3_merge4<kTwoNT, kTwoIT, K>;
             const int smem2 = nk3_2l_smem_bytes();
-            static bool attr2 = false;
-            if (!attr2) {
+            static int grid2 = 0;
+            if (!grid2) {
                 DC_CUDA(p, cudaFuncSetAttribute(k32, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                 smem2));
-                attr2 = true;
+                int dev = 0, sms = 148, occ = 1;
+                cudaGetDevice(&dev);
+                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, kTwoNT + 64, smem2);
+                grid2 = sms * (occ > 0 ? occ : 1);
             }
-            const int tiles2 = (int)num_tiles(n, kTwoT);
             for (; w < n; w *= 4) {
-                const int K1 = (int)(2 * w / kTwoG + 1);
-                const int64_t entries = 2 * ((n + 4 * w - 1) / (4 * w)) * K1;
+                const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), kTwoT);
+                const int tiles2 = (int)(((n + 4 * w - 1) / (4 * w)) * tpg);
                 {
                     TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-                    dc::nk2a_granules<K><<<(unsigned)((entries + 255) / 256), 256, 0, p->stream>>>(
-                        cur_k, n, w, kTwoG, K1, entries, tab);
-                    DC_LAUNCHED(p);
-                    dc::nk2b_partition2<K><<<(tiles2 + 3) / 4, 128, 0, p->stream>>>(
-                        cur_k, n, w, kTwoT, kTwoG, K1, tab, tiles2, bnd);
+                    dc::nk2_select4<K><<<(tiles2 + 3) / 4, 128, 0, p->stream>>>(
+                        cur_k, n, w, kTwoT, tpg, tiles2, cuts);
                     DC_LAUNCHED(p);
                 }
                 {
                     TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                    k32<<<tiles2, C.nt3 + 32, smem2, p->stream>>>(cur_k, oth_k, n, w, bnd);
+                    k32<<<std::min(tiles2, grid2), kTwoNT + 64, smem2, p->stream>>>(
+                        cur_k, oth_k, n, w, tpg, cuts, tiles2);
                     DC_LAUNCHED(p);
                 }
                 std::swap(cur_k, oth_k);
@@ -772,6 +781,7 @@ dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t*
     p->b = b;
     p->base_size = base_size;
     if (const char* e = std::getenv("DC_PIPE_CHUNKS")) p->pipe_chunks = std::atoi(e);  // tuning
+    if (const char* e = std::getenv("DC_TWO_LEVEL")) p->two_level = std::atoi(e) != 0;  // tuning
     // Level i: a^i nodes of size ceil(n / b^i); stop at the first level whose
     // size is <= base_size (leaves at level log_b n for base 1).
     int64_t nodes = 1, size = n, bpow = 1;

@@ -1,0 +1,488 @@
+// sort4_kernels.cuh -- two levels of the merge tree per HBM pass.
+//
+// A pass over runs of width w merges every group of four adjacent runs
+// (R0 R1 R2 R3) into one run of 4w: merge(merge(R0, R1), merge(R2, R3)),
+// i.e. Alg 7's combine applied at two consecutive levels of the
+// binary tree, the intermediate runs living only in shared memory.  Every
+// merge is the stable one of the one-level pass (earlier run wins ties), so
+// the output order is the composite order (key, run, position) and the result
+// is bit-identical to two one-level passes; only the HBM traffic halves.
+//
+//   NK2-4 select : for every output tile boundary of a group, the exact cut
+//                  (c0, c1, c2, c3), c_q = #R_q elements among the first d
+//                  outputs -- a warp-parallel multi-sequence selection that
+//                  brackets 8 pivots per run every round (one dependent load
+//                  per round instead of a nested binary search);
+//   NK3-4 merge  : persistent CTAs, double-buffered: the four pieces of the
+//                  next tile arrive by TMA while the current tile is merged
+//                  (stage 1: piece pairs -> X, Y in registers; stage 2: X with
+//                  Y in a bitonic layout), the tile leaves by a TMA bulk store.
+//
+// Tiles: every group is cut into tpg = ceil(min(4w, n) / T) output tiles of T
+// keys (the last one of a group short, trailing ones of the last group
+// empty); tile j is local tile j % tpg of group j / tpg.  Positions inside a
+// group fit in int32 (n < 2^31).
+//
+// Keys-only (u32 / i32): equal keys are identical bit patterns, so the merges
+// use +inf pads instead of bounds checks (see merge_pad).
+#pragma once
+#include <cstdint>
+
+namespace dc {
+
+struct Cut4 {
+    int c[4];
+};
+
+// Tile j of a two-level pass over runs of width w in [0, n): its group start
+// s, the four run lengths, the group length and the tile's output range
+// [d0, d1) relative to s (empty when d0 >= tot, in the last group).
+struct Tile4Geo {
+    long long s;
+    int l[4];
+    int tot, d0, d1;
+    __device__ __forceinline__ Tile4Geo(long long n, long long w, int T, int tpg, int j) {
+        const int G = j / tpg;
+        s = (long long)G * 4 * w;
+        tot = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            l[q] = (int)max(0LL, min(w, n - s - q * w));
+            tot += l[q];
+        }
+        const long long e0 = (long long)(j - G * tpg) * T;   // may pass tot (empty tile)
+        d0 = (int)min(e0, (long long)tot);
+        d1 = (int)min(e0 + T, (long long)tot);
+    }
+};
+
+// Composite order of the 4-way stable merge: element x of run qx precedes
+// element e of run qe iff x < e, or x == e and qx < qe (same run: position).
+template <class K>
+__device__ __forceinline__ bool precedes(uint32_t x, int qx, uint32_t e, int qe) {
+    return K::lt(x, e) | ((!K::lt(e, x)) & (qx < qe));
+}
+
+// Position of pivot t (0..7) in a window [lo, lo + W): evenly spaced when
+// W >= 9 (strictly inside the window), every position when W <= 8.
+__device__ __forceinline__ int sel4_pivot(int lo, int W, int step, int t) {
+    return lo + (W >= 9 ? (t + 1) * step : min(t, W - 1));
+}
+
+// ------------------------------------------------------------------ NK2-4
+#ifndef DC_SEL4_EXACT_FROM
+#define DC_SEL4_EXACT_FROM 48
+#endif
+// One warp per tile boundary.  Lane L owns pivot t = L & 7 of run q = L >> 3.
+// Invariant: lo_q <= c_q <= hi_q, with the values R_q[lo_q - 1] (taken) and
+// R_q[hi_q] (not taken) known.  Every round each run with a non-empty window
+// puts 8 pivots in it; a pivot E (run q, position p) is
+//   * taken      if it precedes a known taken edge of another run, or if
+//                 p + sum_q' U_q'(E) < d,
+//   * not taken  if a known untaken edge precedes it, or p + sum L_q'(E) >= d,
+// where [L_q', U_q'] brackets #R_q' elements preceding E between the
+// neighbouring pivots of run q' (positions in closed form, values by
+// shuffle).  The largest taken pivot raises lo_q, the smallest untaken one
+// lowers hi_q.  Once every window has <= 8 elements all of them are pivots,
+// the brackets are exact and every window closes: c_q = lo_q.
+template <class K>
+__global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long long w, int T,
+                            int tpg, int num_tiles, Cut4* __restrict__ cut) {
+    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    if (j >= num_tiles) return;                       // warp-uniform
+    const int lane = threadIdx.x & 31;
+    const int q = lane >> 3, t = lane & 7;
+    const Tile4Geo g(n, w, T, tpg, j);
+    const int d = g.d0;
+    if (d >= g.tot) return;                           // empty tile (last group)
+    const uint32_t* R[4];
+#pragma unroll
+    for (int r = 0; r < 4; ++r) R[r] = src + g.s + r * w;
+    const uint32_t* Rq = R[0];
+#pragma unroll
+    for (int r = 1; r < 4; ++r)
+        if (q == r) Rq = R[r];
+    int lo[4], hi[4];
+    uint32_t elo[4], ehi[4];
+    {
+        // initial windows and their edge values (lane r: R_r[lo_r - 1], lane 4+r: R_r[hi_r])
+        uint32_t ev = 0;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            lo[r] = max(0, d - (g.tot - g.l[r]));
+            hi[r] = min(g.l[r], d);
+            const int pos = lane == r ? lo[r] - 1 : hi[r];
+            if ((lane == r || lane == 4 + r) && pos >= 0 && pos < g.l[r]) ev = __ldg(R[r] + pos);
+        }
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            elo[r] = __shfl_sync(0xffffffffu, ev, r);
+            ehi[r] = __shfl_sync(0xffffffffu, ev, 4 + r);
+        }
+    }
+#ifdef DC_SEL4_MAXROUNDS
+    int dbg_rounds = 0;
+#endif
+    for (int round = 0;; ++round) {
+        // Progress guard: from round DC_SEL4_EXACT_FROM on, every undecided
+        // pivot's brackets are resolved by exact binary searches, so every
+        // round decides every pivot (never reached on the tested inputs).
+        const bool exact = round >= DC_SEL4_EXACT_FROM;
+#ifdef DC_SEL4_MAXROUNDS
+        if (++dbg_rounds > DC_SEL4_MAXROUNDS) {
+            if (lane == 0) printf("select4 stall j=%d d=%d\n", j, d);
+            break;
+        }
+#endif
+        int W[4], st[4], open = 0;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            W[r] = hi[r] - lo[r];
+            st[r] = W[r] / 9;
+            open |= W[r];
+        }
+        if (open == 0) break;
+        int Wq = W[0], loq = lo[0], stq = st[0];
+#pragma unroll
+        for (int r = 1; r < 4; ++r)
+            if (q == r) { Wq = W[r]; loq = lo[r]; stq = st[r]; }
+        const bool active = Wq > 0;
+        const int p = sel4_pivot(loq, Wq, stq, t);
+        const uint32_t v = active ? __ldg(Rq + p) : 0u;
+        int SL = p, SU = p;
+        bool dt = false, du = false;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            // #pivots of run r preceding this lane's pivot (search over lanes 8r..8r+7)
+            int a = 0;                                   // in [0, 8]
+#pragma unroll
+            for (int step = 4; step >= 1; step >>= 1) {
+                const uint32_t V = __shfl_sync(0xffffffffu, v, 8 * r + a + step - 1);
+                if (precedes<K>(V, r, v, q)) a += step;
+            }
+            {
+                const uint32_t V = __shfl_sync(0xffffffffu, v, 8 * r + 7);
+                if (a == 7 && precedes<K>(V, r, v, q)) a = 8;
+            }
+            if (r == q) continue;
+            if (lo[r] > 0 && !precedes<K>(elo[r], r, v, q)) dt = true;      // E before a taken edge
+            if (hi[r] < g.l[r] && precedes<K>(ehi[r], r, v, q)) du = true;  // untaken edge before E
+            int Lp = lo[r], Up = hi[r];
+            if (W[r] > 0) {
+                if (a > 0) Lp = sel4_pivot(lo[r], W[r], st[r], a - 1) + 1;
+                if (a < 8) Up = sel4_pivot(lo[r], W[r], st[r], a);
+            }
+            if (exact && !(dt | du) && active) {
+                int x0 = Lp, x1 = Up;                    // first position not preceding E
+                while (x0 < x1) {
+                    const int mid = (x0 + x1) >> 1;
+                    if (precedes<K>(__ldg(R[r] + mid), r, v, q)) x0 = mid + 1;
+                    else x1 = mid;
+                }
+                Lp = Up = x0;
+            }
+            SL += Lp;
+            SU += Up;
+        }
+        // The brackets hold only for a pivot between every other run's edges;
+        // an edge decision takes precedence (dt and du exclude each other).
+        const bool taken = active && (dt || (!du && SU < d));
+        const bool untaken = active && (du || (!dt && SL >= d));
+        const unsigned mt = __ballot_sync(0xffffffffu, taken);
+        const unsigned mu = __ballot_sync(0xffffffffu, untaken);
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+            const unsigned gt = (mt >> (8 * r)) & 0xffu, gu = (mu >> (8 * r)) & 0xffu;
+            const int lo0 = lo[r];                        // this round's pivot base
+            if (gt) {                                     // largest taken pivot
+                const int tt = 31 - __clz(gt);
+                elo[r] = __shfl_sync(0xffffffffu, v, 8 * r + tt);
+                lo[r] = sel4_pivot(lo0, W[r], st[r], tt) + 1;
+            }
+            if (gu) {                                     // smallest untaken pivot
+                const int tu = __ffs(gu) - 1;
+                ehi[r] = __shfl_sync(0xffffffffu, v, 8 * r + tu);
+                hi[r] = sel4_pivot(lo0, W[r], st[r], tu);
+            }
+        }
+    }
+    if (lane == 0) {
+        Cut4 c;
+#pragma unroll
+        for (int r = 0; r < 4; ++r) c.c[r] = lo[r];
+        cut[j] = c;
+    }
+}
+
+// ------------------------------------------------------------------ NK3-4
+// Pad-safe serial merge of IT outputs (keys only): each piece in shared memory
+// is followed by >= IT pads of K::kPad (the maximum key).  "take B iff b < a"
+// then never needs a bound: an exhausted side reads pads, which lose against
+// every smaller key, and against an equal (maximum) key the pad is emitted in
+// its place -- the same bit pattern, and only maximum keys remain.
+template <class K, int IT>
+__device__ __forceinline__ void merge_pad(uint32_t ai, uint32_t bi, uint32_t (&out)[IT]) {
+    uint32_t a = lds(ai), b = lds(bi);
+    const uint32_t c0 = ai + bi;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+        const bool p = K::lt(b, a);
+        out[j] = p ? b : a;
+        if (!p) ai += 4u;
+        bi = c0 + 4u * (j + 1) - ai;
+        const uint32_t v = lds(p ? bi : ai);
+        if (p) b = v; else a = v;
+    }
+}
+
+// Per-buffer tile descriptor, written by the issuing thread.
+struct Tile4 {
+    long long g0[4];  // global start of each piece
+    int len[4];
+    int at[4];        // word offset of each piece's first element in the buffer
+    long long out;    // global output offset of the tile
+    int total;
+    int pad_;
+};
+
+// Shared words per buffer: the four pieces with their alignment heads and IT
+// pads each, rounded; a guard of IT + 4 words sits below every buffer (the
+// bitonic stage-2 merge of a short tile may read just below it).
+__host__ __device__ constexpr int m4_guard(int IT) { return (IT + 4 + 3) / 4 * 4; }
+__host__ __device__ constexpr int m4_buf_words(int T, int IT) {
+    return m4_guard(IT) + (T + 4 * (IT + 8) + 16 + 3) / 4 * 4;
+}
+__host__ __device__ constexpr int m4_smem_bytes(int T, int IT) { return 2 * m4_buf_words(T, IT) * 4; }
+
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+// Barrier among the NC consumer threads only (named barrier 1).
+template <int NC>
+__device__ __forceinline__ void consumer_sync() {
+    asm volatile("bar.sync 1, %0;" ::"n"(NC) : "memory");
+}
+
+// NK3-4: persistent 4-way tile merge, warp-specialised and double-buffered.
+// NT + 64 threads.  Consumers (threads 0..NT+31): stage 1 needs up to NT + 1
+// windows of IT outputs (X and Y windowed separately), stage 2 uses NT
+// threads.  Producer (the last warp): fills a buffer with a tile (pads and
+// ragged piece ends by plain stores, the 16-byte-aligned interior of every
+// piece by TMA), and once the consumers have written a tile's output back
+// into its buffer, bulk-stores it and refills the buffer with the tile two
+// ahead.  full[b]: tile data present (producer arrive + TMA bytes);
+// empty[b]: output written (one arrive per consumer warp).  Tiles
+// J = blockIdx.x + i * gridDim.x; empty tiles (end of the last group) pass
+// through with no work.
+#ifndef DC_M4_MINB   // CTAs per SM the register budget is sized for (1: 768 x 33 tiles)
+#define DC_M4_MINB 1
+#endif
+template <int NT, int IT, class K>
+__global__ void __launch_bounds__(NT + 64, DC_M4_MINB)
+nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long long n, long long w,
+           int tpg, const Cut4* __restrict__ cut, int num_tiles) {
+    static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
+    constexpr int T = NT * IT;
+    constexpr int NC = NT + 32;                        // consumer threads
+    constexpr int BW = m4_buf_words(T, IT);
+    constexpr int GU = m4_guard(IT);
+    extern __shared__ __align__(16) uint32_t sm[];
+    __shared__ __align__(8) uint64_t full[2], empty[2];
+    __shared__ Tile4 meta[2];
+    const int tid = threadIdx.x;
+    const int lane = tid & 31;
+    const uint32_t SM0 = smem_addr(sm);
+    const long long n4 = n & ~3LL;
+    const int my_tiles = (int)blockIdx.x < num_tiles
+                             ? (num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+
+    if (tid == 0) {
+#pragma unroll
+        for (int b = 0; b < 2; ++b) {
+            mbar_init(smem_addr(&full[b]), 1);
+            mbar_init(smem_addr(&empty[b]), NC / 32);
+        }
+    }
+    __syncthreads();
+
+    if (tid >= NC) {
+        // ------------------------------------------------------ producer warp
+        // Fill buffer b with tile J: cut vectors (start; end = next tile's
+        // start or the run lengths at the end of a group) -> pieces.  The TMA
+        // copies each piece's 16-byte-aligned interior [g0 & ~3, tend); the
+        // lanes store the ragged end (< 4 words, or the part at/after n4) and
+        // IT pads behind each piece.
+        auto fill = [&](int J, int b) {
+            const Tile4Geo g(n, w, T, tpg, J);
+            int c0[4], c1[4];
+            if (g.d0 < g.tot) {
+                const Cut4 a = cut[J];
+                Cut4 e;
+                if (g.d1 == g.tot) {
+#pragma unroll
+                    for (int r = 0; r < 4; ++r) e.c[r] = g.l[r];
+                } else {
+                    e = cut[J + 1];
+                }
+#pragma unroll
+                for (int r = 0; r < 4; ++r) { c0[r] = a.c[r]; c1[r] = e.c[r]; }
+            } else {
+#pragma unroll
+                for (int r = 0; r < 4; ++r) c0[r] = c1[r] = 0;
+            }
+            Tile4 m;
+            m.out = g.s + g.d0;
+            m.total = max(0, g.d1 - g.d0);
+            uint32_t* buf = sm + b * BW + GU;
+            const uint32_t base = SM0 + 4u * (b * BW + GU);
+            uint32_t bytes = 0;
+            long long tend[4];
+            int o = 0;
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                m.g0[r] = g.s + r * w + c0[r];
+                m.len[r] = c1[r] - c0[r];
+                m.at[r] = o + (int)(m.g0[r] & 3);
+                const long long al0 = m.g0[r] & ~3LL;
+                long long al1 = (m.g0[r] + m.len[r]) & ~3LL;
+                if (al1 > n4) al1 = n4;
+                if (al1 < al0) al1 = al0;
+                tend[r] = al1;
+                if (al1 > al0) bytes += (uint32_t)(4 * (al1 - al0));
+                o = (m.at[r] + m.len[r] + IT + 1 + 3) & ~3;
+                const int e0 = (int)(max(al1, m.g0[r]) - m.g0[r]);
+                for (int e = e0 + lane; e < m.len[r] + IT; e += 32)
+                    buf[m.at[r] + e] = e < m.len[r] ? src[m.g0[r] + e] : K::kPad;
+            }
+            __syncwarp();
+            if (lane == 0) {
+                meta[b] = m;
+                const uint32_t fb = smem_addr(&full[b]);
+                mbar_arrive_expect_tx(fb, bytes);        // release: pads + meta
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    const long long al0 = m.g0[r] & ~3LL;
+                    if (tend[r] > al0)
+                        bulk_g2s(base + 4u * (m.at[r] - (int)(m.g0[r] & 3)), src + al0,
+                                 (uint32_t)(4 * (tend[r] - al0)), fb);
+                }
+            }
+        };
+        if (my_tiles > 0) fill(blockIdx.x, 0);
+        if (my_tiles > 1) fill(blockIdx.x + gridDim.x, 1);
+        for (int i = 0; i < my_tiles; ++i) {
+            const int b = i & 1;
+            mbar_wait(smem_addr(&empty[b]), (i >> 1) & 1);   // output of tile i written
+            if (lane == 0) {
+                const Tile4 m = meta[b];
+                const int body = m.total & ~3;
+                if (body > 0) {
+                    bulk_s2g(dst + m.out, SM0 + 4u * (b * BW + GU), 4u * body);
+                    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                }
+                if (i + 2 < my_tiles) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+            }
+            __syncwarp();
+            if (i + 2 < my_tiles) fill(blockIdx.x + (i + 2) * gridDim.x, b);
+        }
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+        return;
+    }
+
+    // ---------------------------------------------------------- consumers
+#ifndef DC_M4_SKIP   // measurement knob: bit 0 skips stage 1, bit 1 stage 2
+#define DC_M4_SKIP 0
+#endif
+    for (int i = 0; i < my_tiles; ++i) {
+        const int b = i & 1;
+        uint32_t* buf = sm + b * BW + GU;
+        const uint32_t B0 = SM0 + 4u * (b * BW + GU);
+        mbar_wait(smem_addr(&full[b]), (i >> 1) & 1);
+        const Tile4 m = meta[b];
+
+        // stage 1: X = merge(P0, P1), Y = merge(P2, P3), IT-output windows
+        const int nx = m.len[0] + m.len[1], ny = m.len[2] + m.len[3];
+        const int wx = (nx + IT - 1) / IT, wy = (ny + IT - 1) / IT;
+        uint32_t k[IT];
+        int valid = 0, base_out = 0;
+        bool up = true;
+        if (!(DC_M4_SKIP & 1) && tid < wx + wy) {
+            const bool first = tid < wx;
+            const int na = first ? m.len[0] : m.len[2], nb = first ? m.len[1] : m.len[3];
+            const uint32_t A = B0 + 4u * (first ? m.at[0] : m.at[2]);
+            const uint32_t Bq = B0 + 4u * (first ? m.at[1] : m.at[3]);
+            const int diag = (first ? tid : tid - wx) * IT;
+            const int ci = corank_smem<K>(A, na, Bq, nb, diag);
+            merge_pad<K, IT>(A + 4u * ci, Bq + 4u * (diag - ci), k);
+            valid = min(IT, na + nb - diag);
+            // X ascending at [0, nx); Y descending at [nx, nx + ny)
+            up = first;
+            base_out = first ? diag : nx + ny - 1 - diag;
+        }
+        consumer_sync<NC>();                           // all pieces consumed
+        if (valid == IT) {                             // full window: unconditional stores
+            uint32_t* o = buf + base_out;
+            if (up) {
+#pragma unroll
+                for (int q = 0; q < IT; ++q) o[q] = k[q];
+            } else {
+#pragma unroll
+                for (int q = 0; q < IT; ++q) o[-q] = k[q];
+            }
+        } else {
+#pragma unroll
+            for (int q = 0; q < IT; ++q)
+                if (q < valid) buf[up ? base_out + q : base_out - q] = k[q];
+        }
+        consumer_sync<NC>();
+
+        // stage 2: bitonic merge of X (ascending) and Y (descending)
+        const int total = nx + ny;
+        const int diag = tid * IT;
+        const bool act2 = tid < NT && diag < total;
+        if (act2 && !(DC_M4_SKIP & 2)) {
+            const uint32_t Ab = B0, Bb = B0 + 4u * (total - diag);
+            int lo = max(0, diag - ny), hi = min(diag, nx);
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (!K::lt(lds(Bb + 4u * mid), lds(Ab + 4u * mid))) lo = mid + 1;
+                else hi = mid;
+            }
+            uint32_t ai = Ab + 4u * lo;
+            const uint32_t bi0 = B0 + 4u * (total - 1 - (diag - lo));
+            const uint32_t D = ai - bi0;
+            uint32_t a = lds(ai), bv = lds(bi0);
+#pragma unroll
+            for (int q = 0; q < IT; ++q) {
+                const bool p = K::lt(bv, a);
+                k[q] = p ? bv : a;
+                if (!p) ai += 4u;
+                const uint32_t bi = ai - D - 4u * (q + 1);
+                const uint32_t v = lds(p ? bi : ai);
+                if (p) bv = v; else a = v;
+            }
+        }
+        consumer_sync<NC>();
+        // output back into the buffer (the producer bulk-stores the 16-byte
+        // body); the < 4-word tail of a short tile straight from registers
+        // (tile outputs start at multiples of 4 words: T and 4w are)
+        const int body = total & ~3;
+        if (act2) {
+            if (diag + IT <= body) {
+#pragma unroll
+                for (int q = 0; q < IT; ++q) buf[diag + q] = k[q];
+            } else {
+#pragma unroll
+                for (int q = 0; q < IT; ++q) {
+                    if (diag + q < body) buf[diag + q] = k[q];
+                    else if (diag + q < total) dst[m.out + diag + q] = k[q];
+                }
+            }
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(smem_addr(&empty[b]));
+    }
+}
+
+}  // namespace dc

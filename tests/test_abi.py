@@ -108,14 +108,14 @@ def test_schedule(n, kt, vals):
     t = s["tile"]
     assert s["fused_levels"] == math.ceil(math.log2(t))
     assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))
-    # one level per HBM pass by default; keys-only sorts can fold two (f1)
+    # large keys-only u32/i32 sorts fold two levels per HBM pass by default (f1);
+    # stable sorts (values, f32) and small n (small tiles) run one level per pass
     P = s["global_passes"]
-    assert s["hbm_passes"] == P
+    folds = not (vals or kt == "f32" or P < 2 or n < (1 << 23))
+    assert s["hbm_passes"] == (P % 2 + P // 2 if folds else P)
     p2 = dc.Plan(n)
-    p2.set_two_level(True)
-    s2 = p2.schedule(kt, vals)
-    folds = not (vals or kt == "f32" or P < 2 or n < (1 << 23))   # small n: small tiles, one level
-    assert s2["hbm_passes"] == (P % 2 + P // 2 if folds else P)
+    p2.set_two_level(False)
+    assert p2.schedule(kt, vals)["hbm_passes"] == P
     # fused + global levels cover the whole tree: ceil(log2 n) combine levels
     if n > 1:
         assert s["fused_levels"] + s["global_passes"] >= math.ceil(math.log2(n))

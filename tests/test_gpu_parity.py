@@ -98,6 +98,30 @@ def test_sort_two_level_vs_one_level(dc, oracle_mod, n, dist, key_type):
         assert np.array_equal(_np_keys(k, key_type).view(np.uint32), expect), two
 
 
+# one group of four runs, several groups with a partial last group, ragged tails
+TWO_LEVEL_EDGE = [(1 << 23) + 1, 4 * 26112 * 128 + 26112 * 5 + 3, (1 << 25) - 5]
+
+
+@pytest.mark.parametrize("n", TWO_LEVEL_EDGE)
+@pytest.mark.parametrize("dist", ["sorted", "equal", "paper", "maxkeys", "blocks"])
+def test_sort_two_level_edge_distributions(dc, oracle_mod, n, dist):
+    """4-way passes: the exact 4-run selection on ties, presorted runs and pad-valued keys."""
+    if dist == "maxkeys":      # real keys equal to the +inf pad of the pad-safe merges
+        keys = dcgen.sort_keys(n, "few", seed=21, device="cuda")
+        keys[keys.remainder(3) == 0] = -1
+    elif dist == "blocks":     # runs whose key ranges are disjoint / nested
+        keys = dcgen.sort_keys(n, "uniform", seed=22, device="cuda").remainder(1 << 12)
+        keys += (torch.arange(n, device="cuda") // 26112 % 4) * (1 << 12)
+        keys = keys.to(torch.int32)
+    else:
+        keys = dcgen.sort_keys(n, dist, seed=23, device="cuda")
+    expect = oracle_mod.mergesort(_np_keys(keys, "u32"), key_type="u32")
+    plan = dc.Plan(n)
+    plan.set_two_level(True)
+    plan.sort_(keys, key_type="u32")
+    assert np.array_equal(_np_keys(keys, "u32"), expect)
+
+
 def test_sort_max_key_values_and_pads(dc, oracle_mod):
     # real keys equal to the pad value (0xFFFFFFFF) in a ragged last tile
     n = 3 * TILE + 100
@@ -360,5 +384,5 @@ def test_launch_counts(dc):
     p.sort_(keys, key_type="u32")
     s = p.schedule("u32", False)
     P, H = s["global_passes"], s["hbm_passes"]
-    single = P - 2 * (P - H)          # one-level passes: 2 launches; two-level: 3 launches
-    assert p.launch_count() == 1 + 2 * single + 3 * (H - single)
+    single = P - 2 * (P - H)          # one-level and two-level passes: 2 launches each
+    assert p.launch_count() == 1 + 2 * single + 2 * (H - single)
