@@ -109,7 +109,6 @@ size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 int nk1_smem_bytes(SortCfg c, bool vals) {
     return (vals ? 3 : 1) * dc::tile_words(c.tile(), 0) * 4;
 }
-int nk3_2l_smem_bytes();
 int nk3_smem_bytes(SortCfg c, bool vals) {
     return (vals ? 2 : 1) * dc::tile_words(c.tout(), c.it + 16) * 4;
 }
@@ -129,26 +128,38 @@ int global_passes(int64_t n, int64_t tile) {
 
 size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kMinTout) + 1; }
 
-// Two-level passes (keys-only): 4-way output tiles of kTwoT keys, one cut
-// vector (4 ints) per tile; every group of 4 runs is cut into ceil(4w/kTwoT)
-// tiles (at most one more per group than n / kTwoT in total).
+// Two-level passes: 4-way output tiles of NT*IT keys, one cut vector (4 ints)
+// per tile; every group of 4 runs is cut into ceil(min(4w, n)/T) tiles.  Keys
+// only: 768 x 33 (T = 25344; one CTA per SM, 2 x 102 KB of buffers); with
+// values the key and value regions share the same budget: 512 x 25.
 #ifndef DC_TWO_NT
 #define DC_TWO_NT 768
 #endif
 #ifndef DC_TWO_IT
 #define DC_TWO_IT 33
 #endif
-constexpr int kTwoNT = DC_TWO_NT;
-constexpr int kTwoIT = DC_TWO_IT;
-constexpr int kTwoT = kTwoNT * kTwoIT;
-int nk3_2l_smem_bytes() { return dc::m4_smem_bytes(kTwoT, kTwoIT); }
+#ifndef DC_TWO_NT_KV
+#define DC_TWO_NT_KV 512
+#endif
+#ifndef DC_TWO_IT_KV
+#define DC_TWO_IT_KV 25
+#endif
+struct TwoCfg {
+    int nt, it;
+    constexpr int T() const { return nt * it; }
+};
+constexpr TwoCfg kTwoKeys{DC_TWO_NT, DC_TWO_IT};
+constexpr TwoCfg kTwoKV{DC_TWO_NT_KV, DC_TWO_IT_KV};
+constexpr int kTwoMinT = cmin(kTwoKeys.T(), kTwoKV.T());
+template <bool V>
+constexpr TwoCfg two_cfg() { return V ? kTwoKV : kTwoKeys; }
 
 size_t two_level_tab_entries(int64_t) { return 0; }
 size_t two_level_bnd_entries(int64_t n) {
     // groups at the smallest width (w = tile) have the most tiles
-    const int64_t w = kCfgFast.tile();
+    const int64_t w = std::min(kCfgFast.tile(), kCfgStable.tile());
     const int64_t groups = (n + 4 * w - 1) / (4 * w);
-    return 4 * ((size_t)(groups * num_tiles(4 * w, kTwoT)) + 2);
+    return 4 * ((size_t)(groups * num_tiles(4 * w, kTwoMinT)) + 2);
 }
 
 size_t scratch_needed(int64_t n, bool vals) {
@@ -282,7 +293,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     // two levels into one pass (4-way groups, sort4_kernels.cuh); with P odd
     // one single-level pass goes first.
     const int P = global_passes(n, C.tile());
-    constexpr bool kTwoCapable = !V && !K::kNeedStable && !SMALL;
+    constexpr bool kTwoCapable = !SMALL;
     const bool two = kTwoCapable && p->two_level && P >= 2;
     const int single = two ? (P % 2) : P;
     const int passes = two ? single + (P - single) / 2 : P;
@@ -387,34 +398,36 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         if (two) {
             int* tab = split + align_up(split_entries(n) * 4, 256) / 4;
             dc::Cut4* cuts = (dc::Cut4*)(tab + align_up(two_level_tab_entries(n) * 4, 256) / 4);
-            auto* k32 = dc::nk3_merge4<kTwoNT, kTwoIT, K>;
-            const int smem2 = nk3_2l_smem_bytes();
-            static int grid2 = 0;
+            constexpr TwoCfg TC = two_cfg<V>();
+            auto* k32 = dc::nk3_merge4<TC.nt, TC.it, K, V>;
+            constexpr int smem2 = dc::m4_smem_bytes(TC.T(), TC.it, V);
+            static int grid2 = 0;                        // per instantiation
             if (!grid2) {
                 DC_CUDA(p, cudaFuncSetAttribute(k32, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                 smem2));
                 int dev = 0, sms = 148, occ = 1;
                 cudaGetDevice(&dev);
                 cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, kTwoNT + 64, smem2);
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, TC.nt + 64, smem2);
                 grid2 = sms * (occ > 0 ? occ : 1);
             }
             for (; w < n; w *= 4) {
-                const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), kTwoT);
+                const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), TC.T());
                 const int tiles2 = (int)(((n + 4 * w - 1) / (4 * w)) * tpg);
                 {
                     TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
                     dc::nk2_select4<K><<<(tiles2 + 3) / 4, 128, 0, p->stream>>>(
-                        cur_k, n, w, kTwoT, tpg, tiles2, cuts);
+                        cur_k, n, w, TC.T(), tpg, tiles2, cuts);
                     DC_LAUNCHED(p);
                 }
                 {
                     TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                    k32<<<std::min(tiles2, grid2), kTwoNT + 64, smem2, p->stream>>>(
-                        cur_k, oth_k, n, w, tpg, cuts, tiles2);
+                    k32<<<std::min(tiles2, grid2), TC.nt + 64, smem2, p->stream>>>(
+                        cur_k, cur_v, oth_k, oth_v, n, w, tpg, cuts, tiles2);
                     DC_LAUNCHED(p);
                 }
                 std::swap(cur_k, oth_k);
+                std::swap(cur_v, oth_v);
             }
         }
     }
@@ -825,7 +838,7 @@ dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32
     if (fused_levels) *fused_levels = f;
     const int P = global_passes(p->n, c.tile());
     if (passes) *passes = P;
-    const bool two = p->two_level && !with_vals && kt != DC_KEY_F32 && P >= 2 && p->n >= kSmallN;
+    const bool two = p->two_level && P >= 2 && p->n >= kSmallN;
     if (hbm_passes) *hbm_passes = two ? (P % 2) + (P - P % 2) / 2 : P;
     return DC_OK;
 }

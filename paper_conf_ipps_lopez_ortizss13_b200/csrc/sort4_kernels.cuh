@@ -235,24 +235,28 @@ __device__ __forceinline__ void merge_pad(uint32_t ai, uint32_t bi, uint32_t (&o
     }
 }
 
-// Per-buffer tile descriptor, written by the issuing thread.
+// Per-buffer tile descriptor, written by the producer.
 struct Tile4 {
     long long g0[4];  // global start of each piece
     int len[4];
-    int at[4];        // word offset of each piece's first element in the buffer
+    int at[4];        // word offset of each piece's first element in the region
     long long out;    // global output offset of the tile
     int total;
     int pad_;
 };
 
-// Shared words per buffer: the four pieces with their alignment heads and IT
-// pads each, rounded; a guard of IT + 4 words sits below every buffer (the
-// bitonic stage-2 merge of a short tile may read just below it).
+// Shared words of one key (or value) region of a buffer: a guard of IT + 4
+// words (the bitonic stage-2 merge of a short tile may read just below the
+// region), then the four pieces with their alignment heads and IT pads each.
+// A buffer is one key region (keys only) or a key region followed by a value
+// region with the same layout; there are two buffers.
 __host__ __device__ constexpr int m4_guard(int IT) { return (IT + 4 + 3) / 4 * 4; }
-__host__ __device__ constexpr int m4_buf_words(int T, int IT) {
+__host__ __device__ constexpr int m4_region_words(int T, int IT) {
     return m4_guard(IT) + (T + 4 * (IT + 8) + 16 + 3) / 4 * 4;
 }
-__host__ __device__ constexpr int m4_smem_bytes(int T, int IT) { return 2 * m4_buf_words(T, IT) * 4; }
+__host__ __device__ constexpr int m4_smem_bytes(int T, int IT, bool vals) {
+    return 2 * (vals ? 2 : 1) * m4_region_words(T, IT) * 4;
+}
 
 __device__ __forceinline__ void mbar_arrive(uint32_t bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
@@ -274,18 +278,28 @@ __device__ __forceinline__ void consumer_sync() {
 // empty[b]: output written (one arrive per consumer warp).  Tiles
 // J = blockIdx.x + i * gridDim.x; empty tiles (end of the last group) pass
 // through with no work.
-#ifndef DC_M4_MINB   // CTAs per SM the register budget is sized for (1: 768 x 33 tiles)
+//
+// Keys-only u32/i32 (equal keys indistinguishable): pad-safe merges and a
+// bitonic stage 2 (Y stored descending), no bounds checks.  Stable variants
+// (values, or f32 keys whose +0/-0 must keep their order): bounds-checked
+// stable merges (earlier run wins ties: R0 < R1 within X, R2 < R3 within Y,
+// X < Y), values gathered through the source address of every key.
+#ifndef DC_M4_MINB   // CTAs per SM the register budget is sized for
 #define DC_M4_MINB 1
 #endif
-template <int NT, int IT, class K>
+template <int NT, int IT, class K, bool V>
 __global__ void __launch_bounds__(NT + 64, DC_M4_MINB)
-nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long long n, long long w,
+nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
+           uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v, long long n, long long w,
            int tpg, const Cut4* __restrict__ cut, int num_tiles) {
     static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
+    constexpr bool kStable = V || K::kNeedStable;
     constexpr int T = NT * IT;
     constexpr int NC = NT + 32;                        // consumer threads
-    constexpr int BW = m4_buf_words(T, IT);
+    constexpr int KW = m4_region_words(T, IT);
+    constexpr int BW = (V ? 2 : 1) * KW;               // words per buffer
     constexpr int GU = m4_guard(IT);
+    constexpr uint32_t VOFF = 4u * KW;                 // key -> value byte offset
     extern __shared__ __align__(16) uint32_t sm[];
     __shared__ __align__(8) uint64_t full[2], empty[2];
     __shared__ Tile4 meta[2];
@@ -348,11 +362,14 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
                 if (al1 > n4) al1 = n4;
                 if (al1 < al0) al1 = al0;
                 tend[r] = al1;
-                if (al1 > al0) bytes += (uint32_t)(4 * (al1 - al0));
+                if (al1 > al0) bytes += (uint32_t)(4 * (al1 - al0)) * (V ? 2 : 1);
                 o = (m.at[r] + m.len[r] + IT + 1 + 3) & ~3;
                 const int e0 = (int)(max(al1, m.g0[r]) - m.g0[r]);
-                for (int e = e0 + lane; e < m.len[r] + IT; e += 32)
-                    buf[m.at[r] + e] = e < m.len[r] ? src[m.g0[r] + e] : K::kPad;
+                for (int e = e0 + lane; e < m.len[r] + IT; e += 32) {
+                    const bool real = e < m.len[r];
+                    buf[m.at[r] + e] = real ? src_k[m.g0[r] + e] : K::kPad;
+                    if (V) buf[KW + m.at[r] + e] = real ? src_v[m.g0[r] + e] : 0u;
+                }
             }
             __syncwarp();
             if (lane == 0) {
@@ -362,9 +379,12 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
 #pragma unroll
                 for (int r = 0; r < 4; ++r) {
                     const long long al0 = m.g0[r] & ~3LL;
-                    if (tend[r] > al0)
-                        bulk_g2s(base + 4u * (m.at[r] - (int)(m.g0[r] & 3)), src + al0,
-                                 (uint32_t)(4 * (tend[r] - al0)), fb);
+                    if (tend[r] > al0) {
+                        const uint32_t d = base + 4u * (m.at[r] - (int)(m.g0[r] & 3));
+                        const uint32_t nb = (uint32_t)(4 * (tend[r] - al0));
+                        bulk_g2s(d, src_k + al0, nb, fb);
+                        if (V) bulk_g2s(d + VOFF, src_v + al0, nb, fb);
+                    }
                 }
             }
         };
@@ -377,7 +397,9 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
                 const Tile4 m = meta[b];
                 const int body = m.total & ~3;
                 if (body > 0) {
-                    bulk_s2g(dst + m.out, SM0 + 4u * (b * BW + GU), 4u * body);
+                    const uint32_t sb = SM0 + 4u * (b * BW + GU);
+                    bulk_s2g(dst_k + m.out, sb, 4u * body);
+                    if (V) bulk_s2g(dst_v + m.out, sb + VOFF, 4u * body);
                     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
                 }
                 if (i + 2 < my_tiles) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
@@ -402,8 +424,9 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
 
         // stage 1: X = merge(P0, P1), Y = merge(P2, P3), IT-output windows
         const int nx = m.len[0] + m.len[1], ny = m.len[2] + m.len[3];
+        const int total = nx + ny;
         const int wx = (nx + IT - 1) / IT, wy = (ny + IT - 1) / IT;
-        uint32_t k[IT];
+        uint32_t k[IT], src[IT], vv[IT];
         int valid = 0, base_out = 0;
         bool up = true;
         if (!(DC_M4_SKIP & 1) && tid < wx + wy) {
@@ -413,18 +436,32 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
             const uint32_t Bq = B0 + 4u * (first ? m.at[1] : m.at[3]);
             const int diag = (first ? tid : tid - wx) * IT;
             const int ci = corank_smem<K>(A, na, Bq, nb, diag);
-            merge_pad<K, IT>(A + 4u * ci, Bq + 4u * (diag - ci), k);
+            if constexpr (kStable) {
+                serial_merge<K, IT, V>(A + 4u * ci, A + 4u * na, Bq + 4u * (diag - ci),
+                                       Bq + 4u * nb, k, src);
+                if (V) {
+#pragma unroll
+                    for (int q = 0; q < IT; ++q) vv[q] = lds(src[q] + VOFF);
+                }
+                // X at [0, nx), Y at [nx, nx + ny), both ascending
+                base_out = first ? diag : nx + diag;
+            } else {
+                merge_pad<K, IT>(A + 4u * ci, Bq + 4u * (diag - ci), k);
+                // X ascending at [0, nx); Y descending at [nx, nx + ny)
+                up = first;
+                base_out = first ? diag : nx + ny - 1 - diag;
+            }
             valid = min(IT, na + nb - diag);
-            // X ascending at [0, nx); Y descending at [nx, nx + ny)
-            up = first;
-            base_out = first ? diag : nx + ny - 1 - diag;
         }
         consumer_sync<NC>();                           // all pieces consumed
         if (valid == IT) {                             // full window: unconditional stores
             uint32_t* o = buf + base_out;
             if (up) {
 #pragma unroll
-                for (int q = 0; q < IT; ++q) o[q] = k[q];
+                for (int q = 0; q < IT; ++q) {
+                    o[q] = k[q];
+                    if (V) o[KW + q] = vv[q];
+                }
             } else {
 #pragma unroll
                 for (int q = 0; q < IT; ++q) o[-q] = k[q];
@@ -432,34 +469,48 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
         } else {
 #pragma unroll
             for (int q = 0; q < IT; ++q)
-                if (q < valid) buf[up ? base_out + q : base_out - q] = k[q];
+                if (q < valid) {
+                    const int at = up ? base_out + q : base_out - q;
+                    buf[at] = k[q];
+                    if (V) buf[KW + at] = vv[q];
+                }
         }
         consumer_sync<NC>();
 
-        // stage 2: bitonic merge of X (ascending) and Y (descending)
-        const int total = nx + ny;
         const int diag = tid * IT;
         const bool act2 = tid < NT && diag < total;
         if (act2 && !(DC_M4_SKIP & 2)) {
-            const uint32_t Ab = B0, Bb = B0 + 4u * (total - diag);
-            int lo = max(0, diag - ny), hi = min(diag, nx);
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (!K::lt(lds(Bb + 4u * mid), lds(Ab + 4u * mid))) lo = mid + 1;
-                else hi = mid;
-            }
-            uint32_t ai = Ab + 4u * lo;
-            const uint32_t bi0 = B0 + 4u * (total - 1 - (diag - lo));
-            const uint32_t D = ai - bi0;
-            uint32_t a = lds(ai), bv = lds(bi0);
+            if constexpr (kStable) {
+                // stage 2: stable merge of X and Y (X wins ties)
+                const int c = corank_smem<K>(B0, nx, B0 + 4u * nx, ny, diag);
+                serial_merge<K, IT, V>(B0 + 4u * c, B0 + 4u * nx, B0 + 4u * (nx + diag - c),
+                                       B0 + 4u * total, k, src);
+                if (V) {
 #pragma unroll
-            for (int q = 0; q < IT; ++q) {
-                const bool p = K::lt(bv, a);
-                k[q] = p ? bv : a;
-                if (!p) ai += 4u;
-                const uint32_t bi = ai - D - 4u * (q + 1);
-                const uint32_t v = lds(p ? bi : ai);
-                if (p) bv = v; else a = v;
+                    for (int q = 0; q < IT; ++q) vv[q] = lds(src[q] + VOFF);
+                }
+            } else {
+                // stage 2: bitonic merge of X (ascending) and Y (descending)
+                const uint32_t Ab = B0, Bb = B0 + 4u * (total - diag);
+                int lo = max(0, diag - ny), hi = min(diag, nx);
+                while (lo < hi) {
+                    const int mid = (lo + hi) >> 1;
+                    if (!K::lt(lds(Bb + 4u * mid), lds(Ab + 4u * mid))) lo = mid + 1;
+                    else hi = mid;
+                }
+                uint32_t ai = Ab + 4u * lo;
+                const uint32_t bi0 = B0 + 4u * (total - 1 - (diag - lo));
+                const uint32_t D = ai - bi0;
+                uint32_t a = lds(ai), bv = lds(bi0);
+#pragma unroll
+                for (int q = 0; q < IT; ++q) {
+                    const bool p = K::lt(bv, a);
+                    k[q] = p ? bv : a;
+                    if (!p) ai += 4u;
+                    const uint32_t bi = ai - D - 4u * (q + 1);
+                    const uint32_t v = lds(p ? bi : ai);
+                    if (p) bv = v; else a = v;
+                }
             }
         }
         consumer_sync<NC>();
@@ -470,12 +521,20 @@ nk3_merge4(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, long lo
         if (act2) {
             if (diag + IT <= body) {
 #pragma unroll
-                for (int q = 0; q < IT; ++q) buf[diag + q] = k[q];
+                for (int q = 0; q < IT; ++q) {
+                    buf[diag + q] = k[q];
+                    if (V) buf[KW + diag + q] = vv[q];
+                }
             } else {
 #pragma unroll
                 for (int q = 0; q < IT; ++q) {
-                    if (diag + q < body) buf[diag + q] = k[q];
-                    else if (diag + q < total) dst[m.out + diag + q] = k[q];
+                    if (diag + q < body) {
+                        buf[diag + q] = k[q];
+                        if (V) buf[KW + diag + q] = vv[q];
+                    } else if (diag + q < total) {
+                        dst_k[m.out + diag + q] = k[q];
+                        if (V) dst_v[m.out + diag + q] = vv[q];
+                    }
                 }
             }
         }

@@ -122,6 +122,26 @@ def test_sort_two_level_edge_distributions(dc, oracle_mod, n, dist):
     assert np.array_equal(_np_keys(keys, "u32"), expect)
 
 
+STABLE_TWO_LEVEL = [(1 << 23) + 7, 5 * 16896 * 128 + 16896 * 3 + 11]
+
+
+@pytest.mark.parametrize("n", STABLE_TWO_LEVEL)
+@pytest.mark.parametrize("dist", ["uniform", "few", "equal"])
+@pytest.mark.parametrize("key_type,with_vals", [("u32", True), ("i32", True), ("f32", True),
+                                                ("f32", False)])
+def test_sort_two_level_stable(dc, oracle_mod, n, dist, key_type, with_vals):
+    """Stable 4-way passes (values, or f32 keys with +0/-0): ties keep run order."""
+    k_in, k_out, v_out = run_sort(dc, n, dist, key_type, with_vals, seed=29)
+    plan_sched = dc.Plan(n).schedule(key_type, with_vals)
+    assert plan_sched["hbm_passes"] < plan_sched["global_passes"]      # 4-way passes ran
+    vals_in = np.arange(n, dtype=np.uint32) if with_vals else None
+    res = oracle_mod.mergesort(_np_keys(k_in, key_type), vals_in, key_type=key_type)
+    ek = res[0] if with_vals else res
+    assert np.array_equal(_np_keys(k_out, key_type).view(np.uint32), ek.view(np.uint32))
+    if with_vals:
+        assert np.array_equal(v_out.cpu().numpy().view(np.uint32), res[1])
+
+
 def test_sort_max_key_values_and_pads(dc, oracle_mod):
     # real keys equal to the pad value (0xFFFFFFFF) in a ragged last tile
     n = 3 * TILE + 100

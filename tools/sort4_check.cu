@@ -29,10 +29,10 @@
     } while (0)
 
 #ifndef NT_
-#define NT_ 512
+#define NT_ 768
 #endif
 #ifndef IT_
-#define IT_ 25
+#define IT_ 33
 #endif
 constexpr int NT = NT_, IT = IT_, T = NT * IT;
 
@@ -95,15 +95,15 @@ int main(int argc, char** argv) {
                 printf("cut mismatch tile %d run %d: gpu %d host %d\n", j, q, gc[j].c[q], hc[j].c[q]);
     printf("select4: %d mismatches over %d tiles\n", bad, tiles);
     CK(cudaMemcpy(dcut, hc.data(), tiles * sizeof(dc::Cut4), cudaMemcpyHostToDevice));
-    auto* k = dc::nk3_merge4<NT, IT, dc::KeyU32>;
-    const int smem = dc::m4_smem_bytes(T, IT);
+    auto* k = dc::nk3_merge4<NT, IT, dc::KeyU32, false>;
+    const int smem = dc::m4_smem_bytes(T, IT, false);
     CK(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     int occ = 0, sms = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, NT + 64, smem));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
     const int grid = std::min(tiles, sms * occ);
     printf("merge4: smem %d B, occupancy %d CTAs/SM, grid %d\n", smem, occ, grid);
-    k<<<grid, NT + 64, smem>>>(dsrc, ddst, n, w, tpg, dcut, tiles);
+    k<<<grid, NT + 64, smem>>>(dsrc, nullptr, ddst, nullptr, n, w, tpg, dcut, tiles);
     CK(cudaGetLastError());
     CK(cudaDeviceSynchronize());
     std::vector<uint32_t> out(n), ref(h);
@@ -126,7 +126,7 @@ int main(int argc, char** argv) {
             cudaEventElapsedTime(&t, e0, e1);
             if (i) ms_s += t;
             cudaEventRecord(e0);
-            k<<<grid, NT + 64, smem>>>(dsrc, ddst, n, w, tpg, dcut, tiles);
+            k<<<grid, NT + 64, smem>>>(dsrc, nullptr, ddst, nullptr, n, w, tpg, dcut, tiles);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
             cudaEventElapsedTime(&t, e0, e1);
