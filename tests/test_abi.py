@@ -108,10 +108,10 @@ def test_schedule(n, kt, vals):
     t = s["tile"]
     assert s["fused_levels"] == math.ceil(math.log2(t))
     assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))
-    # large keys-only u32/i32 sorts fold two levels per HBM pass by default (f1);
-    # stable sorts (values, f32) and small n (small tiles) run one level per pass
+    # large sorts (n >= 2^23) fold two levels per HBM pass by default (f1);
+    # small n (small tiles) runs one level per pass
     P = s["global_passes"]
-    folds = not (vals or kt == "f32" or P < 2 or n < (1 << 23))
+    folds = not (P < 2 or n < (1 << 23))
     assert s["hbm_passes"] == (P % 2 + P // 2 if folds else P)
     p2 = dc.Plan(n)
     p2.set_two_level(False)
