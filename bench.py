@@ -341,7 +341,7 @@ def run_dc(args, wl):
         "levels_per_launch": 2 if two else 1,
         "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
         "frac": achieved / peak if achieved else None,
-        "traffic": ncu_traffic("nk3_merge", wl),
+        "traffic": ncu_traffic("nk3_merge4" if two else "nk3_merge", wl),
         "algorithmic_bytes_per_launch": bytes_per_key * n,
         "avg_launch_ms": nk3_avg, "peak_source": peak_src,
         "share_of_step": nk3_ms / args.steps / ms_instr if ms_instr else None,
@@ -352,9 +352,11 @@ def run_dc(args, wl):
         "nk1_blocksort": {"avg_ms": nk1_avg, "launches_per_step": nk1_n / args.steps,
                           "hbm_gbs": bytes_per_key * n / (nk1_avg / 1e3) / 1e9 if nk1_n else None,
                           "share_of_step": nk1_ms / args.steps / ms_instr},
-        "nk2_partition": {"avg_ms": nk2_ms / max(nk2_n, 1), "launches_per_step": nk2_n / args.steps,
+        "nk2_partition": {"kernel": "nk2_select4" if two else "nk2_partition",
+                          "avg_ms": nk2_ms / max(nk2_n, 1), "launches_per_step": nk2_n / args.steps,
                           "share_of_step": nk2_ms / args.steps / ms_instr},
-        "nk3_merge": {"avg_ms": nk3_avg, "launches_per_step": nk3_n / args.steps,
+        "nk3_merge": {"kernel": "nk3_merge4" if two else "nk3_merge",
+                      "avg_ms": nk3_avg, "launches_per_step": nk3_n / args.steps,
                       "hbm_gbs": achieved, "share_of_step": nk3_ms / args.steps / ms_instr},
     }
 

@@ -391,8 +391,8 @@ dc_status dc_mg_merge_peers(dc_plan_t plan, dc_key_type key_type,
 
 /* Kernel classes for dc_plan_kernel_time. */
 #define DC_KERNEL_NK1_BLOCKSORT 0 /* fused bottom levels              */
-#define DC_KERNEL_NK2_PARTITION 1 /* merge-path co-ranks of one level */
-#define DC_KERNEL_NK3_MERGE 2     /* one global merge level           */
+#define DC_KERNEL_NK2_PARTITION 1 /* co-ranks of one pass (2- or 4-run) */
+#define DC_KERNEL_NK3_MERGE 2     /* one HBM merge pass (1 or 2 levels) */
 #define DC_KERNEL_NK4_MAXSUB 3    /* max-subarray tiles + top combine */
 #define DC_KERNEL_COUNT 4
 

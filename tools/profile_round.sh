@@ -9,13 +9,13 @@ done
 timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk3_merge -s 20 -c 1 \
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk3_merge4 -s 20 -c 1 \
   -o gpurun_out/prof_nk3 python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk1_blocksort -s 1 -c 1 \
   -o gpurun_out/prof_nk1 python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > /dev/null 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk2_partition -s 20 -c 1 \
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk2_select4 -s 20 -c 1 \
   -o gpurun_out/prof_nk2 python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > /dev/null 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk3_merge -s 20 -c 1 \
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk3_merge4 -s 20 -c 1 \
   -o gpurun_out/prof_nk3_kv python bench.py --workload sort_kv --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:nk4_maxsub -s 3 -c 1 \
   -o gpurun_out/prof_nk4 python bench.py --workload maxsub --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1

@@ -13,3 +13,15 @@ for tool in memcheck racecheck synccheck initcheck; do
     > gpurun_out/sanitize_$tool.txt 2>&1
   echo "$tool rc=$? $(grep -E 'SUMMARY|sanitize_run ok' gpurun_out/sanitize_$tool.txt | tr '\n' ' ')"
 done
+# The two-level pass kernels (nk2_select4, nk3_merge4: mbarriers, named barriers, TMA) run only
+# for n >= 2^23 inside the library; check them in isolation at small sizes (many tiles per CTA).
+nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -lineinfo \
+  -I paper_conf_ipps_lopez_ortizss13_b200/csrc tools/sort4_check.cu -o /tmp/sort4_check
+for tool in memcheck racecheck synccheck; do
+  out=gpurun_out/sanitize_sort4_$tool.txt
+  : > $out
+  for a in "200000 26112 0 0 2" "1000003 26112 1 0 3" "500001 26112 2" "400000 104448 3 0 1"; do
+    timeout 900 compute-sanitizer --tool $tool --print-limit 20 /tmp/sort4_check $a >> $out 2>&1
+  done
+  echo "sort4 $tool: $(grep -cE 'mismatches' $out) checks, $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY' $out | tr '\n' ' ')"
+done

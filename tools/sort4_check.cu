@@ -2,7 +2,7 @@
 // (nk2_select4, nk3_merge4) against a host reference, one stage at a time.
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17
 //        -I paper_conf_ipps_lopez_ortizss13_b200/csrc tools/sort4_check.cu -o /tmp/sort4_check
-// Usage: sort4_check <n> <w> <dist 0..3> [iters]
+// Usage: sort4_check <n> <w> <dist 0..3> [iters] [max_grid]
 #include <cuda_runtime.h>
 #include <cstdio>
 #ifndef DC_SEL4_MAXROUNDS
@@ -42,6 +42,7 @@ int main(int argc, char** argv) {
     long long w = argc > 2 ? atoll(argv[2]) : 26112;
     int dist = argc > 3 ? atoi(argv[3]) : 0;
     int iters = argc > 4 ? atoi(argv[4]) : 0;
+    const int max_grid = argc > 5 ? atoi(argv[5]) : 0;   // >0: few CTAs, many tiles each
     std::mt19937_64 rng(7);
     std::vector<uint32_t> h(n);
     for (long long i = 0; i < n; ++i) {
@@ -101,7 +102,8 @@ int main(int argc, char** argv) {
     int occ = 0, sms = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, NT + 64, smem));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
-    const int grid = std::min(tiles, sms * occ);
+    int grid = std::min(tiles, sms * occ);
+    if (max_grid > 0) grid = std::min(grid, max_grid);
     printf("merge4: smem %d B, occupancy %d CTAs/SM, grid %d\n", smem, occ, grid);
     k<<<grid, NT + 64, smem>>>(dsrc, nullptr, ddst, nullptr, n, w, tpg, dcut, tiles);
     CK(cudaGetLastError());

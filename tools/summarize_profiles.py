@@ -56,8 +56,8 @@ if os.path.exists(lpath):
 
 # ---- full captures
 summary = {}
-caps = {"prof_nk1": ("sort_u32", "nk1_blocksort"), "prof_nk2": ("sort_u32", "nk2_partition"),
-        "prof_nk3": ("sort_u32", "nk3_merge"), "prof_nk3_kv": ("sort_kv", "nk3_merge"),
+caps = {"prof_nk1": ("sort_u32", "nk1_blocksort"), "prof_nk2": ("sort_u32", "nk2_select4"),
+        "prof_nk3": ("sort_u32", "nk3_merge4"), "prof_nk3_kv": ("sort_kv", "nk3_merge4"),
         "prof_nk4": ("maxsub", "nk4_maxsub"), "prof_nk1_kv": ("sort_kv", "nk1_blocksort"),
         "prof_sum": ("sum", "breadth_first_reduce")}
 for cap, (wl, kern) in caps.items():
