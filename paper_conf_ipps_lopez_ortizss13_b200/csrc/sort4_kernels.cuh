@@ -151,6 +151,8 @@ __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long 
         const uint32_t v = active ? __ldg(Rq + p) : 0u;
         int SL = p, SU = p;
         bool dt = false, du = false;
+        // (every shuffle below runs unconditionally on the converged warp; the
+        //  own run and closed windows are masked with selects)
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
             // #pivots of run r preceding this lane's pivot (search over lanes 8r..8r+7)
@@ -158,21 +160,19 @@ __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long 
 #pragma unroll
             for (int step = 4; step >= 1; step >>= 1) {
                 const uint32_t V = __shfl_sync(0xffffffffu, v, 8 * r + a + step - 1);
-                if (precedes<K>(V, r, v, q)) a += step;
+                a += precedes<K>(V, r, v, q) ? step : 0;
             }
-            {
-                const uint32_t V = __shfl_sync(0xffffffffu, v, 8 * r + 7);
-                if (a == 7 && precedes<K>(V, r, v, q)) a = 8;
-            }
-            if (r == q) continue;
-            if (lo[r] > 0 && !precedes<K>(elo[r], r, v, q)) dt = true;      // E before a taken edge
-            if (hi[r] < g.l[r] && precedes<K>(ehi[r], r, v, q)) du = true;  // untaken edge before E
+            const uint32_t V7 = __shfl_sync(0xffffffffu, v, 8 * r + 7);
+            a += (a == 7 && precedes<K>(V7, r, v, q)) ? 1 : 0;
+            const bool other = r != q;
+            dt |= other & (lo[r] > 0) & !precedes<K>(elo[r], r, v, q);      // E before a taken edge
+            du |= other & (hi[r] < g.l[r]) & precedes<K>(ehi[r], r, v, q);  // untaken edge before E
             int Lp = lo[r], Up = hi[r];
             if (W[r] > 0) {
                 if (a > 0) Lp = sel4_pivot(lo[r], W[r], st[r], a - 1) + 1;
                 if (a < 8) Up = sel4_pivot(lo[r], W[r], st[r], a);
             }
-            if (exact && !(dt | du) && active) {
+            if (exact && other && !(dt | du) && active) {
                 int x0 = Lp, x1 = Up;                    // first position not preceding E
                 while (x0 < x1) {
                     const int mid = (x0 + x1) >> 1;
@@ -181,8 +181,8 @@ __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long 
                 }
                 Lp = Up = x0;
             }
-            SL += Lp;
-            SU += Up;
+            SL += other ? Lp : 0;
+            SU += other ? Up : 0;
         }
         // The brackets hold only for a pivot between every other run's edges;
         // an edge decision takes precedence (dt and du exclude each other).
@@ -193,15 +193,17 @@ __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long 
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
             const unsigned gt = (mt >> (8 * r)) & 0xffu, gu = (mu >> (8 * r)) & 0xffu;
-            const int lo0 = lo[r];                        // this round's pivot base
-            if (gt) {                                     // largest taken pivot
-                const int tt = 31 - __clz(gt);
-                elo[r] = __shfl_sync(0xffffffffu, v, 8 * r + tt);
+            const int tt = 31 - __clz(gt | 1u);             // largest taken pivot (0 if none)
+            const int tu = __ffs(gu | 0x80u) - 1;           // smallest untaken pivot (7 if none)
+            const uint32_t vt = __shfl_sync(0xffffffffu, v, 8 * r + tt);
+            const uint32_t vu = __shfl_sync(0xffffffffu, v, 8 * r + tu);
+            const int lo0 = lo[r];                          // this round's pivot base
+            if (gt) {
+                elo[r] = vt;
                 lo[r] = sel4_pivot(lo0, W[r], st[r], tt) + 1;
             }
-            if (gu) {                                     // smallest untaken pivot
-                const int tu = __ffs(gu) - 1;
-                ehi[r] = __shfl_sync(0xffffffffu, v, 8 * r + tu);
+            if (gu) {
+                ehi[r] = vu;
                 hi[r] = sel4_pivot(lo0, W[r], st[r], tu);
             }
         }
