@@ -381,7 +381,9 @@ def run_dc(args, wl):
                    "key_type": "u32", "values": kv, "tile": sched["tile"],
                    "fused_levels": sched["fused_levels"], "global_passes": sched["global_passes"],
                    "hbm_passes": sched["hbm_passes"],
-                   "l2": "flushed before every step (512 MiB write); input 1 GiB > L2",
+                   "l2": "flushed before every step (512 MiB write); input "
+                         + (f"{n * (8 if kv else 4) / 2**30:.0f} GiB > L2" if n * 4 > (126 << 20)
+                            else f"{n * (8 if kv else 4) / 2**20:.0f} MiB, L2-resident after the first level"),
                    "step_ms_min": min(step_ms), "step_ms_max": max(step_ms),
                    "instrumented_step_ms": ms_instr,
                    "sorted_check": sorted_ok},
