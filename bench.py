@@ -103,21 +103,26 @@ class ClockSampler:
             nv.nvmlInit()
             h = nv.nvmlDeviceGetHandleByIndex(self.index)
             mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
-            while not self.stop.is_set():
+            while True:
                 sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
                 rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
                 self.samples.append((sm, mx, rs))
-                self.stop.wait(0.01)
+                self.ready.set()
+                if self.stop.wait(0.01):
+                    break
         except Exception as e:  # noqa: BLE001 - reported in the JSON line
             self.err = repr(e)
+        finally:
+            self.ready.set()
 
     def __enter__(self):
         import threading
 
         self.stop = threading.Event()
+        self.ready = threading.Event()   # set after NVML init + the first sample
         self.t = threading.Thread(target=self._run, daemon=True)
         self.t.start()
-        time.sleep(0.05)
+        self.ready.wait(timeout=30)
         return self
 
     def __exit__(self, *a):
