@@ -32,17 +32,23 @@ namespace {
 // Sort configuration per instantiation (tuned on B200 with tools/sweep.sh,
 // see DESIGN.md Sec. 5).  Keys-only u32/i32 (stability unobservable): 512
 // threads x 51 items = tiles of 26112 keys (9 shared-memory merge levels on
-// top of a 51-input register network; 14 global passes at 2^28), merge CTAs
-// of 256 x 51 = 13056 outputs.  Stable variants (values, or f32 keys whose
-// +0/-0 must keep their order) carry a tile-local index: 512 x 33 = 16896-key
-// tiles, merge CTAs of 256 x 33 outputs.
+// top of a 51-input register network; 14 global levels at 2^28), one-level
+// merge CTAs of 256 x 51 = 13056 outputs.  (1024 x 51 tiles save a global
+// level at 2^28 but cost more in NK1 than they save: 6.38 vs 6.19 ms.)
+// Stable variants (values, or f32 keys whose +0/-0 must keep their order)
+// carry a tile-local index: 512 x 33 = 16896-key tiles, merge CTAs of 256 x 33
+// outputs.  Merge tiles need not divide a pair: every pair is cut into
+// ceil(2w / tout) tiles, the last one short.
 struct SortCfg {
-    int nt1, it, nt3;
-    constexpr int tile() const { return nt1 * it; }
+    int nt1, it1, nt3, it;   // NK1 threads x items, one-level merge threads x items
+    constexpr int tile() const { return nt1 * it1; }
     constexpr int tout() const { return nt3 * it; }
 };
 #ifndef DC_FAST_NT1
 #define DC_FAST_NT1 512
+#endif
+#ifndef DC_FAST_IT1
+#define DC_FAST_IT1 51
 #endif
 #ifndef DC_FAST_IT
 #define DC_FAST_IT 51
@@ -59,17 +65,13 @@ struct SortCfg {
 #ifndef DC_STABLE_NT3
 #define DC_STABLE_NT3 256
 #endif
-constexpr SortCfg kCfgFast{DC_FAST_NT1, DC_FAST_IT, DC_FAST_NT3};
-constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3};
+constexpr SortCfg kCfgFast{DC_FAST_NT1, DC_FAST_IT1, DC_FAST_NT3, DC_FAST_IT};
+constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3, DC_STABLE_IT};
 // Small inputs (n < kSmallN, L2-resident): quarter-size tiles so that the
 // fused kernel and every merge level still launch >= ~150 CTAs.
-constexpr SortCfg kCfgFastSmall{128, DC_FAST_IT, 128};
-constexpr SortCfg kCfgStableSmall{128, DC_STABLE_IT, 128};
+constexpr SortCfg kCfgFastSmall{128, DC_FAST_IT, 128, DC_FAST_IT};
+constexpr SortCfg kCfgStableSmall{128, DC_STABLE_IT, 128, DC_STABLE_IT};
 constexpr int64_t kSmallN = 1LL << 23;
-static_assert((2 * kCfgFast.tile()) % kCfgFast.tout() == 0, "merge tiles must not straddle pairs");
-static_assert((2 * kCfgStable.tile()) % kCfgStable.tout() == 0, "merge tiles must not straddle pairs");
-static_assert((2 * kCfgFastSmall.tile()) % kCfgFastSmall.tout() == 0, "tiles straddle pairs");
-static_assert((2 * kCfgStableSmall.tile()) % kCfgStableSmall.tout() == 0, "tiles straddle pairs");
 constexpr int cmin(int a, int b) { return a < b ? a : b; }
 constexpr int kMinTout = cmin(cmin(kCfgFast.tout(), kCfgStable.tout()),
                               cmin(kCfgFastSmall.tout(), kCfgStableSmall.tout()));
@@ -126,7 +128,13 @@ int global_passes(int64_t n, int64_t tile) {
     return p;
 }
 
-size_t split_entries(int64_t n) { return (size_t)num_tiles(n, kMinTout) + 1; }
+// One-level pass: every pair of width 2w is cut into ceil(2w / tout) tiles, so
+// at most one extra (short) tile per pair; pairs <= n / (2 * min tile) + 1.
+constexpr int kMinTile = cmin(cmin(kCfgFast.tile(), kCfgStable.tile()),
+                              cmin(kCfgFastSmall.tile(), kCfgStableSmall.tile()));
+size_t split_entries(int64_t n) {
+    return (size_t)num_tiles(n, kMinTout) + (size_t)num_tiles(n, 2 * (int64_t)kMinTile) + 2;
+}
 
 // Two-level passes: 4-way output tiles of NT*IT keys, one cut vector (4 ints)
 // per tile; every group of 4 runs is cut into ceil(min(4w, n)/T) tiles.  Keys
@@ -278,7 +286,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     int* split = (int*)((char*)p->scratch + kb + (hv ? kb : 0));
 
     constexpr SortCfg C = cfg_for<K, V, SMALL>();
-    auto* k1 = dc::nk1_blocksort<C.nt1, C.it, K, V>;
+    auto* k1 = dc::nk1_blocksort<C.nt1, C.it1, K, V>;
     auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
     static bool attr_done = false;   // per key/value instantiation
     if (!attr_done) {
@@ -306,8 +314,9 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
 
     // One merge level over [org, end) on stream `st` (split region `sp`).
     auto level = [&](int64_t org, int64_t end, int64_t w, int* sp, cudaStream_t st) -> dc_status {
-        const int tiles = (int)num_tiles(end - org, C.tout());
-        const dc::PairGeom g{org, w, w, end};
+        const int tpg = (int)num_tiles(std::min<int64_t>(2 * w, end - org), C.tout());
+        const int tiles = (int)(num_tiles(end - org, 2 * w) * tpg);
+        const dc::PairGeom g{org, w, w, end, tpg};
         {
             TimedScope ts(p, DC_KERNEL_NK2_PARTITION, st);
 #ifndef DC_NK2_WARP_ALL
@@ -347,7 +356,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         st = ensure_pipeline(p, chunks);
         if (st != DC_OK) return st;
         const int64_t clen = (int64_t)C.tile() << lc;
-        const size_t split_per = (size_t)num_tiles(clen, C.tout()) + 1;
+        const size_t split_per = (size_t)num_tiles(clen, C.tout()) + (size_t)num_tiles(clen, 2 * (int64_t)C.tile()) + 2;
         DC_CUDA(p, cudaEventRecord(p->pipe_events[0], p->stream));
         for (int c = 0; c < chunks; ++c) {
             cudaStream_t cs = p->pipe_streams[c];
@@ -626,8 +635,8 @@ dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* 
         for (size_t r = 0; r < runs.size(); r += 2) {
             const int64_t la = runs[r], lb = (r + 1 < runs.size()) ? runs[r + 1] : 0;
             if (la + lb > 0) {
-                const dc::PairGeom g{org, la, lb, org + la + lb};
                 const int tiles = (int)num_tiles(la + lb, C.tout());
+                const dc::PairGeom g{org, la, lb, org + la + lb, tiles};
                 {
                     TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
                     dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(

@@ -447,26 +447,32 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
 // (the buffer base stays 16-byte aligned for TMA).
 struct PairGeom {
     long long org, wa, wb, end;
-    // pair containing merged position d0 (relative to org): absolute start s
-    __device__ __forceinline__ void pair_of(long long d0, long long& s, long long& a_len,
-                                            long long& b_len) const {
-        s = org + (d0 / (wa + wb)) * (wa + wb);
+    int tpg;   // output tiles per pair: ceil((wa + wb) / tout) (the last one short)
+    // Tile j: absolute pair start s, run lengths, tile output range [dd0, dd1)
+    // relative to s (empty when dd0 >= a_len + b_len: trailing tiles of a
+    // short last pair).
+    __device__ __forceinline__ void tile_of(int j, int tout, long long& s, long long& a_len,
+                                            long long& b_len, long long& dd0,
+                                            long long& dd1) const {
+        const int p = j / tpg;
+        s = org + (long long)p * (wa + wb);
         a_len = min(wa, end - s);
         b_len = max(0LL, min(wb, end - s - a_len));
+        dd0 = (long long)(j - p * tpg) * tout;
+        dd1 = min(dd0 + tout, a_len + b_len);
     }
 };
 
-// Co-rank of the first output of every merge tile: tile j covers merged
-// positions [j*tout, (j+1)*tout) (tout divides wa + wb, or there is one pair).
+// Co-rank of the first output of every merge tile (tile j: tile_of).
 template <class K>
 __global__ void nk2_partition(const uint32_t* __restrict__ src, PairGeom g, int tout,
                               int num_tiles, int* __restrict__ split) {
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= num_tiles) return;
-    const long long d0 = (long long)j * tout;
-    long long s, a_len, b_len;
-    g.pair_of(d0, s, a_len, b_len);
-    split[j] = (int)corank_global<K>(src + s, a_len, src + s + a_len, b_len, d0 - (s - g.org));
+    long long s, a_len, b_len, dd0, dd1;
+    g.tile_of(j, tout, s, a_len, b_len, dd0, dd1);
+    if (dd0 >= a_len + b_len) return;                 // empty tile
+    split[j] = (int)corank_global<K>(src + s, a_len, src + s + a_len, b_len, dd0);
 }
 
 // First index in [a, b] where a monotone (true ... false) predicate on [a, b)
@@ -500,10 +506,9 @@ __global__ void nk2_partition_warp(const uint32_t* __restrict__ src, PairGeom g,
                                    int num_tiles, int* __restrict__ split) {
     const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
     if (j >= num_tiles) return;                       // warp-uniform
-    const long long d0 = (long long)j * tout;
-    long long s, a_len, b_len;
-    g.pair_of(d0, s, a_len, b_len);
-    const long long diag = d0 - (s - g.org);
+    long long s, a_len, b_len, diag, dd1;
+    g.tile_of(j, tout, s, a_len, b_len, diag, dd1);
+    if (diag >= a_len + b_len) return;                // empty tile
     const uint32_t* A = src + s;
     const uint32_t* B = src + s + a_len;
     const long long lo = max(0LL, diag - b_len), hi = min(diag, a_len);
@@ -626,17 +631,15 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
     extern __shared__ __align__(16) uint32_t smem[];
     __shared__ __align__(8) uint64_t bar;
     const int j = blockIdx.x;
-    const long long d0 = (long long)j * TOUT;
-    long long s, a_len, b_len;
-    g.pair_of(d0, s, a_len, b_len);
-    const long long dd0 = d0 - (s - g.org);
-    const long long dd1 = min(dd0 + TOUT, a_len + b_len);
+    long long s, a_len, b_len, dd0, dd1;
+    g.tile_of(j, TOUT, s, a_len, b_len, dd0, dd1);
+    if (dd0 >= a_len + b_len) return;                 // empty tile (whole CTA)
     const int i0 = split[j];
     const int i1 = (dd1 == a_len + b_len) ? (int)a_len : split[j + 1];
     const int na = i1 - i0;
     const int nb = (int)(dd1 - dd0) - na;
     merge_tile<NT, IT, K, V>(src_k, src_v, g.end, s + i0, na, src_k, src_v, g.end,
-                             s + a_len + (dd0 - i0), nb, dst_k, dst_v, g.org + d0, smem,
+                             s + a_len + (dd0 - i0), nb, dst_k, dst_v, s + dd0, smem,
                              smem + TW, smem_addr(&bar));
 }
 

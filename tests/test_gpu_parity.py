@@ -14,7 +14,7 @@ import dcgen
 
 pytestmark = pytest.mark.gpu
 
-TILE = 26112  # keys-only fused tile (512 x 51); stable tiles are 16896
+TILE = 26112  # keys-only fused tile (512 x 51) from 2^23 keys; stable tiles are 16896
 
 
 @pytest.fixture(scope="module")
@@ -99,7 +99,7 @@ def test_sort_two_level_vs_one_level(dc, oracle_mod, n, dist, key_type):
 
 
 # one group of four runs, several groups with a partial last group, ragged tails
-TWO_LEVEL_EDGE = [(1 << 23) + 1, 4 * 26112 * 128 + 26112 * 5 + 3, (1 << 25) - 5]
+TWO_LEVEL_EDGE = [(1 << 23) + 1, 4 * TILE * 128 + TILE * 5 + 3, 4 * 52224 * 64 + 52224 * 5 + 3, (1 << 25) - 5]
 
 
 @pytest.mark.parametrize("n", TWO_LEVEL_EDGE)
@@ -111,7 +111,7 @@ def test_sort_two_level_edge_distributions(dc, oracle_mod, n, dist):
         keys[keys.remainder(3) == 0] = -1
     elif dist == "blocks":     # runs whose key ranges are disjoint / nested
         keys = dcgen.sort_keys(n, "uniform", seed=22, device="cuda").remainder(1 << 12)
-        keys += (torch.arange(n, device="cuda") // 26112 % 4) * (1 << 12)
+        keys += (torch.arange(n, device="cuda") // TILE % 4) * (1 << 12)
         keys = keys.to(torch.int32)
     else:
         keys = dcgen.sort_keys(n, dist, seed=23, device="cuda")
@@ -321,13 +321,15 @@ def test_full_size_2pow28_keys(dc, dist):
 
 
 def test_max_size_keys(dc):
-    """n = 2^31 - 1, the largest per-GPU size of the ABI (17 global passes,
-    int32 co-ranks at their limit)."""
+    """n = 2^31 - 1, the largest per-GPU size of the ABI (16-17 global passes
+    depending on the tile, int32 co-ranks at their limit)."""
     n = (1 << 31) - 1
     keys = dcgen.sort_keys(n, "uniform", seed=7, device="cuda")
     k_in = keys.clone()
     plan = dc.Plan(n)
-    assert plan.schedule("u32")["global_passes"] == 17
+    sch = plan.schedule("u32")
+    runs = -(-n // sch["tile"])
+    assert sch["global_passes"] == (runs - 1).bit_length() >= 16
     plan.sort_(keys, key_type="u32")
     torch.cuda.synchronize()
     del plan

@@ -1,0 +1,65 @@
+"""GPU parity of tile-shape variants the default build does not exercise.
+
+The one-level merge pass cuts every pair of runs (width 2w) into
+ceil(2w / tout) output tiles, the last one short (PairGeom.tile_of).  With the
+default shapes tout divides 2w; this builds the library with 160-thread merge
+CTAs (tout = 160 x 51 = 8160, 2 x 26112 / 8160 = 6.4) and checks the one-level
+schedule bit-exactly against the oracle in a subprocess bound to that build.
+"""
+import os
+import subprocess
+import sys
+
+import pytest
+import torch
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+SCRIPT = r"""
+import sys
+import numpy as np
+import torch
+sys.path.insert(0, {root!r})
+import dcgen, oracle
+import paper_conf_ipps_lopez_ortizss13_b200 as dc
+oracle.build()
+sch = dc.Plan(1 << 23).schedule("u32")
+assert sch["tile"] == 26112, sch
+for n, dist, kt, vals in [((1 << 23) + 12345, "uniform", "u32", False),
+                          (2 * 26112 * 5 + 7, "few", "u32", False),
+                          ((1 << 23) + 99, "uniform", "i32", False),
+                          ((1 << 23) + 5, "few", "u32", True)]:
+    keys = dcgen.sort_keys(n, dist, seed=41, key_type=kt, device="cuda")
+    v = dcgen.sort_vals(n, device="cuda") if vals else None
+    ka = keys.cpu().numpy()
+    ka = ka.view(np.uint32) if kt == "u32" else ka.view(np.int32)
+    if vals:
+        ek, ev = oracle.mergesort(ka, v.cpu().numpy().view(np.uint32), key_type=kt)
+    else:
+        ek = oracle.mergesort(ka, key_type=kt)
+    plan = dc.Plan(n)
+    plan.set_two_level(False)
+    plan.sort_(keys, v, key_type=kt)
+    torch.cuda.synchronize()
+    got = keys.cpu().numpy().view(ek.dtype)
+    assert np.array_equal(got, ek), (n, dist, kt)
+    if vals:
+        assert np.array_equal(v.cpu().numpy().view(np.uint32), ev), (n, dist, kt)
+print("variant ok")
+"""
+
+
+def test_one_level_tiles_not_dividing_pairs(tmp_path):
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_lopez_ortizss13_b200 import build
+
+    lib = build.build(out=str(tmp_path / "libdc_nt160.so"),
+                      defines=["DC_FAST_NT3=160", "DC_STABLE_NT3=160"])
+    env = dict(os.environ, DC_LIB=lib)
+    r = subprocess.run([sys.executable, "-c", SCRIPT.format(root=ROOT)], env=env,
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert "variant ok" in r.stdout
