@@ -1354,7 +1354,7 @@ dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys
             DC_CUDA(p, cudaEventRecord(hs.out_done, p->d2h));
         }
     }
-    auto& hs = p->hslot[p->submits & 1];
+    auto& hs = p->hslot[p->submits % dc_plan_s::kHostSlots];
     const size_t kb = align_up((size_t)p->n * 4, 256);
     const size_t need = h_in_vals ? 2 * kb : kb;
     if (hs.bytes < need) {
@@ -1379,7 +1379,7 @@ dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys
     DC_CUDA(p, cudaMemcpyAsync(dk, h_in_keys, bytes, cudaMemcpyHostToDevice, p->h2d));
     if (dv) DC_CUDA(p, cudaMemcpyAsync(dv, h_in_vals, bytes, cudaMemcpyHostToDevice, p->h2d));
     DC_CUDA(p, cudaEventRecord(hs.in_done, p->h2d));
-    // sort on the compute stream (sorts of the two slots serialise: shared scratch)
+    // sort on the compute stream (sorts of the slots serialise: shared scratch)
     DC_CUDA(p, cudaStreamWaitEvent(p->comp, hs.in_done, 0));
     cudaStream_t user = p->stream;
     p->stream = p->comp;

@@ -75,13 +75,15 @@ struct dc_plan_s {
     // host-buffer (end-to-end) staging
     void* d_stage = nullptr;
     size_t d_stage_bytes = 0;
-    // streaming host sorts: two device slots, copy-in / compute / copy-out streams
+    // streaming host sorts: three device slots (copy-in of step i+2 overlaps the
+    // copy-out of step i and the sort of step i+1), copy-in / compute / copy-out streams
     struct HostSlot {
         void* d = nullptr;              // keys [n] (+ vals [n])
         size_t bytes = 0;
         cudaEvent_t in_done = nullptr, sort_done = nullptr, out_done = nullptr;
     };
-    HostSlot hslot[2];
+    static constexpr int kHostSlots = 3;
+    HostSlot hslot[kHostSlots];
     cudaStream_t h2d = nullptr, d2h = nullptr, comp = nullptr;
     cudaEvent_t join_in = nullptr, join_out = nullptr;   // order against the plan stream
     int64_t submits = 0;
