@@ -6,6 +6,11 @@ timeout 600 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_
 for w in sort_kv sort_u32_small maxsub sum; do
   timeout 300 python bench.py --workload $w --steps 10 --warmup 3 > gpurun_out/bench_$w.json 2>&1
 done
+for d in sorted reverse few; do
+  timeout 300 python bench.py --dist $d --steps 10 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/bench_sort_u32_$d.json 2>&1
+done
+timeout 300 python bench.py --workload sort_kv --dist few --steps 10 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/bench_sort_kv_few.json 2>&1
+timeout 120 python tools/pcie_probe.py > gpurun_out/pcie_probe.json 2>&1
 timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1

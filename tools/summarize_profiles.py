@@ -73,3 +73,18 @@ for cap, (wl, kern) in caps.items():
                                         "source": f"profiles/{rnd}/ncu_{wl}_{kern}.json"}
     print(wl, kern, s["gpu__time_duration.sum"], f"dram {(rd + wr) / 1e9:.4f} GB")
 json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
+
+# ---- bench lines of the same build (last JSON line of each gpurun_out/bench_*.json)
+import glob  # noqa: E402
+
+for bp in sorted(glob.glob(os.path.join(G, "bench_*.json"))) + [os.path.join(G, "pcie_probe.json")]:
+    if not os.path.exists(bp):
+        continue
+    lines = [ln for ln in open(bp).read().splitlines() if ln.startswith("{")]
+    if not lines:
+        continue
+    with open(os.path.join(out, os.path.basename(bp)), "w") as f:
+        f.write(lines[-1] + "\n")
+    d = json.loads(lines[-1])
+    if "ms_per_step" in d:
+        print(os.path.basename(bp), round(d["ms_per_step"], 4), "ms", d.get("value"), d.get("unit"))
