@@ -156,7 +156,7 @@ dc_status dc_run_mergesort_host(dc_plan_t plan, dc_key_type key_type, void *h_ke
                                 uint32_t *h_vals);
 
 /* Streaming end-to-end sorts of HOST buffers (pinned for overlap).  Each
- * submission copies h_in_keys (+h_in_vals) into one of two plan-owned device
+ * submission copies h_in_keys (+h_in_vals) into one of three plan-owned device
  * slots, sorts there and copies the result to h_out_keys (+h_out_vals); the
  * host input is not modified.  Work of consecutive submissions overlaps: the
  * upload of one, the sort of the previous and the download of the one before
