@@ -113,6 +113,13 @@ dc_status dc_plan_schedule(dc_plan_t plan, dc_key_type key_type, int32_t with_va
  * sort4_kernels.cuh).  Results are identical either way. */
 dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
 
+/* Enable (default) or disable the fused partition of L2-resident sorts (n <
+ * 2^23): every one-level merge CTA finds the co-ranks of its own output tile
+ * (two 33-ary warp searches, Alg 3's fn(id, param) inside the merge kernel,
+ * P:L325-332) instead of a separate NK2 launch per level.  Results are
+ * identical either way. */
+dc_status dc_plan_set_fused_partition(dc_plan_t plan, int32_t enable);
+
 /* Enable (default) or disable CUDA-graph replay of the sort's launch sequence:
  * the first dc_run_mergesort for a given (keys, vals, key type) runs eagerly,
  * the second captures a graph, later ones replay it.  Disabled automatically

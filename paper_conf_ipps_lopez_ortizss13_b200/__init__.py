@@ -63,6 +63,7 @@ _SIGS = {
     "dc_plan_schedule": ([_P, ctypes.c_int, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
                           ctypes.POINTER(_I32), ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
+    "dc_plan_set_fused_partition": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_graphs": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_pipeline": ([_P, _I32], ctypes.c_int),
     "dc_sort_host_submit": ([_P, ctypes.c_int, _P, _P, _P, _P], ctypes.c_int),
@@ -301,8 +302,12 @@ class Plan:
         """CUDA-graph replay of the sort's launch sequence (default on)."""
         _check(lib().dc_plan_set_graphs(self._h, int(enable)))
 
+    def set_fused_partition(self, enable: bool) -> None:
+        """L2-resident sorts: merge CTAs find their own co-ranks (default on)."""
+        _check(lib().dc_plan_set_fused_partition(self._h, int(enable)))
+
     def set_two_level(self, enable: bool) -> None:
-        """Two merge levels per HBM pass for keys-only sorts (default off)."""
+        """Two merge levels per HBM pass for keys-only sorts of n >= 2^23 (default on)."""
         _check(lib().dc_plan_set_two_level(self._h, int(enable)))
 
     def scratch_bytes(self, with_vals: bool = False) -> int:

@@ -69,7 +69,13 @@ constexpr SortCfg kCfgFast{DC_FAST_NT1, DC_FAST_IT1, DC_FAST_NT3, DC_FAST_IT};
 constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3, DC_STABLE_IT};
 // Small inputs (n < kSmallN, L2-resident): quarter-size tiles so that the
 // fused kernel and every merge level still launch >= ~150 CTAs.
-constexpr SortCfg kCfgFastSmall{128, DC_FAST_IT, 128, DC_FAST_IT};
+#ifndef DC_SMALL_NT1
+#define DC_SMALL_NT1 128
+#endif
+#ifndef DC_SMALL_IT1
+#define DC_SMALL_IT1 DC_FAST_IT
+#endif
+constexpr SortCfg kCfgFastSmall{DC_SMALL_NT1, DC_SMALL_IT1, 128, DC_FAST_IT};
 constexpr SortCfg kCfgStableSmall{128, DC_STABLE_IT, 128, DC_STABLE_IT};
 constexpr int64_t kSmallN = 1LL << 23;
 constexpr int cmin(int a, int b) { return a < b ? a : b; }
@@ -288,12 +294,16 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     constexpr SortCfg C = cfg_for<K, V, SMALL>();
     auto* k1 = dc::nk1_blocksort<C.nt1, C.it1, K, V>;
     auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
+    auto* k3sp = dc::nk3_merge_sp<C.nt3, C.it, K, V>;   // partition fused (SMALL)
     static bool attr_done = false;   // per key/value instantiation
     if (!attr_done) {
         DC_CUDA(p, cudaFuncSetAttribute(k1, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         nk1_smem_bytes(C, hv)));
         DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         nk3_smem_bytes(C, hv)));
+        if (SMALL)
+            DC_CUDA(p, cudaFuncSetAttribute(k3sp, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            nk3_smem_bytes(C, hv)));
         attr_done = true;
     }
 
@@ -317,6 +327,13 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         const int tpg = (int)num_tiles(std::min<int64_t>(2 * w, end - org), C.tout());
         const int tiles = (int)(num_tiles(end - org, 2 * w) * tpg);
         const dc::PairGeom g{org, w, w, end, tpg};
+        if (SMALL && p->fuse_partition) {
+            // L2-resident: every merge CTA finds its own co-ranks (one launch per level)
+            TimedScope ts(p, DC_KERNEL_NK3_MERGE, st);
+            k3sp<<<tiles, C.nt3, nk3_smem_bytes(C, hv), st>>>(cur_k, cur_v, oth_k, oth_v, g);
+            DC_LAUNCHED(p);
+            return DC_OK;
+        }
         {
             TimedScope ts(p, DC_KERNEL_NK2_PARTITION, st);
 #ifndef DC_NK2_WARP_ALL
@@ -863,6 +880,13 @@ static void drop_graphs(dc_plan_t p) {
 dc_status dc_plan_set_two_level(dc_plan_t p, int32_t enable) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     p->two_level = enable != 0;
+    drop_graphs(p);
+    return DC_OK;
+}
+
+dc_status dc_plan_set_fused_partition(dc_plan_t p, int32_t enable) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    p->fuse_partition = enable != 0;
     drop_graphs(p);
     return DC_OK;
 }

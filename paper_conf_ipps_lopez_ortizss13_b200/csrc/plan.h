@@ -67,6 +67,7 @@ struct dc_plan_s {
     // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
     // two-level partition costs 0.21 ms per pass vs 2 x 0.03.
     bool two_level = true;    // 4-way passes for large keys-only sorts (sort4_kernels.cuh)
+    bool fuse_partition = true;   // small sorts: merge CTAs find their own co-ranks
     // D&C sum (f4): per-CTA parts + ticket + result
     long long* sum_state = nullptr;
     int sum_grid = 0;

@@ -643,6 +643,45 @@ nk3_merge(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v
                              smem + TW, smem_addr(&bar));
 }
 
+// One merge level with the partition fused in (L2-resident sorts, where a
+// level is a few microseconds and a separate NK2 launch is a large share):
+// warps 0 and 1 of CTA j find the co-ranks of the tile's first and last+1
+// outputs with 33-ary warp searches (a few dependent L2 round trips), then
+// the CTA merges its tile as nk3_merge does.
+template <int NT, int IT, class K, bool V>
+__global__ void __launch_bounds__(NT)
+nk3_merge_sp(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
+             uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v, PairGeom g) {
+    static_assert(NT >= 64, "two searching warps");
+    constexpr int TOUT = NT * IT;
+    constexpr int TW = tile_words(TOUT, IT + 16);
+    extern __shared__ __align__(16) uint32_t smem[];
+    __shared__ __align__(8) uint64_t bar;
+    __shared__ int cr[2];
+    const int j = blockIdx.x;
+    long long s, a_len, b_len, dd0, dd1;
+    g.tile_of(j, TOUT, s, a_len, b_len, dd0, dd1);
+    if (dd0 >= a_len + b_len) return;                 // empty tile (whole CTA)
+    const int warp = threadIdx.x >> 5;
+    if (warp < 2) {
+        const long long diag = warp == 0 ? dd0 : dd1;
+        const uint32_t* A = src_k + s;
+        const uint32_t* B = src_k + s + a_len;
+        const long long lo = max(0LL, diag - b_len), hi = min(diag, a_len);
+        const long long c = warp_first_false(lo, hi, [&](long long m) {
+            return !K::lt(__ldg(B + (diag - 1 - m)), __ldg(A + m));
+        });
+        if ((threadIdx.x & 31) == 0) cr[warp] = (int)c;
+    }
+    __syncthreads();
+    const int i0 = cr[0], i1 = cr[1];
+    const int na = i1 - i0;
+    const int nb = (int)(dd1 - dd0) - na;
+    merge_tile<NT, IT, K, V>(src_k, src_v, g.end, s + i0, na, src_k, src_v, g.end,
+                             s + a_len + (dd0 - i0), nb, dst_k, dst_v, s + dd0, smem,
+                             smem + TW, smem_addr(&bar));
+}
+
 // ------------------------------------------- merges of separately stored runs
 // The first round of the multi-GPU G-way merge reads its two runs straight
 // from the sorted shards of two (peer) GPUs -- the exchange fused into the

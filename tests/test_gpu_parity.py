@@ -171,6 +171,31 @@ def test_sort_small_config_boundaries(dc, oracle_mod, n, with_vals):
     assert np.array_equal(_np_keys(k_out, "u32"), ek)
 
 
+@pytest.mark.parametrize("n", [SMALL_TILE + 1, 5 * SMALL_TILE + 77, 1 << 20, (1 << 22) + 3])
+@pytest.mark.parametrize("key_type,with_vals", [("u32", False), ("i32", False), ("f32", False),
+                                                ("u32", True)])
+def test_sort_small_partition_fused_vs_separate(dc, oracle_mod, n, key_type, with_vals):
+    """L2-resident sorts: merge CTAs that find their own co-ranks (default) and
+    the separate NK2 launch give the oracle's result bit for bit."""
+    keys = dcgen.sort_keys(n, "few" if n % 2 else "uniform", seed=77, key_type=key_type,
+                           device="cuda")
+    k_np = _np_keys(keys, key_type)
+    if with_vals:
+        ek, ev = oracle_mod.mergesort(k_np, np.arange(n, dtype=np.uint32), key_type=key_type)
+    else:
+        ek = oracle_mod.mergesort(k_np, key_type=key_type)
+    for fused in (True, False):
+        k = keys.clone()
+        v = dcgen.sort_vals(n, device="cuda") if with_vals else None
+        plan = dc.Plan(n)
+        plan.set_fused_partition(fused)
+        plan.sort_(k, v, key_type=key_type)
+        torch.cuda.synchronize()
+        assert np.array_equal(_np_keys(k, key_type).view(np.uint32), ek.view(np.uint32)), fused
+        if with_vals:
+            assert np.array_equal(v.cpu().numpy().view(np.uint32), ev), fused
+
+
 @pytest.mark.parametrize("n", [1 << 20, (1 << 23) + 5])
 def test_sort_graph_replay_same_buffers(dc, oracle_mod, n):
     """First call eager, second captures a CUDA graph, later calls replay it."""
