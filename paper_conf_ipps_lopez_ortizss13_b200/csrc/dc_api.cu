@@ -67,6 +67,14 @@ struct SortCfg {
 #endif
 constexpr SortCfg kCfgFast{DC_FAST_NT1, DC_FAST_IT1, DC_FAST_NT3, DC_FAST_IT};
 constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3, DC_STABLE_IT};
+// Key-value NK1: (key, index) pairs in registers need ~107 registers, so a
+// 512-thread CTA runs alone on its SM (16 warps, latency-bound); 256-thread
+// CTAs run two per SM.  Their 8448-key tiles cost one more global level, but
+// NK1 drops 4.45 -> 3.33 ms at 2^28 (11.71 -> 11.23 ms per sort, measured).
+#ifndef DC_KV_NT1
+#define DC_KV_NT1 256
+#endif
+constexpr SortCfg kCfgKV{DC_KV_NT1, DC_STABLE_IT, DC_STABLE_NT3, DC_STABLE_IT};
 // Small inputs (n < kSmallN, L2-resident): quarter-size tiles so that the
 // fused kernel and every merge level still launch >= ~150 CTAs.
 #ifndef DC_SMALL_NT1
@@ -79,17 +87,19 @@ constexpr SortCfg kCfgFastSmall{DC_SMALL_NT1, DC_SMALL_IT1, 128, DC_FAST_IT};
 constexpr SortCfg kCfgStableSmall{128, DC_STABLE_IT, 128, DC_STABLE_IT};
 constexpr int64_t kSmallN = 1LL << 23;
 constexpr int cmin(int a, int b) { return a < b ? a : b; }
-constexpr int kMinTout = cmin(cmin(kCfgFast.tout(), kCfgStable.tout()),
+constexpr int kMinTout = cmin(cmin(cmin(kCfgFast.tout(), kCfgStable.tout()), kCfgKV.tout()),
                               cmin(kCfgFastSmall.tout(), kCfgStableSmall.tout()));
 
 template <class K, bool V, bool SMALL>
 constexpr SortCfg cfg_for() {
-    return (V || K::kNeedStable) ? (SMALL ? kCfgStableSmall : kCfgStable)
+    return V ? (SMALL ? kCfgStableSmall : kCfgKV)
+           : K::kNeedStable ? (SMALL ? kCfgStableSmall : kCfgStable)
                                  : (SMALL ? kCfgFastSmall : kCfgFast);
 }
 SortCfg cfg_for_runtime(dc_key_type kt, bool vals, int64_t n) {
     const bool small = n < kSmallN;
-    return (vals || kt == DC_KEY_F32) ? (small ? kCfgStableSmall : kCfgStable)
+    return vals ? (small ? kCfgStableSmall : kCfgKV)
+           : kt == DC_KEY_F32 ? (small ? kCfgStableSmall : kCfgStable)
                                       : (small ? kCfgFastSmall : kCfgFast);
 }
 
@@ -136,7 +146,7 @@ int global_passes(int64_t n, int64_t tile) {
 
 // One-level pass: every pair of width 2w is cut into ceil(2w / tout) tiles, so
 // at most one extra (short) tile per pair; pairs <= n / (2 * min tile) + 1.
-constexpr int kMinTile = cmin(cmin(kCfgFast.tile(), kCfgStable.tile()),
+constexpr int kMinTile = cmin(cmin(cmin(kCfgFast.tile(), kCfgStable.tile()), kCfgKV.tile()),
                               cmin(kCfgFastSmall.tile(), kCfgStableSmall.tile()));
 size_t split_entries(int64_t n) {
     return (size_t)num_tiles(n, kMinTout) + (size_t)num_tiles(n, 2 * (int64_t)kMinTile) + 2;
@@ -171,7 +181,7 @@ constexpr TwoCfg two_cfg() { return V ? kTwoKV : kTwoKeys; }
 size_t two_level_tab_entries(int64_t) { return 0; }
 size_t two_level_bnd_entries(int64_t n) {
     // groups at the smallest width (w = tile) have the most tiles
-    const int64_t w = std::min(kCfgFast.tile(), kCfgStable.tile());
+    const int64_t w = cmin(cmin(kCfgFast.tile(), kCfgStable.tile()), kCfgKV.tile());
     const int64_t groups = (n + 4 * w - 1) / (4 * w);
     return 4 * ((size_t)(groups * num_tiles(4 * w, kTwoMinT)) + 2);
 }

@@ -122,7 +122,7 @@ def test_sort_two_level_edge_distributions(dc, oracle_mod, n, dist):
     assert np.array_equal(_np_keys(keys, "u32"), expect)
 
 
-STABLE_TWO_LEVEL = [(1 << 23) + 7, 5 * 16896 * 128 + 16896 * 3 + 11]
+STABLE_TWO_LEVEL = [(1 << 23) + 7, 5 * 16896 * 128 + 16896 * 3 + 11, 9 * 8448 * 128 + 8448 * 5 + 13]
 
 
 @pytest.mark.parametrize("n", STABLE_TWO_LEVEL)
@@ -423,13 +423,17 @@ def test_maxsub_host_buffer(dc, oracle_mod):
     assert dc.Plan(n).max_subarray_host(x) == oracle_mod.maxsub(x.numpy())
 
 
-def test_launch_counts(dc):
-    n = 1 << 20
+@pytest.mark.parametrize("n,fused", [(1 << 20, True), (1 << 20, False), ((1 << 23) + 5, True)])
+def test_launch_counts(dc, n, fused):
+    """NK1 + per pass: NK2 + NK3 (a two-level pass: select + 4-way merge); below
+    2^23 keys the fused partition makes a one-level pass a single launch."""
     p = dc.Plan(n)
     p.set_graphs(False)
+    p.set_fused_partition(fused)
     keys = dcgen.sort_keys(n, "uniform", device="cuda")
     p.sort_(keys, key_type="u32")
     s = p.schedule("u32", False)
     P, H = s["global_passes"], s["hbm_passes"]
-    single = P - 2 * (P - H)          # one-level and two-level passes: 2 launches each
-    assert p.launch_count() == 1 + 2 * single + 2 * (H - single)
+    single = P - 2 * (P - H)          # one-level passes; the rest are two-level passes
+    per_single = 1 if (fused and n < (1 << 23)) else 2
+    assert p.launch_count() == 1 + per_single * single + 2 * (H - single)
