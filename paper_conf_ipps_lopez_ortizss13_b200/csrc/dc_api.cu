@@ -168,15 +168,31 @@ size_t split_entries(int64_t n) {
 #ifndef DC_TWO_IT_KV
 #define DC_TWO_IT_KV 25
 #endif
+// Keys only, selection fused into the pass (nk3_merge4 NSEL > 0, built with
+// -DDC_M4_NSEL=3): selector warps join the CTA, so the merge threads shrink
+// to 736 (896 threads x 72 registers fit the register file).  Measured at
+// 2^28: merges + selection 5.02 ms (3 selector warps) / 4.70 ms (6, with 640
+// merge threads) vs 4.36 ms for the separate nk2_select4 launch (0, default):
+// a boundary's ~11 dependent rounds need many warps in flight, which a
+// separate full-GPU launch provides and a few warps per SM do not.
+#ifndef DC_M4_NSEL
+#define DC_M4_NSEL 0
+#endif
+#ifndef DC_TWO_NT_FUSED
+#define DC_TWO_NT_FUSED 736
+#endif
 struct TwoCfg {
-    int nt, it;
+    int nt, it, nsel;
     constexpr int T() const { return nt * it; }
+    constexpr int threads() const { return nt + 64 + 32 * nsel; }
 };
-constexpr TwoCfg kTwoKeys{DC_TWO_NT, DC_TWO_IT};
-constexpr TwoCfg kTwoKV{DC_TWO_NT_KV, DC_TWO_IT_KV};
-constexpr int kTwoMinT = cmin(kTwoKeys.T(), kTwoKV.T());
-template <bool V>
-constexpr TwoCfg two_cfg() { return V ? kTwoKV : kTwoKeys; }
+constexpr TwoCfg kTwoKeys = DC_M4_NSEL > 0 ? TwoCfg{DC_TWO_NT_FUSED, DC_TWO_IT, DC_M4_NSEL}
+                                           : TwoCfg{DC_TWO_NT, DC_TWO_IT, 0};
+constexpr TwoCfg kTwoKV{DC_TWO_NT_KV, DC_TWO_IT_KV, 0};
+constexpr TwoCfg kTwoF32{DC_TWO_NT, DC_TWO_IT, 0};   // f32 keys: stable merges, separate select
+constexpr int kTwoMinT = cmin(cmin(kTwoKeys.T(), kTwoKV.T()), kTwoF32.T());
+template <class K, bool V>
+constexpr TwoCfg two_cfg() { return V ? kTwoKV : (K::kNeedStable ? kTwoF32 : kTwoKeys); }
 
 size_t two_level_tab_entries(int64_t) { return 0; }
 size_t two_level_bnd_entries(int64_t n) {
@@ -434,8 +450,10 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         if (two) {
             int* tab = split + align_up(split_entries(n) * 4, 256) / 4;
             dc::Cut4* cuts = (dc::Cut4*)(tab + align_up(two_level_tab_entries(n) * 4, 256) / 4);
-            constexpr TwoCfg TC = two_cfg<V>();
-            auto* k32 = dc::nk3_merge4<TC.nt, TC.it, K, V>;
+            constexpr TwoCfg TC = two_cfg<K, V>();
+            auto* k32 = dc::nk3_merge4<TC.nt, TC.it, K, V, (K::kNeedStable ? 0 : TC.nsel)>;
+            constexpr bool fused_sel = !K::kNeedStable && TC.nsel > 0;
+            constexpr int thr2 = fused_sel ? TC.threads() : TC.nt + 64;
             constexpr int smem2 = dc::m4_smem_bytes(TC.T(), TC.it, V);
             static int grid2 = 0;                        // per instantiation
             if (!grid2) {
@@ -444,13 +462,13 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
                 int dev = 0, sms = 148, occ = 1;
                 cudaGetDevice(&dev);
                 cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, TC.nt + 64, smem2);
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, thr2, smem2);
                 grid2 = sms * (occ > 0 ? occ : 1);
             }
             for (; w < n; w *= 4) {
                 const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), TC.T());
                 const int tiles2 = (int)(((n + 4 * w - 1) / (4 * w)) * tpg);
-                {
+                if (!fused_sel) {
                     TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
                     dc::nk2_select4<K><<<(tiles2 + 3) / 4, 128, 0, p->stream>>>(
                         cur_k, n, w, TC.T(), tpg, tiles2, cuts);
@@ -458,7 +476,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
                 }
                 {
                     TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                    k32<<<std::min(tiles2, grid2), TC.nt + 64, smem2, p->stream>>>(
+                    k32<<<std::min(tiles2, grid2), thr2, smem2, p->stream>>>(
                         cur_k, cur_v, oth_k, oth_v, n, w, tpg, cuts, tiles2);
                     DC_LAUNCHED(p);
                 }

@@ -85,16 +85,17 @@ __device__ __forceinline__ int sel4_pivot(int lo, int W, int step, int t) {
 // shuffle).  The largest taken pivot raises lo_q, the smallest untaken one
 // lowers hi_q.  Once every window has <= 8 elements all of them are pivots,
 // the brackets are exact and every window closes: c_q = lo_q.
+// The cut of tile j's first output, computed by one converged warp (the
+// result is valid in every lane).  An empty tile (end of the last group)
+// gets the zero cut.
 template <class K>
-__global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long long w, int T,
-                            int tpg, int num_tiles, Cut4* __restrict__ cut) {
-    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
-    if (j >= num_tiles) return;                       // warp-uniform
+__device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, long long n,
+                                             long long w, int T, int tpg, int j) {
     const int lane = threadIdx.x & 31;
     const int q = lane >> 3, t = lane & 7;
     const Tile4Geo g(n, w, T, tpg, j);
     const int d = g.d0;
-    if (d >= g.tot) return;                           // empty tile (last group)
+    if (d >= g.tot) return Cut4{{0, 0, 0, 0}};      // empty tile (last group)
     const uint32_t* R[4];
 #pragma unroll
     for (int r = 0; r < 4; ++r) R[r] = src + g.s + r * w;
@@ -208,12 +209,22 @@ __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long 
             }
         }
     }
-    if (lane == 0) {
-        Cut4 c;
+    Cut4 c;
 #pragma unroll
-        for (int r = 0; r < 4; ++r) c.c[r] = lo[r];
-        cut[j] = c;
-    }
+    for (int r = 0; r < 4; ++r) c.c[r] = lo[r];
+    return c;
+}
+
+// NK2-4 as its own launch: one warp per tile boundary.
+template <class K>
+__global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long long w, int T,
+                            int tpg, int num_tiles, Cut4* __restrict__ cut) {
+    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    if (j >= num_tiles) return;                       // warp-uniform
+    const Tile4Geo g(n, w, T, tpg, j);
+    if (g.d0 >= g.tot) return;                        // empty tile (last group)
+    const Cut4 c = select4_warp<K>(src, n, w, T, tpg, j);
+    if ((threadIdx.x & 31) == 0) cut[j] = c;
 }
 
 // ------------------------------------------------------------------ NK3-4
@@ -281,6 +292,16 @@ __device__ __forceinline__ void consumer_sync() {
 // J = blockIdx.x + i * gridDim.x; empty tiles (end of the last group) pass
 // through with no work.
 //
+// NSEL > 0 fuses NK2-4 into the pass: the CTA owns a contiguous tile range
+// [t0, t1), and NSEL selector warps compute the cuts of its boundaries
+// t0 .. t1 (boundary i by warp i % NSEL) into a ring of RS slots in shared
+// memory, running ahead of the producer.  cfull[s]: cut written (selector
+// lane 0 arrives); cempty[s]: the producer has filled the tile that starts
+// at that boundary (it waits for every boundary in order, so each slot is
+// at most one phase ahead).  The standalone select launch and its ~11
+// dependent rounds per boundary move off the critical path, except for the
+// CTA's first two boundaries.
+//
 // Keys-only u32/i32 (equal keys indistinguishable): pad-safe merges and a
 // bitonic stage 2 (Y stored descending), no bounds checks.  Stable variants
 // (values, or f32 keys whose +0/-0 must keep their order): bounds-checked
@@ -289,8 +310,8 @@ __device__ __forceinline__ void consumer_sync() {
 #ifndef DC_M4_MINB   // CTAs per SM the register budget is sized for
 #define DC_M4_MINB 1
 #endif
-template <int NT, int IT, class K, bool V>
-__global__ void __launch_bounds__(NT + 64, DC_M4_MINB)
+template <int NT, int IT, class K, bool V, int NSEL = 0>
+__global__ void __launch_bounds__(NT + 64 + 32 * NSEL, DC_M4_MINB)
 nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
            uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v, long long n, long long w,
            int tpg, const Cut4* __restrict__ cut, int num_tiles) {
@@ -302,15 +323,23 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
     constexpr int BW = (V ? 2 : 1) * KW;               // words per buffer
     constexpr int GU = m4_guard(IT);
     constexpr uint32_t VOFF = 4u * KW;                 // key -> value byte offset
+    constexpr int RS = NSEL > 0 ? 3 * NSEL : 1;        // cut ring slots (multiple of NSEL)
     extern __shared__ __align__(16) uint32_t sm[];
     __shared__ __align__(8) uint64_t full[2], empty[2];
+    __shared__ __align__(8) uint64_t cfull[RS], cempty[RS];
     __shared__ Tile4 meta[2];
+    __shared__ Cut4 ring[RS];
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint32_t SM0 = smem_addr(sm);
     const long long n4 = n & ~3LL;
-    const int my_tiles = (int)blockIdx.x < num_tiles
-                             ? (num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+    // tile i of this CTA: interleaved (cuts from NK2-4) or a contiguous range
+    const int t0 = NSEL > 0 ? (int)(((long long)blockIdx.x * num_tiles) / gridDim.x) : 0;
+    const int t1 = NSEL > 0 ? (int)(((long long)(blockIdx.x + 1) * num_tiles) / gridDim.x) : 0;
+    const int my_tiles = NSEL > 0 ? t1 - t0
+                         : ((int)blockIdx.x < num_tiles
+                                ? (num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0);
+    auto tile_of = [&](int i) { return NSEL > 0 ? t0 + i : (int)blockIdx.x + i * (int)gridDim.x; };
 
     if (tid == 0) {
 #pragma unroll
@@ -318,8 +347,30 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
             mbar_init(smem_addr(&full[b]), 1);
             mbar_init(smem_addr(&empty[b]), NC / 32);
         }
+        if (NSEL > 0) {
+            for (int r = 0; r < RS; ++r) {
+                mbar_init(smem_addr(&cfull[r]), 1);
+                mbar_init(smem_addr(&cempty[r]), 1);
+            }
+        }
     }
     __syncthreads();
+
+    if (NSEL > 0 && tid >= NC + 32) {
+        // ---------------------------------------------------- selector warps
+        const int sw = (tid - NC - 32) >> 5;
+        for (int i = sw; i <= my_tiles; i += NSEL) {
+            const int slot = i % RS, rnd = i / RS;
+            if (rnd > 0) mbar_wait(smem_addr(&cempty[slot]), (uint32_t)((rnd - 1) & 1));
+            const Cut4 c = select4_warp<K>(src_k, n, w, T, tpg, t0 + i);
+            if (lane == 0) {
+                ring[slot] = c;
+                mbar_arrive(smem_addr(&cfull[slot]));   // release: the cut
+            }
+            __syncwarp();
+        }
+        return;
+    }
 
     if (tid >= NC) {
         // ------------------------------------------------------ producer warp
@@ -328,15 +379,21 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
         // copies each piece's 16-byte-aligned interior [g0 & ~3, tend); the
         // lanes store the ragged end (< 4 words, or the part at/after n4) and
         // IT pads behind each piece.
-        auto fill = [&](int J, int b) {
+        auto fill = [&](int i, int b) {
+            const int J = tile_of(i);
             const Tile4Geo g(n, w, T, tpg, J);
             int c0[4], c1[4];
+            if (NSEL > 0)   // boundary i, in order (see the ring protocol above)
+                mbar_wait(smem_addr(&cfull[i % RS]), (uint32_t)((i / RS) & 1));
             if (g.d0 < g.tot) {
-                const Cut4 a = cut[J];
+                const Cut4 a = NSEL > 0 ? ring[i % RS] : cut[J];
                 Cut4 e;
                 if (g.d1 == g.tot) {
 #pragma unroll
                     for (int r = 0; r < 4; ++r) e.c[r] = g.l[r];
+                } else if (NSEL > 0) {
+                    mbar_wait(smem_addr(&cfull[(i + 1) % RS]), (uint32_t)(((i + 1) / RS) & 1));
+                    e = ring[(i + 1) % RS];
                 } else {
                     e = cut[J + 1];
                 }
@@ -345,6 +402,10 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
             } else {
 #pragma unroll
                 for (int r = 0; r < 4; ++r) c0[r] = c1[r] = 0;
+            }
+            if (NSEL > 0) {      // boundary i is dead once every lane has read it
+                __syncwarp();
+                if (lane == 0) mbar_arrive(smem_addr(&cempty[i % RS]));
             }
             Tile4 m;
             m.out = g.s + g.d0;
@@ -390,8 +451,8 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
                 }
             }
         };
-        if (my_tiles > 0) fill(blockIdx.x, 0);
-        if (my_tiles > 1) fill(blockIdx.x + gridDim.x, 1);
+        if (my_tiles > 0) fill(0, 0);
+        if (my_tiles > 1) fill(1, 1);
         for (int i = 0; i < my_tiles; ++i) {
             const int b = i & 1;
             mbar_wait(smem_addr(&empty[b]), (i >> 1) & 1);   // output of tile i written
@@ -407,7 +468,7 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
                 if (i + 2 < my_tiles) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
             }
             __syncwarp();
-            if (i + 2 < my_tiles) fill(blockIdx.x + (i + 2) * gridDim.x, b);
+            if (i + 2 < my_tiles) fill(i + 2, b);
         }
         if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
         return;
