@@ -124,15 +124,17 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
 #ifdef DC_SEL4_MAXROUNDS
     int dbg_rounds = 0;
 #endif
-    for (int round = 0;; ++round) {
-        // Progress guard: from round DC_SEL4_EXACT_FROM on, every undecided
-        // pivot's brackets are resolved by exact binary searches, so every
-        // round decides every pivot (never reached on the tested inputs).
-        const bool exact = round >= DC_SEL4_EXACT_FROM;
+    // One round; false once every window is closed.  Progress guard: from
+    // round DC_SEL4_EXACT_FROM on (the EXACT instantiation, a separate loop
+    // so the common rounds carry no fallback code), every undecided pivot's
+    // brackets are resolved by exact binary searches, so every round decides
+    // every pivot (never reached on the tested inputs).
+    auto round_step = [&](auto exact_tag) -> bool {
+        constexpr bool exact = decltype(exact_tag)::value;
 #ifdef DC_SEL4_MAXROUNDS
         if (++dbg_rounds > DC_SEL4_MAXROUNDS) {
             if (lane == 0) printf("select4 stall j=%d d=%d\n", j, d);
-            break;
+            return false;
         }
 #endif
         int W[4], st[4], open = 0;
@@ -142,7 +144,7 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
             st[r] = W[r] / 9;
             open |= W[r];
         }
-        if (open == 0) break;
+        if (open == 0) return false;
         int Wq = W[0], loq = lo[0], stq = st[0];
 #pragma unroll
         for (int r = 1; r < 4; ++r)
@@ -173,14 +175,16 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
                 if (a > 0) Lp = sel4_pivot(lo[r], W[r], st[r], a - 1) + 1;
                 if (a < 8) Up = sel4_pivot(lo[r], W[r], st[r], a);
             }
-            if (exact && other && !(dt | du) && active) {
-                int x0 = Lp, x1 = Up;                    // first position not preceding E
-                while (x0 < x1) {
-                    const int mid = (x0 + x1) >> 1;
-                    if (precedes<K>(__ldg(R[r] + mid), r, v, q)) x0 = mid + 1;
-                    else x1 = mid;
+            if constexpr (exact) {
+                if (other && !(dt | du) && active) {
+                    int x0 = Lp, x1 = Up;                // first position not preceding E
+                    while (x0 < x1) {
+                        const int mid = (x0 + x1) >> 1;
+                        if (precedes<K>(__ldg(R[r] + mid), r, v, q)) x0 = mid + 1;
+                        else x1 = mid;
+                    }
+                    Lp = Up = x0;
                 }
-                Lp = Up = x0;
             }
             SL += other ? Lp : 0;
             SU += other ? Up : 0;
@@ -208,7 +212,12 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
                 hi[r] = sel4_pivot(lo0, W[r], st[r], tu);
             }
         }
-    }
+        return true;
+    };
+    int round = 0;
+    bool more = true;
+    for (; more && round < DC_SEL4_EXACT_FROM; ++round) more = round_step(std::false_type{});
+    for (; more; ++round) more = round_step(std::true_type{});
     Cut4 c;
 #pragma unroll
     for (int r = 0; r < 4; ++r) c.c[r] = lo[r];
