@@ -63,39 +63,48 @@ __device__ __forceinline__ bool precedes(uint32_t x, int qx, uint32_t e, int qe)
     return K::lt(x, e) | ((!K::lt(e, x)) & (qx < qe));
 }
 
-// Position of pivot t (0..7) in a window [lo, lo + W): evenly spaced when
-// W >= 9 (strictly inside the window), every position when W <= 8.
+// Position of pivot t (0..PV-1) in a window [lo, lo + W): evenly spaced when
+// W >= PV + 1 (strictly inside the window), every position when W <= PV.
+template <int PV>
 __device__ __forceinline__ int sel4_pivot(int lo, int W, int step, int t) {
-    return lo + (W >= 9 ? (t + 1) * step : min(t, W - 1));
+    return lo + (W >= PV + 1 ? (t + 1) * step : min(t, W - 1));
 }
 
 // ------------------------------------------------------------------ NK2-4
 #ifndef DC_SEL4_EXACT_FROM
 #define DC_SEL4_EXACT_FROM 48
 #endif
-// One warp per tile boundary.  Lane L owns pivot t = L & 7 of run q = L >> 3.
-// Invariant: lo_q <= c_q <= hi_q, with the values R_q[lo_q - 1] (taken) and
-// R_q[hi_q] (not taken) known.  Every round each run with a non-empty window
-// puts 8 pivots in it; a pivot E (run q, position p) is
+// A group of LB = 4*PV lanes per tile boundary (PV = 8: one boundary per
+// warp; PV = 4: two).  Lane l of a group owns pivot t = l % PV of run
+// q = l / PV.  Invariant: lo_q <= c_q <= hi_q, with the values R_q[lo_q - 1]
+// (taken) and R_q[hi_q] (not taken) known.  Every round each run with a
+// non-empty window puts PV pivots in it; a pivot E (run q, position p) is
 //   * taken      if it precedes a known taken edge of another run, or if
 //                 p + sum_q' U_q'(E) < d,
 //   * not taken  if a known untaken edge precedes it, or p + sum L_q'(E) >= d,
 // where [L_q', U_q'] brackets #R_q' elements preceding E between the
 // neighbouring pivots of run q' (positions in closed form, values by
 // shuffle).  The largest taken pivot raises lo_q, the smallest untaken one
-// lowers hi_q.  Once every window has <= 8 elements all of them are pivots,
+// lowers hi_q.  Once every window has <= PV elements all of them are pivots,
 // the brackets are exact and every window closes: c_q = lo_q.
-// The cut of tile j's first output, computed by one converged warp (the
-// result is valid in every lane).  An empty tile (end of the last group)
-// gets the zero cut.
-template <class K>
+// The cut of tile j's first output, computed by a converged warp (valid in
+// every lane of the boundary's group).  An empty tile (end of the last
+// group) or !valid gets the zero cut; its lanes still take part in the
+// warp's shuffles until every group of the warp is done.
+template <class K, int PV = 8>
 __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, long long n,
-                                             long long w, int T, int tpg, int j) {
+                                             long long w, int T, int tpg, int j,
+                                             bool valid = true) {
+    static_assert(PV == 8 || PV == 4, "8 pivots (one boundary per warp) or 4 (two)");
+    constexpr int LB = 4 * PV;
     const int lane = threadIdx.x & 31;
-    const int q = lane >> 3, t = lane & 7;
-    const Tile4Geo g(n, w, T, tpg, j);
+    const int base = lane & ~(LB - 1);                 // first lane of this boundary's group
+    const int ll = lane - base;
+    const int q = ll / PV, t = ll % PV;
+    const Tile4Geo g(n, w, T, tpg, valid ? j : 0);
     const int d = g.d0;
-    if (d >= g.tot) return Cut4{{0, 0, 0, 0}};      // empty tile (last group)
+    const bool live = valid && d < g.tot;
+    if (PV == 8 && !live) return Cut4{{0, 0, 0, 0}}; // whole warp: uniform exit
     const uint32_t* R[4];
 #pragma unroll
     for (int r = 0; r < 4; ++r) R[r] = src + g.s + r * w;
@@ -106,34 +115,37 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
     int lo[4], hi[4];
     uint32_t elo[4], ehi[4];
     {
-        // initial windows and their edge values (lane r: R_r[lo_r - 1], lane 4+r: R_r[hi_r])
+        // initial windows and their edge values (group lane r: R_r[lo_r - 1],
+        // group lane 4+r: R_r[hi_r]); a dead group has every window closed
         uint32_t ev = 0;
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
-            lo[r] = max(0, d - (g.tot - g.l[r]));
-            hi[r] = min(g.l[r], d);
-            const int pos = lane == r ? lo[r] - 1 : hi[r];
-            if ((lane == r || lane == 4 + r) && pos >= 0 && pos < g.l[r]) ev = __ldg(R[r] + pos);
+            lo[r] = live ? max(0, d - (g.tot - g.l[r])) : 0;
+            hi[r] = live ? min(g.l[r], d) : 0;
+            const int pos = ll == r ? lo[r] - 1 : hi[r];
+            if (live && (ll == r || ll == 4 + r) && pos >= 0 && pos < g.l[r])
+                ev = __ldg(R[r] + pos);
         }
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
-            elo[r] = __shfl_sync(0xffffffffu, ev, r);
-            ehi[r] = __shfl_sync(0xffffffffu, ev, 4 + r);
+            elo[r] = __shfl_sync(0xffffffffu, ev, base + r);
+            ehi[r] = __shfl_sync(0xffffffffu, ev, base + 4 + r);
         }
     }
 #ifdef DC_SEL4_MAXROUNDS
     int dbg_rounds = 0;
 #endif
-    // One round; false once every window is closed.  Progress guard: from
-    // round DC_SEL4_EXACT_FROM on (the EXACT instantiation, a separate loop
-    // so the common rounds carry no fallback code), every undecided pivot's
-    // brackets are resolved by exact binary searches, so every round decides
-    // every pivot (never reached on the tested inputs).
+    // One round; false once every window of every group in the warp is
+    // closed.  Progress guard: from round DC_SEL4_EXACT_FROM on (the EXACT
+    // instantiation, a separate loop so the common rounds carry no fallback
+    // code), every undecided pivot's brackets are resolved by exact binary
+    // searches, so every round decides every pivot (never reached on the
+    // tested inputs).
     auto round_step = [&](auto exact_tag) -> bool {
         constexpr bool exact = decltype(exact_tag)::value;
 #ifdef DC_SEL4_MAXROUNDS
         if (++dbg_rounds > DC_SEL4_MAXROUNDS) {
-            if (lane == 0) printf("select4 stall j=%d d=%d\n", j, d);
+            if (ll == 0) printf("select4 stall j=%d d=%d\n", j, d);
             return false;
         }
 #endif
@@ -141,16 +153,20 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
             W[r] = hi[r] - lo[r];
-            st[r] = W[r] / 9;
+            st[r] = W[r] / (PV + 1);
             open |= W[r];
         }
-        if (open == 0) return false;
+        if (PV == 8) {
+            if (open == 0) return false;
+        } else if (!__any_sync(0xffffffffu, open != 0)) {
+            return false;
+        }
         int Wq = W[0], loq = lo[0], stq = st[0];
 #pragma unroll
         for (int r = 1; r < 4; ++r)
             if (q == r) { Wq = W[r]; loq = lo[r]; stq = st[r]; }
         const bool active = Wq > 0;
-        const int p = sel4_pivot(loq, Wq, stq, t);
+        const int p = sel4_pivot<PV>(loq, Wq, stq, t);
         const uint32_t v = active ? __ldg(Rq + p) : 0u;
         int SL = p, SU = p;
         bool dt = false, du = false;
@@ -158,22 +174,22 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
         //  own run and closed windows are masked with selects)
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
-            // #pivots of run r preceding this lane's pivot (search over lanes 8r..8r+7)
-            int a = 0;                                   // in [0, 8]
+            // #pivots of run r preceding this lane's pivot (search over the group's lanes PV*r ..)
+            int a = 0;                                   // in [0, PV]
 #pragma unroll
-            for (int step = 4; step >= 1; step >>= 1) {
-                const uint32_t V = __shfl_sync(0xffffffffu, v, 8 * r + a + step - 1);
+            for (int step = PV / 2; step >= 1; step >>= 1) {
+                const uint32_t V = __shfl_sync(0xffffffffu, v, base + PV * r + a + step - 1);
                 a += precedes<K>(V, r, v, q) ? step : 0;
             }
-            const uint32_t V7 = __shfl_sync(0xffffffffu, v, 8 * r + 7);
-            a += (a == 7 && precedes<K>(V7, r, v, q)) ? 1 : 0;
+            const uint32_t VL = __shfl_sync(0xffffffffu, v, base + PV * r + PV - 1);
+            a += (a == PV - 1 && precedes<K>(VL, r, v, q)) ? 1 : 0;
             const bool other = r != q;
             dt |= other & (lo[r] > 0) & !precedes<K>(elo[r], r, v, q);      // E before a taken edge
             du |= other & (hi[r] < g.l[r]) & precedes<K>(ehi[r], r, v, q);  // untaken edge before E
             int Lp = lo[r], Up = hi[r];
             if (W[r] > 0) {
-                if (a > 0) Lp = sel4_pivot(lo[r], W[r], st[r], a - 1) + 1;
-                if (a < 8) Up = sel4_pivot(lo[r], W[r], st[r], a);
+                if (a > 0) Lp = sel4_pivot<PV>(lo[r], W[r], st[r], a - 1) + 1;
+                if (a < PV) Up = sel4_pivot<PV>(lo[r], W[r], st[r], a);
             }
             if constexpr (exact) {
                 if (other && !(dt | du) && active) {
@@ -193,23 +209,24 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
         // an edge decision takes precedence (dt and du exclude each other).
         const bool taken = active && (dt || (!du && SU < d));
         const bool untaken = active && (du || (!dt && SL >= d));
-        const unsigned mt = __ballot_sync(0xffffffffu, taken);
-        const unsigned mu = __ballot_sync(0xffffffffu, untaken);
+        const unsigned mt = __ballot_sync(0xffffffffu, taken) >> base;
+        const unsigned mu = __ballot_sync(0xffffffffu, untaken) >> base;
+        constexpr unsigned PM = (1u << PV) - 1u;
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
-            const unsigned gt = (mt >> (8 * r)) & 0xffu, gu = (mu >> (8 * r)) & 0xffu;
+            const unsigned gt = (mt >> (PV * r)) & PM, gu = (mu >> (PV * r)) & PM;
             const int tt = 31 - __clz(gt | 1u);             // largest taken pivot (0 if none)
-            const int tu = __ffs(gu | 0x80u) - 1;           // smallest untaken pivot (7 if none)
-            const uint32_t vt = __shfl_sync(0xffffffffu, v, 8 * r + tt);
-            const uint32_t vu = __shfl_sync(0xffffffffu, v, 8 * r + tu);
+            const int tu = __ffs(gu | (1u << (PV - 1))) - 1;   // smallest untaken (PV-1 if none)
+            const uint32_t vt = __shfl_sync(0xffffffffu, v, base + PV * r + tt);
+            const uint32_t vu = __shfl_sync(0xffffffffu, v, base + PV * r + tu);
             const int lo0 = lo[r];                          // this round's pivot base
             if (gt) {
                 elo[r] = vt;
-                lo[r] = sel4_pivot(lo0, W[r], st[r], tt) + 1;
+                lo[r] = sel4_pivot<PV>(lo0, W[r], st[r], tt) + 1;
             }
             if (gu) {
                 ehi[r] = vu;
-                hi[r] = sel4_pivot(lo0, W[r], st[r], tu);
+                hi[r] = sel4_pivot<PV>(lo0, W[r], st[r], tu);
             }
         }
         return true;
@@ -225,15 +242,25 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
 }
 
 // NK2-4 as its own launch: one warp per tile boundary.
+// NK2-4 as its own launch: BPW = 32 / (4 PV) tile boundaries per warp.
+#ifndef DC_SEL4_PV
+#define DC_SEL4_PV 4
+#endif
+constexpr int kSel4BPW = 32 / (4 * DC_SEL4_PV);      // boundaries per warp
 template <class K>
 __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long long w, int T,
                             int tpg, int num_tiles, Cut4* __restrict__ cut) {
-    const int j = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
-    if (j >= num_tiles) return;                       // warp-uniform
-    const Tile4Geo g(n, w, T, tpg, j);
-    if (g.d0 >= g.tot) return;                        // empty tile (last group)
-    const Cut4 c = select4_warp<K>(src, n, w, T, tpg, j);
-    if ((threadIdx.x & 31) == 0) cut[j] = c;
+    constexpr int PV = DC_SEL4_PV, LB = 4 * PV, BPW = 32 / LB;
+    const int wj = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * BPW;
+    if (wj >= num_tiles) return;                      // warp-uniform
+    const int lane = threadIdx.x & 31;
+    const int j = wj + lane / LB;
+    const bool valid = j < num_tiles;
+    const Cut4 c = select4_warp<K, PV>(src, n, w, T, tpg, j, valid);
+    if (valid && lane % LB == 0) {
+        const Tile4Geo g(n, w, T, tpg, j);
+        if (g.d0 < g.tot) cut[j] = c;                 // (empty tiles: no cut)
+    }
 }
 
 // ------------------------------------------------------------------ NK3-4

@@ -1,0 +1,7 @@
+#!/bin/bash
+mkdir -p gpurun_out /tmp/dcvar
+python paper_conf_ipps_lopez_ortizss13_b200/build.py --out /tmp/dcvar/lib_pv4.so -D DC_SEL4_PV=4 > /dev/null 2>&1
+DC_LIB=/tmp/dcvar/lib_pv4.so timeout 900 python -m pytest tests -m gpu -x -q -k "two_level or full_size or edge or launch" > gpurun_out/pytest_pv4.txt 2>&1
+timeout 600 python -m pytest tests -m gpu -x -q -k "two_level or edge" > gpurun_out/pytest_pv8.txt 2>&1
+bash tools/sweep.sh "pv8:DC_SEL4_PV=8 pv4:DC_SEL4_PV=4" sort_u32 > gpurun_out/sweep_pv.txt 2>&1
+bash tools/sweep.sh "pv8:DC_SEL4_PV=8 pv4:DC_SEL4_PV=4" sort_kv >> gpurun_out/sweep_pv.txt 2>&1
