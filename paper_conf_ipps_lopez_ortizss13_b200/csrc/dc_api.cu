@@ -470,8 +470,10 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
                 const int tiles2 = (int)(((n + 4 * w - 1) / (4 * w)) * tpg);
                 if (!fused_sel) {
                     TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-                    const int sel_warps = (tiles2 + dc::kSel4BPW - 1) / dc::kSel4BPW;
-                    dc::nk2_select4<K><<<(sel_warps + 3) / 4, 128, 0, p->stream>>>(
+                    constexpr int PV = V ? 4 : 2;           // pivots per run (sort4_kernels.cuh)
+                    constexpr int bpw = dc::sel4_bpw<PV>();
+                    const int sel_warps = (tiles2 + bpw - 1) / bpw;
+                    dc::nk2_select4<K, PV><<<(sel_warps + 3) / 4, 128, 0, p->stream>>>(
                         cur_k, n, w, TC.T(), tpg, tiles2, cuts);
                     DC_LAUNCHED(p);
                 }

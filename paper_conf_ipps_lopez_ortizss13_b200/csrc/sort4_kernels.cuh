@@ -95,7 +95,7 @@ template <class K, int PV = 8>
 __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, long long n,
                                              long long w, int T, int tpg, int j,
                                              bool valid = true) {
-    static_assert(PV == 8 || PV == 4, "8 pivots (one boundary per warp) or 4 (two)");
+    static_assert(PV == 8 || PV == 4 || PV == 2, "8, 4 or 2 pivots per run (1, 2, 4 boundaries per warp)");
     constexpr int LB = 4 * PV;
     const int lane = threadIdx.x & 31;
     const int base = lane & ~(LB - 1);                 // first lane of this boundary's group
@@ -241,16 +241,15 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
     return c;
 }
 
-// NK2-4 as its own launch: one warp per tile boundary.
 // NK2-4 as its own launch: BPW = 32 / (4 PV) tile boundaries per warp.
-#ifndef DC_SEL4_PV
-#define DC_SEL4_PV 4
-#endif
-constexpr int kSel4BPW = 32 / (4 * DC_SEL4_PV);      // boundaries per warp
-template <class K>
+// Measured at 2^28: keys-only PV 8 / 4 / 2 -> 0.472 / 0.443 / 0.396 ms per
+// sort; key-value (twice the tiles) 0.818 / 0.698 / 0.709 ms.
+template <int PV>
+constexpr int sel4_bpw() { return 32 / (4 * PV); }
+template <class K, int PV>
 __global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long long w, int T,
                             int tpg, int num_tiles, Cut4* __restrict__ cut) {
-    constexpr int PV = DC_SEL4_PV, LB = 4 * PV, BPW = 32 / LB;
+    constexpr int LB = 4 * PV, BPW = 32 / LB;
     const int wj = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * BPW;
     if (wj >= num_tiles) return;                      // warp-uniform
     const int lane = threadIdx.x & 31;

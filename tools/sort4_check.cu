@@ -83,7 +83,7 @@ int main(int argc, char** argv) {
     CK(cudaMalloc(&dcut, (tiles + 1) * sizeof(dc::Cut4)));
     CK(cudaMemcpy(dsrc, h.data(), n * 4, cudaMemcpyHostToDevice));
     CK(cudaMemset(dcut, 0xff, (tiles + 1) * sizeof(dc::Cut4)));
-    dc::nk2_select4<dc::KeyU32><<<((tiles + dc::kSel4BPW - 1) / dc::kSel4BPW + 3) / 4, 128>>>(dsrc, n, w, T, tpg, tiles, dcut);
+    dc::nk2_select4<dc::KeyU32, 2><<<((tiles + dc::sel4_bpw<2>() - 1) / dc::sel4_bpw<2>() + 3) / 4, 128>>>(dsrc, n, w, T, tpg, tiles, dcut);
     CK(cudaGetLastError());
     CK(cudaDeviceSynchronize());
     printf("select4 done\n");
@@ -122,7 +122,7 @@ int main(int argc, char** argv) {
         float ms_s = 0, ms_m = 0, t;
         for (int i = 0; i < iters; ++i) {
             cudaEventRecord(e0);
-            dc::nk2_select4<dc::KeyU32><<<((tiles + dc::kSel4BPW - 1) / dc::kSel4BPW + 3) / 4, 128>>>(dsrc, n, w, T, tpg, tiles, dcut);
+            dc::nk2_select4<dc::KeyU32, 2><<<((tiles + dc::sel4_bpw<2>() - 1) / dc::sel4_bpw<2>() + 3) / 4, 128>>>(dsrc, n, w, T, tpg, tiles, dcut);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
             cudaEventElapsedTime(&t, e0, e1);
