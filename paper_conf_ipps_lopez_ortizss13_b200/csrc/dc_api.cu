@@ -30,15 +30,17 @@ namespace {
 
 // ---------------------------------------------------------------- config
 // Sort configuration per instantiation (tuned on B200 with tools/sweep.sh,
-// see DESIGN.md Sec. 5).  Keys-only u32/i32 (stability unobservable): 512
-// threads x 51 items = tiles of 26112 keys (9 shared-memory merge levels on
-// top of a 51-input register network; 14 global levels at 2^28), one-level
-// merge CTAs of 256 x 51 = 13056 outputs.  (1024 x 51 tiles save a global
-// level at 2^28 but cost more in NK1 than they save: 6.38 vs 6.19 ms.)
-// Stable variants (values, or f32 keys whose +0/-0 must keep their order)
-// carry a tile-local index: 512 x 33 = 16896-key tiles, merge CTAs of 256 x 33
-// outputs.  Merge tiles need not divide a pair: every pair is cut into
-// ceil(2w / tout) tiles, the last one short.
+// see DESIGN.md Sec. 5).  Keys-only u32/i32 (stability unobservable): NK1 of
+// 512 threads x 49 items = tiles of 25088 keys (9 shared-memory merge levels
+// on top of a 49-input register network; 14 global levels at 2^28), one-level
+// merge CTAs of 256 x 51 = 13056 outputs.  49 rather than 51 items: a group of
+// four 25088-key runs splits into four 4-way tiles of <= 25344 keys, where four
+// 26112-key runs need a fifth 3072-key sliver tile (2^28: 6.08 -> 5.96 ms).
+// (1024 x 51 tiles save a global level at 2^28 but cost more in NK1 than they
+// save: 6.38 vs 6.19 ms.)  f32 keys carry a tile-local index for stability:
+// 512 x 33 = 16896-key tiles, merge CTAs of 256 x 33 outputs; key-value
+// NK1 uses 256-thread CTAs (kCfgKV).  Merge tiles need not divide a pair:
+// every pair is cut into ceil(2w / tout) tiles, the last one short.
 struct SortCfg {
     int nt1, it1, nt3, it;   // NK1 threads x items, one-level merge threads x items
     constexpr int tile() const { return nt1 * it1; }
@@ -48,7 +50,7 @@ struct SortCfg {
 #define DC_FAST_NT1 512
 #endif
 #ifndef DC_FAST_IT1
-#define DC_FAST_IT1 51
+#define DC_FAST_IT1 49
 #endif
 #ifndef DC_FAST_IT
 #define DC_FAST_IT 51

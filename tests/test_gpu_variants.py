@@ -3,7 +3,7 @@
 The one-level merge pass cuts every pair of runs (width 2w) into
 ceil(2w / tout) output tiles, the last one short (PairGeom.tile_of).  With the
 default shapes tout divides 2w; this builds the library with 160-thread merge
-CTAs (tout = 160 x 51 = 8160, 2 x 26112 / 8160 = 6.4) and checks the one-level
+CTAs (tout = 160 x 51 = 8160, 2 x 25088 / 8160 = 6.1) and checks the one-level
 schedule bit-exactly against the oracle in a subprocess bound to that build.
 """
 import os
@@ -26,9 +26,9 @@ import dcgen, oracle
 import paper_conf_ipps_lopez_ortizss13_b200 as dc
 oracle.build()
 sch = dc.Plan(1 << 23).schedule("u32")
-assert sch["tile"] == 26112, sch
+assert sch["tile"] == 25088, sch
 for n, dist, kt, vals in [((1 << 23) + 12345, "uniform", "u32", False),
-                          (2 * 26112 * 5 + 7, "few", "u32", False),
+                          (2 * 25088 * 5 + 7, "few", "u32", False),
                           ((1 << 23) + 99, "uniform", "i32", False),
                           ((1 << 23) + 5, "few", "u32", True)]:
     keys = dcgen.sort_keys(n, dist, seed=41, key_type=kt, device="cuda")

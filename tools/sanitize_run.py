@@ -41,7 +41,7 @@ def main():
         check_sort(n, "f32", vals=True)
         check_sort(n, vals=True)
     if large:   # the large-tile config (>= 2^23 keys) incl. two-level passes
-        n = (1 << 23) + 26112 + 3
+        n = (1 << 23) + 25088 + 3
         check_sort(n)
         check_sort(n, vals=True)
         keys = dcgen.sort_keys(n, "uniform", seed=6, device="cuda")
