@@ -76,7 +76,10 @@ constexpr SortCfg kCfgStable{DC_STABLE_NT1, DC_STABLE_IT, DC_STABLE_NT3, DC_STAB
 #ifndef DC_KV_NT1
 #define DC_KV_NT1 256
 #endif
-constexpr SortCfg kCfgKV{DC_KV_NT1, DC_STABLE_IT, DC_STABLE_NT3, DC_STABLE_IT};
+#ifndef DC_KV_IT1
+#define DC_KV_IT1 DC_STABLE_IT
+#endif
+constexpr SortCfg kCfgKV{DC_KV_NT1, DC_KV_IT1, DC_STABLE_NT3, DC_STABLE_IT};
 // Small inputs (n < kSmallN, L2-resident): quarter-size tiles so that the
 // fused kernel and every merge level still launch >= ~150 CTAs.
 #ifndef DC_SMALL_NT1
