@@ -426,7 +426,7 @@ def e2e_sort(args, plan, n, kv, pristine_k, pristine_v):
             "h2d_bytes_per_step": n * 4 * (2 if kv else 1),
             "d2h_bytes_per_step": n * 4 * (2 if kv else 1),
             "mode": "streamed host sorts, 3 device slots, copies overlapped across steps",
-            "copy_bound": "tools/pcie_probe.py on the B200 box: pinned 1 GiB H2D 54 GB/s, D2H 57 GB/s alone, 49 GB/s each way concurrent = 21.9 ms per GiB in + GiB out"}
+            "copy_bound": "tools/pcie_probe.py (profiles/r01/pcie_probe.json): pinned 1 GiB H2D ~55 GB/s, D2H ~57 GB/s alone, 45-50 GB/s each way concurrent (varies by box) = 21.5-23.5 ms per GiB in + GiB out"}
 
 
 def run_dc_maxsub(args, wl, desc, n):
