@@ -575,7 +575,11 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
 #ifndef DC_MS_J
 #define DC_MS_J 2
 #endif
+#ifndef DC_MS_VONLY       // values-only element fold + chunk-index recovery (measured slower)
+#define DC_MS_VONLY 0
+#endif
 constexpr int kMsP = DC_MS_P, kMsS = DC_MS_S, kMsTNT = DC_MS_TNT, kMsJ = DC_MS_J;
+constexpr bool kMsVO = DC_MS_VONLY != 0;
 constexpr int ms_tma_smem() { return kMsS * kMsTNT * kMsP * 4; }   // S x NW x 32*L words
 
 // Max-subarray grid: about one wave of resident CTAs (occupancy x SMs),
@@ -587,7 +591,7 @@ int ms_grid(dc_plan_t p) {
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (DC_MS_TMA) {
-            auto* k = dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ>;
+            auto* k = dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ, kMsVO>;
             cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, ms_tma_smem());
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kMsTNT, ms_tma_smem());
         } else {
@@ -627,7 +631,7 @@ dc_status maxsub_launch(dc_plan_t p, const int32_t* d_x, int64_t off, int mode,
         // warp ranges of RW elements, a multiple of the 32*L-element segment
         const int64_t warps = (int64_t)grid * (kMsTNT / 32), seg = 32LL * kMsP;
         const int64_t R = ((p->n + warps - 1) / warps + seg - 1) / seg * seg;
-        dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ><<<grid, kMsTNT, ms_tma_smem(), p->stream>>>(
+        dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ, kMsVO><<<grid, kMsTNT, ms_tma_smem(), p->stream>>>(
             d_x, p->n, R, p->ms_tiles, p->ms_ticket, off, mode, out_res, out_tup);
     } else {
         dc::nk4_maxsub<kNK4Threads, kNK4Chunk><<<grid, kNK4Threads, 0, p->stream>>>(

@@ -13,6 +13,15 @@
 // bank-conflict free) as J interleaved chains, and an ordered FP64 warp tree
 // folds the 32 lane summaries into the warp's running summary.  Warps, then
 // CTAs (atomic ticket, last CTA), are combined in order as before.
+//
+// VO (values-only, opt-in -DDC_MS_VONLY=1; measured slower): the per-element fold keeps only the four
+// values (tot, pre, suf, best: two DADDs and three max) and no indices; each
+// lane's L-element chunk then enters the ordered combine as one leaf labelled
+// by its chunk start.  The combine's tie rules pick the lexicographically
+// smallest (start chunk, end chunk) pair, and that pair holds the
+// lexicographically smallest optimal (start, end) (reading R21), so
+// the last CTA recovers the exact element indices by re-scanning at most
+// four chunks (ms_recover).
 #pragma once
 #include <cstdint>
 
@@ -45,7 +54,80 @@ __device__ __forceinline__ MsFold ms_fold_warp(MsFold t) {
     return t;
 }
 
-template <int NT, int L, int S, int J>
+// Values-only fold of one chunk (no indices).  Same FP64 exactness argument
+// as MsFold; fmax reproduces the strict/tie rules' values (only the indices
+// depend on ties, and those are recovered separately).
+struct MsVal {
+    double tot, pre, suf, best;
+    __device__ __forceinline__ void init() {
+        tot = 0.0; pre = (double)kMsNeg; suf = (double)kMsNeg; best = (double)kMsNeg;
+    }
+    __device__ __forceinline__ void step(int x) {
+        const double xd = (double)x;
+        tot += xd;
+        pre = fmax(pre, tot);
+        suf = fmax(suf, 0.0) + xd;
+        best = fmax(best, suf);
+    }
+    __device__ __forceinline__ void absorb(const MsVal& R) {   // R right of this
+        best = fmax(best, fmax(suf + R.pre, R.best));
+        pre = fmax(pre, tot + R.pre);
+        suf = fmax(R.tot + suf, R.suf);
+        tot += R.tot;
+    }
+};
+
+// Chunk [c, min(c+L, n)): smallest e maximising sum(x[c..e]) (the prefix end).
+template <int L>
+__device__ long long ms_first_max_prefix(const int* __restrict__ x, long long n, long long c) {
+    const long long e1 = min(n, c + L);
+    long long P = 0, m = kMsNeg, k = c;
+    for (long long j = c; j < e1; ++j) {
+        P += x[j];
+        if (P > m) { m = P; k = j; }
+    }
+    return k;
+}
+// Chunk [c, e1): smallest s maximising sum(x[s..e1-1]) (the suffix start).
+template <int L>
+__device__ long long ms_first_max_suffix(const int* __restrict__ x, long long n, long long c) {
+    const long long e1 = min(n, c + L);
+    long long P = 0, m = 0, k = c;
+    for (long long j = c; j + 1 < e1; ++j) {
+        P += x[j];
+        if (P < m) { m = P; k = j + 1; }
+    }
+    return k;
+}
+
+// Exact indices from chunk labels (warp 0 of the last CTA; lanes 0..3 scan
+// one chunk each).  a's pe/ss/bs/be are chunk starts; on return they are
+// element indices.  pe: first prefix maximum inside its chunk; ss: first
+// suffix maximum inside its chunk; best: the in-chunk Kadane when start and
+// end chunk coincide, else the suffix-start / prefix-end scans of the two.
+template <int L>
+__device__ void ms_recover(const int* __restrict__ x, long long n, MsTupG& a, long long* rec) {
+    const int lane = threadIdx.x & 31;
+    if (lane == 0) rec[0] = ms_first_max_prefix<L>(x, n, a.pe);
+    if (lane == 1) rec[1] = ms_first_max_suffix<L>(x, n, a.ss);
+    if (lane == 2) {
+        if (a.bs == a.be) {
+            MsFold f;
+            f.init();
+            const long long e1 = min(n, a.bs + L);
+            for (long long j = a.bs; j < e1; ++j) f.step(x[j], (int)(j - a.bs));
+            rec[2] = a.bs + f.bs;
+            rec[3] = a.bs + f.be;
+        } else {
+            rec[2] = ms_first_max_suffix<L>(x, n, a.bs);
+        }
+    }
+    if (lane == 3 && a.bs != a.be) rec[3] = ms_first_max_prefix<L>(x, n, a.be);
+    __syncwarp();
+    a.pe = rec[0]; a.ss = rec[1]; a.bs = rec[2]; a.be = rec[3];
+}
+
+template <int NT, int L, int S, int J, bool VO>
 __global__ void __launch_bounds__(NT, 1)
 nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
                dc_maxsub_tuple* __restrict__ parts, unsigned int* __restrict__ ticket,
@@ -102,7 +184,38 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
         const int i0 = (int)(g0 - cbase) + e0;
         MsFold f;
         f.init();
-        if (cnt == SEG) {
+        if (VO) {
+            MsVal v;
+            v.init();
+            if (cnt == SEG) {
+                MsVal g[J];
+#pragma unroll
+                for (int j = 0; j < J; ++j) g[j].init();
+#pragma unroll
+                for (int q = 0; q < VJ; ++q) {
+#pragma unroll
+                    for (int j = 0; j < J; ++j) {
+                        if (j * VJ + q < V && q < VJ) {
+                            const int4 w = *reinterpret_cast<const int4*>(sl + 4 * (j * VJ + q));
+                            g[j].step(w.x);
+                            g[j].step(w.y);
+                            g[j].step(w.z);
+                            g[j].step(w.w);
+                        }
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < J; ++j) v.absorb(g[j]);
+            } else {
+                const int body = cnt & ~3;
+                for (int e = e0; e < min(cnt, e0 + L); ++e)
+                    v.step(e < body ? sl[e - e0] : x[g0 + e]);
+            }
+            // one leaf per lane chunk, labelled by its start (an empty chunk
+            // keeps the identity's sentinels and is absorbed without effect)
+            f.tot = v.tot; f.pre = v.pre; f.suf = v.suf; f.best = v.best;
+            f.pe = f.ss = f.bs = f.be = i0;
+        } else if (cnt == SEG) {
             MsFold g[J];
 #pragma unroll
             for (int j = 0; j < J; ++j) g[j].init();
@@ -156,6 +269,16 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
     MsTupG a = ms_empty<long long>();
     for (int q = tid * per; q < min(np, tid * per + per); ++q) a = ms_combine(a, ms_load_cg(parts + q));
     a = ms_block_combine<NT>(a, redg);
+    if (VO) {
+        __shared__ MsTupG s_a;
+        __shared__ long long rec[4];
+        if (tid == 0) s_a = a;
+        __syncthreads();
+        if (warp == 0) {
+            a = s_a;
+            ms_recover<L>(x, n, a, rec);
+        }
+    }
     if (tid == 0) {
         if (mode == 0) {
             out_res->sum = a.best;

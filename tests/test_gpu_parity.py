@@ -417,6 +417,35 @@ def test_maxsub_tuple_and_combine(dc, oracle_mod):
     assert tuple(out.cpu().tolist()) == oracle_mod.maxsub(x.cpu().numpy())
 
 
+@pytest.mark.parametrize("n", [67, 68, 69, 2176, 2177, 70_001, 1 << 20])
+@pytest.mark.parametrize("lo", [-1, -2])
+def test_maxsub_tie_heavy(dc, oracle_mod, n, lo):
+    # values in {lo..1}: many equal maxima, equal prefix/suffix maxima across
+    # lane-chunk (68) and segment (32*68) boundaries; exercises the chunk-label
+    # recovery of the values-only fold (R13)
+    g = torch.Generator().manual_seed(n * 7 + lo)
+    x = torch.randint(lo, 2, (n,), generator=g, dtype=torch.int32)
+    assert dc.Plan(n).max_subarray(x.cuda()) == oracle_mod.maxsub(x.numpy())
+
+
+@pytest.mark.parametrize("n", [1, 68, 69, 4353, 1 << 20])
+def test_maxsub_tuple_prefix_suffix(dc, n):
+    # whole-array summary: pe = first argmax of the prefix sums, ss = first
+    # argmax of the suffix sums, tot = the total (numpy brute force)
+    g = torch.Generator().manual_seed(n)
+    x = torch.randint(-3, 3, (n,), generator=g, dtype=torch.int32)
+    tup = torch.empty(8, dtype=torch.int64, device="cuda")
+    off = 1000
+    dc.Plan(n).max_subarray_tuple_async(x.cuda(), tup, index_offset=off)
+    t = tup.cpu().tolist()
+    a = x.numpy().astype(np.int64)
+    pre = np.cumsum(a)
+    suf = np.cumsum(a[::-1])[::-1]
+    assert t[0] == int(a.sum())
+    assert (t[1], t[4]) == (int(pre.max()), int(np.argmax(pre)) + off)
+    assert (t[2], t[5]) == (int(suf.max()), int(np.argmax(suf)) + off)
+
+
 def test_maxsub_host_buffer(dc, oracle_mod):
     n = 300_000
     x = dcgen.maxsub_input(n, "small", seed=6).pin_memory()

@@ -104,3 +104,51 @@ def test_two_level_fused_selection(tmp_path):
                        capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     assert "variant ok" in r.stdout
+
+
+VONLY_SCRIPT = r"""
+import sys
+import numpy as np
+import torch
+sys.path.insert(0, {root!r})
+import dcgen, oracle
+import paper_conf_ipps_lopez_ortizss13_b200 as dc
+oracle.build()
+cases = []
+for n in [1, 67, 68, 69, 2176, 2177, 70_001, 1 << 20, (1 << 24) + 3]:
+    for lo in (-1, -2):
+        g = torch.Generator().manual_seed(n * 7 + lo)
+        cases.append(torch.randint(lo, 2, (n,), generator=g, dtype=torch.int32))
+for n, dist in [(1 << 24, "uniform"), ((1 << 20) + 5, "small"), (777, "negative"),
+                (1 << 16, "zero"), (100_003, "positive")]:
+    cases.append(dcgen.maxsub_input(n, dist, seed=2))
+for x in cases:
+    n = x.numel()
+    assert dc.Plan(n).max_subarray(x.cuda()) == oracle.maxsub(x.numpy()), n
+    tup = torch.empty(8, dtype=torch.int64, device="cuda")
+    dc.Plan(n).max_subarray_tuple_async(x.cuda(), tup, index_offset=5)
+    t = tup.cpu().tolist()
+    a = x.numpy().astype(np.int64)
+    pre = np.cumsum(a)
+    suf = np.cumsum(a[::-1])[::-1]
+    s, b, e = oracle.maxsub(x.numpy())
+    assert t == [int(a.sum()), int(pre.max()), int(suf.max()), s,
+                 int(np.argmax(pre)) + 5, int(np.argmax(suf)) + 5, b + 5, e + 5], (n, t)
+print("variant ok")
+"""
+
+
+def test_maxsub_values_only_fold(tmp_path):
+    """NK4 with the values-only element fold and chunk-label index recovery
+    (-DDC_MS_VONLY=1, R21): bit-exact (sum, start, end) and summary
+    tuple on tie-heavy and degenerate inputs."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_lopez_ortizss13_b200 import build
+
+    lib = build.build(out=str(tmp_path / "libdc_vonly.so"), defines=["DC_MS_VONLY=1"])
+    env = dict(os.environ, DC_LIB=lib)
+    r = subprocess.run([sys.executable, "-c", VONLY_SCRIPT.format(root=ROOT)], env=env,
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert "variant ok" in r.stdout
