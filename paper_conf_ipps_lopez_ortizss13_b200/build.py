@@ -6,6 +6,7 @@ repo snapshot to the GPU box (it is git-ignored, not gpurun-ignored).
 """
 from __future__ import annotations
 
+import fcntl
 import glob
 import os
 import subprocess
@@ -44,6 +45,16 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None,
     target = out or LIB
     if out is None and not force and not _stale():
         return LIB
+    # one builder at a time per target (spawned ranks of a test may all find the
+    # library stale); the others wait and re-check instead of rebuilding
+    with open(target + ".lock", "w") as lk:
+        fcntl.flock(lk, fcntl.LOCK_EX)
+        if out is None and not force and not _stale():
+            return LIB
+        return _compile(target, verbose, defines)
+
+
+def _compile(target: str, verbose: bool, defines: list[str] | None) -> str:
     nvcc = os.environ.get("NVCC", "nvcc")
     tmp = target + ".tmp%d" % os.getpid()
     cmd = [nvcc, *NVCC_FLAGS, "-I", INCLUDE, "-I", CSRC, "-o", tmp,
