@@ -14,8 +14,9 @@ keys on one B200 -- the configuration the metric "sorted keys/sec (32-bit,
 the cross-GPU top-level merge (see paper_conf_ipps_lopez_ortizss13_b200/dist.py).
 
 Timing: inputs resident in HBM; before every step (untimed) the keys are
-restored from a pristine device copy and L2 is flushed by writing a 512 MiB
-buffer; each step is bracketed by CUDA events on the launching stream; W
+restored from a pristine device copy and L2 is flushed by READING a 512 MiB
+buffer (a read leaves L2 full of clean lines, so the timed kernels do not pay
+for write-backs of a dirty flush buffer); each step is bracketed by CUDA events on the launching stream; W
 warm-up steps, then exactly K timed steps between barrier + synchronize.
 Per-kernel device times come from the library's own event instrumentation
 (dc_plan_kernel_time) over the same timed steps.
@@ -68,6 +69,24 @@ def peaks():
         return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:
         return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class L2Flush:
+    """Evicts L2 (126 MB) by reading a 512 MiB buffer (sum into a scalar).
+    The buffer is written once at setup; every flush is a pure read, so L2
+    is left holding clean lines and the next kernel's misses cost no
+    write-backs (a write-based flush dirtied L2 and taxed every small-n line)."""
+
+    def __init__(self, dev, mib: int = 512):
+        import torch
+
+        self.buf = torch.ones((mib << 20) // 8, dtype=torch.int64, device=dev)
+        self.out = torch.empty((), dtype=torch.int64, device=dev)
+
+    def __call__(self):
+        import torch
+
+        torch.sum(self.buf, dtype=torch.int64, out=self.out)
 
 
 def ncu_traffic(kernel: str, workload: str):
@@ -157,14 +176,18 @@ def cpu_info():
 # --------------------------------------------------------- oracle timings
 
 def oracle_sort_sample(n_total: int, dist: str, kv: bool, budget_s: float = 12.0,
-                       sample_n: int = 1 << 24):
-    """The oracle (Alg 6, 1 thread) on prefixes of the workload, as it stands."""
+                       sample_n: int | None = None):
+    """The oracle (Alg 6, 1 thread) on the workload, as it stands.  By default
+    on the FULL input (sample_n = n_total: one run, ~30 s at 2^28 on the box's
+    host) so the CPU rate is the rate at the config size (mergesort's per-key
+    rate falls with log n); a smaller sample_n times prefixes, repeated for
+    budget_s."""
     import numpy as np
 
     import dcgen
     import oracle
 
-    sample_n = min(sample_n, n_total)
+    sample_n = n_total if sample_n is None else min(sample_n, n_total)
     keys = dcgen.sort_keys(n_total, dist, seed=3, start=0, count=sample_n).numpy().view(np.uint32)
     vals = np.arange(sample_n, dtype=np.uint32) if kv else None
     reps, t0 = 0, time.perf_counter()
@@ -220,7 +243,16 @@ def run_reference(args, wl):
         import dcgen
         import oracle
 
-        sample_n = 1 << 22
+        # Largest power-of-two prefix whose (W + K) one-thread sorts fit in
+        # about three minutes, from a 2^20 calibration run (the full 2^28 takes
+        # ~30 s per step on the box's host, too long for K = 10).
+        cal = dcgen.sort_keys(n, args.dist, seed=3, count=1 << 20).numpy().view(np.uint32)
+        t0 = time.perf_counter()
+        oracle.mergesort(cal)
+        per_key = (time.perf_counter() - t0) / (1 << 20) * 1.15   # log n growth to 2^26
+        sample_n = 1 << 20
+        while sample_n * 2 <= n and (args.warmup + args.steps) * per_key * sample_n * 2 <= 180.0:
+            sample_n *= 2
         keys = dcgen.sort_keys(n, args.dist, seed=3, count=sample_n).numpy().view(np.uint32)
         vals = np.arange(sample_n, dtype=np.uint32) if kind == "sort_kv" else None
         for i in range(args.warmup + args.steps):
@@ -229,8 +261,9 @@ def run_reference(args, wl):
             if i >= args.warmup:
                 step_times.append(time.perf_counter() - t0)
         unit = "keys/s"
-        sample = (f"oracle Alg 6 recursive mergesort (1 thread) of the first 2^22 keys of the "
-                  f"{desc} workload, per step")
+        sample = (f"oracle Alg 6 recursive mergesort (1 thread) of the first 2^"
+                  f"{sample_n.bit_length() - 1} keys of the {desc} workload, per step (the "
+                  f"largest power-of-two prefix whose {args.warmup + args.steps} steps fit ~3 min)")
     t = statistics.mean(step_times)
     v = sample_n / t
     print(json.dumps({
@@ -275,7 +308,7 @@ def run_dc(args, wl):
     keys = torch.empty_like(pristine_k)
     vals = torch.empty_like(pristine_k) if kv else None
     pristine_v = dcgen.sort_vals(n, device=dev) if kv else None
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    flush = L2Flush(dev)
     plan = dc.Plan(n)
     stream = torch.cuda.current_stream(dev)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -285,7 +318,7 @@ def run_dc(args, wl):
         keys.copy_(pristine_k)
         if kv:
             vals.copy_(pristine_v)
-        flush.zero_()
+        flush()
 
     for i in range(args.warmup):
         prep()
@@ -374,8 +407,10 @@ def run_dc(args, wl):
         v, reps, sn, el = oracle_sort_sample(n, args.dist, kv)
         model, cores = cpu_info()
         cpu = {"value": v, "unit": "keys/s", "cores": 1, "kind": "oracle",
-               "sample": f"oracle Alg 6 recursive mergesort, 1 thread, {reps} x the first {sn} "
-                         f"keys of this workload ({el:.1f} s)",
+               "sample": (f"oracle Alg 6 recursive mergesort, 1 thread, the full {sn}-key input "
+                          f"of this workload ({el:.1f} s)" if sn == n else
+                          f"oracle Alg 6 recursive mergesort, 1 thread, {reps} x the first {sn} "
+                          f"keys of this workload ({el:.1f} s)"),
                "cpu": model, "host_cores": cores}
 
     print(json.dumps({
@@ -386,7 +421,7 @@ def run_dc(args, wl):
                    "key_type": "u32", "values": kv, "tile": sched["tile"],
                    "fused_levels": sched["fused_levels"], "global_passes": sched["global_passes"],
                    "hbm_passes": sched["hbm_passes"],
-                   "l2": "flushed before every step (512 MiB write); input "
+                   "l2": "flushed before every step (512 MiB read); input "
                          + (f"{n * (8 if kv else 4) / 2**30:.0f} GiB > L2" if n * 4 > (126 << 20)
                             else f"{n * (8 if kv else 4) / 2**20:.0f} MiB, L2-resident after the first level"),
                    "step_ms_min": min(step_ms), "step_ms_max": max(step_ms),
@@ -439,13 +474,13 @@ def run_dc_maxsub(args, wl, desc, n):
     x = dcgen.maxsub_input(n, args.dist if args.dist != "uniform" else "uniform", seed=2,
                            device=dev)
     out = torch.empty(3, dtype=torch.int64, device=dev)
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    flush = L2Flush(dev)
     plan = dc.Plan(n)
     stream = torch.cuda.current_stream(dev)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.warmup + args.steps)]
     for i in range(args.warmup):
-        flush.zero_()
+        flush()
         ev[i][0].record(stream)
         plan.max_subarray_async(x, out)
         ev[i][1].record(stream)
@@ -454,7 +489,7 @@ def run_dc_maxsub(args, wl, desc, n):
     l0 = plan.launch_count()
     with ClockSampler(dev.index) as clk:
         for i in range(args.warmup, args.warmup + args.steps):
-            flush.zero_()
+            flush()
             ev[i][0].record(stream)
             plan.max_subarray_async(x, out)
             ev[i][1].record(stream)
@@ -491,7 +526,7 @@ def run_dc_maxsub(args, wl, desc, n):
         "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "i32->i64", "data": "synthetic (counter-based splitmix64)",
         "config": {"workload": wl, "description": desc, "n": n, "dist": args.dist,
-                   "l2": "flushed before every step (512 MiB write)"},
+                   "l2": "flushed before every step (512 MiB read)"},
         "roofline": {"kernel": "nk4_maxsub (tiles + last-CTA top combine)", "bound": "hbm",
                      "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
                      "traffic": ncu_traffic("nk4_maxsub", wl), "avg_launch_ms": avg,
@@ -513,14 +548,14 @@ def run_dc_sum(args, wl, desc, n):
     dev = torch.device("cuda", torch.cuda.current_device())
     x = dcgen.maxsub_input(n, "uniform", seed=2, device=dev)
     out = torch.empty(1, dtype=torch.int64, device=dev)
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    flush = L2Flush(dev)
     plan = dc.Plan(n)
     stream = torch.cuda.current_stream(dev)
     times = []
     l0 = None
     with ClockSampler(dev.index) as clk:
         for i in range(args.warmup + args.steps):
-            flush.zero_()
+            flush()
             if i == args.warmup:
                 l0 = plan.launch_count()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -540,7 +575,7 @@ def run_dc_sum(args, wl, desc, n):
         "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": "i32->i64", "data": "synthetic (counter-based splitmix64)",
         "config": {"workload": wl, "description": desc, "n": n,
-                   "l2": "flushed before every step (512 MiB write)"},
+                   "l2": "flushed before every step (512 MiB read)"},
         "roofline": {"kernel": "breadth_first_reduce<SumI64> (one launch = the step)",
                      "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s",
                      "frac": ach / peak, "traffic": ncu_traffic("breadth_first_reduce", wl),

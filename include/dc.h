@@ -168,7 +168,9 @@ dc_status dc_run_mergesort_host(dc_plan_t plan, dc_key_type key_type, void *h_ke
  * host input is not modified.  Work of consecutive submissions overlaps: the
  * upload of one, the sort of the previous and the download of the one before
  * run on separate streams (PCIe is full duplex).  A submission starts after
- * the work already enqueued on the plan stream.  Returns after enqueueing;
+ * the work already enqueued on the plan stream, and every later run of the
+ * plan that uses its scratch (dc_run_mergesort, dc_mg_merge_*) is ordered on
+ * the plan stream after the submitted sorts.  Returns after enqueueing;
  * the host buffers must stay valid until dc_sort_host_wait returns. */
 dc_status dc_sort_host_submit(dc_plan_t plan, dc_key_type key_type, const void *h_in_keys,
                               const uint32_t *h_in_vals, void *h_out_keys, uint32_t *h_out_vals);
@@ -330,7 +332,9 @@ dc_status dc_plan_last_splits(dc_plan_t plan, int64_t *h_cmat);
 
 /* Words of one rank's splitter send buffer for `world` ranks and windows of
  * wcap keys: 6*(world-1) header words (three int64 per boundary) followed by
- * (world-1)*wcap key words.  0 if world < 2. */
+ * (world-1)*wcap key words, rounded up to a multiple of 4 words so that
+ * back-to-back buffers of all ranks stay 16-byte aligned for any wcap.
+ * 0 if world < 2. */
 int64_t dc_mg_sendbuf_words(int32_t world, int64_t wcap);
 
 /* Samples of a sorted shard: d_samples[j] = d_keys[j*stride] for

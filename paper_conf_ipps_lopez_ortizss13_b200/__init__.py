@@ -195,13 +195,35 @@ def _key_type(t: torch.Tensor, key_type: str | None) -> int:
     raise TypeError(f"unsupported key dtype {t.dtype}")
 
 
-def _require_cuda(t: torch.Tensor, what: str) -> None:
+def _require_cuda(t: torch.Tensor, what: str, numel: int | None = None) -> None:
     if not t.is_cuda:
         raise ValueError(f"{what} must be a CUDA tensor (no CPU fallback)")
     if not t.is_contiguous():
         raise ValueError(f"{what} must be contiguous")
     if t.element_size() != 4:
         raise ValueError(f"{what} must have 4-byte elements")
+    if numel is not None and t.numel() != numel:
+        raise ValueError(f"{what} must have {numel} elements, not {t.numel()}")
+
+
+def _require_host(t: torch.Tensor, what: str, numel: int) -> None:
+    """Host buffers the C side copies n*4 bytes into / out of."""
+    if t.is_cuda:
+        raise ValueError(f"{what} must be a host tensor")
+    if not t.is_contiguous():
+        raise ValueError(f"{what} must be contiguous")
+    if t.element_size() != 4:
+        raise ValueError(f"{what} must have 4-byte elements")
+    if t.numel() != numel:
+        raise ValueError(f"{what} must have {numel} elements, not {t.numel()}")
+
+
+def _require_out(t: torch.Tensor, what: str, min_numel: int) -> None:
+    """Device int64 result buffers written by the library."""
+    if not t.is_cuda or t.dtype != torch.int64 or not t.is_contiguous():
+        raise ValueError(f"{what} must be a contiguous CUDA int64 tensor")
+    if t.numel() < min_numel:
+        raise ValueError(f"{what} needs at least {min_numel} elements")
 
 
 class Plan:
@@ -357,8 +379,9 @@ class Plan:
     def sort_host_(self, keys: torch.Tensor, vals: torch.Tensor | None = None,
                    key_type: str | None = None) -> torch.Tensor:
         """End-to-end sort of HOST tensors (pinned for full speed): H2D, sort, D2H."""
-        if keys.is_cuda or (vals is not None and vals.is_cuda):
-            raise ValueError("sort_host_ takes host tensors")
+        _require_host(keys, "keys", self.n)
+        if vals is not None:
+            _require_host(vals, "vals", self.n)
         kt = _key_type(keys, key_type)
         _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
         _check(lib().dc_run_mergesort_host(self._h, kt, keys.data_ptr(),
@@ -372,9 +395,12 @@ class Plan:
 
         Consecutive submissions overlap (upload / sort / download on separate
         streams); call :meth:`sort_host_wait` before reading the outputs."""
-        for t in (keys_in, keys_out, vals_in, vals_out):
-            if t is not None and (t.is_cuda or t.numel() != self.n):
-                raise ValueError("host tensors of n elements expected")
+        if (vals_in is None) != (vals_out is None):
+            raise ValueError("vals_in and vals_out: both or neither")
+        for name, t in (("keys_in", keys_in), ("keys_out", keys_out), ("vals_in", vals_in),
+                        ("vals_out", vals_out)):
+            if t is not None:
+                _require_host(t, name, self.n)
         _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
         _check(lib().dc_sort_host_submit(self._h, _key_type(keys_in, key_type),
                                          keys_in.data_ptr(),
@@ -390,9 +416,7 @@ class Plan:
         self._host_refs = []
 
     def max_subarray(self, x: torch.Tensor) -> tuple[int, int, int]:
-        _require_cuda(x, "x")
-        if x.numel() != self.n:
-            raise ValueError("x length != plan n")
+        _require_cuda(x, "x", self.n)
         self._bind_stream(x)
         r = MaxsubResult()
         _check(lib().dc_run_maxsubarray(self._h, x.data_ptr(), ctypes.byref(r)))
@@ -400,14 +424,16 @@ class Plan:
 
     def max_subarray_async(self, x: torch.Tensor, out: torch.Tensor, index_offset: int = 0):
         """Enqueue only; ``out`` is a CUDA int64 tensor of 3 elements (sum, start, end)."""
-        _require_cuda(x, "x")
+        _require_cuda(x, "x", self.n)
+        _require_out(out, "out", 3)
         self._bind_stream(x)
         _check(lib().dc_run_maxsubarray_async(self._h, x.data_ptr(), index_offset, out.data_ptr()))
         return out
 
     def max_subarray_tuple_async(self, x: torch.Tensor, out: torch.Tensor, index_offset: int = 0):
         """Enqueue only; ``out`` is a CUDA int64 tensor of 8 elements (segment summary)."""
-        _require_cuda(x, "x")
+        _require_cuda(x, "x", self.n)
+        _require_out(out, "out", 8)
         self._bind_stream(x)
         _check(lib().dc_run_maxsubarray_tuple_async(self._h, x.data_ptr(), index_offset,
                                                     out.data_ptr()))
@@ -415,6 +441,10 @@ class Plan:
 
     def maxsub_combine_async(self, tuples: torch.Tensor, out: torch.Tensor):
         """Ordered combine of a (count, 8) int64 CUDA tensor of summaries into out[3]."""
+        if tuples.dim() != 2 or tuples.shape[1] != 8 or tuples.shape[0] < 1:
+            raise ValueError("tuples must have shape (count >= 1, 8)")
+        _require_out(tuples, "tuples", 8)
+        _require_out(out, "out", 3)
         self._bind_stream(tuples)
         _check(lib().dc_maxsub_combine_async(self._h, tuples.data_ptr(), tuples.shape[0],
                                              out.data_ptr()))
@@ -422,8 +452,7 @@ class Plan:
 
     def max_subarray_host(self, x: torch.Tensor) -> tuple[int, int, int]:
         """End-to-end max subarray of a HOST int32 tensor."""
-        if x.is_cuda:
-            raise ValueError("max_subarray_host takes a host tensor")
+        _require_host(x, "x", self.n)
         _check(lib().dc_plan_set_stream(self._h, torch.cuda.current_stream().cuda_stream))
         r = MaxsubResult()
         _check(lib().dc_run_maxsubarray_host(self._h, x.data_ptr(), ctypes.byref(r)))
@@ -433,22 +462,22 @@ class Plan:
     # ---------------------------------------------------- D&C sum (f4)
     def sum(self, x: torch.Tensor) -> int:
         """Exact int64 sum of an int32 CUDA tensor (Alg 4 through dc_reduce.cuh)."""
-        _require_cuda(x, "x")
+        _require_cuda(x, "x", self.n)
         self._bind_stream(x)
         r = _I64()
         _check(lib().dc_run_sum(self._h, x.data_ptr(), ctypes.byref(r)))
         return r.value
 
     def sum_async(self, x: torch.Tensor, out: torch.Tensor) -> torch.Tensor:
-        _require_cuda(x, "x")
+        _require_cuda(x, "x", self.n)
+        _require_out(out, "out", 1)
         self._bind_stream(x)
         _check(lib().dc_run_sum_async(self._h, x.data_ptr(), out.data_ptr()))
         return out
 
     def sum_alg5(self, work: torch.Tensor) -> int:
         """Alg 5 literally (one launch per level) on an int64 CUDA work tensor (clobbered)."""
-        if not work.is_cuda or work.dtype != torch.int64:
-            raise ValueError("work must be a CUDA int64 tensor")
+        _require_out(work, "work", self.n)
         self._bind_stream(work)
         r = _I64()
         _check(lib().dc_run_sum_alg5(self._h, work.data_ptr(), ctypes.byref(r)))
@@ -458,6 +487,8 @@ class Plan:
     def mg_sample(self, keys: torch.Tensor, stride: int) -> torch.Tensor:
         """Every stride-th key of this rank's sorted shard (uint32 bits as int32)."""
         _require_cuda(keys, "keys")
+        if stride < 1:
+            raise ValueError("stride must be >= 1")
         out = torch.empty((keys.numel() + stride - 1) // stride, dtype=torch.int32,
                           device=keys.device)
         self._bind_stream(keys)
@@ -467,6 +498,10 @@ class Plan:
     def mg_count(self, keys: torch.Tensor, rank: int, cand: torch.Tensor, per_rank: int,
                  stride: int, key_type: str | None = None) -> torch.Tensor:
         """Composite counts of this rank's elements below every candidate (int64)."""
+        _require_cuda(keys, "keys")
+        _require_cuda(cand, "cand")
+        if cand.numel() < 1 or cand.numel() % per_rank:
+            raise ValueError("cand must hold world * per_rank candidates")
         out = torch.empty(cand.numel(), dtype=torch.int64, device=keys.device)
         self._bind_stream(keys)
         _check(lib().dc_mg_count(self._h, _key_type(keys, key_type), keys.data_ptr(),
@@ -476,6 +511,10 @@ class Plan:
 
     def mg_windows(self, keys: torch.Tensor, rank: int, world: int, counts: torch.Tensor,
                    ranks: torch.Tensor, per_rank: int, wcap: int) -> torch.Tensor:
+        _require_cuda(keys, "keys")
+        if counts.numel() != ranks.numel() or counts.dtype != torch.int64 or \
+                ranks.dtype != torch.int64 or not counts.is_cuda or not ranks.is_cuda:
+            raise ValueError("counts and ranks must be CUDA int64 tensors of equal length")
         words = int(lib().dc_mg_sendbuf_words(world, wcap))
         out = torch.zeros(words, dtype=torch.int32, device=keys.device)
         self._bind_stream(keys)
@@ -486,6 +525,7 @@ class Plan:
 
     def mg_split_matrix(self, gathered: torch.Tensor, world: int, shard_n: int, wcap: int,
                         key_type: str) -> torch.Tensor:
+        _require_cuda(gathered, "gathered", world * int(lib().dc_mg_sendbuf_words(world, wcap)))
         out = torch.empty((world, world + 1), dtype=torch.int64, device=gathered.device)
         self._bind_stream(gathered)
         _check(lib().dc_mg_split_matrix(self._h, _KEY_NAMES[key_type], gathered.data_ptr(),
@@ -503,6 +543,15 @@ class Plan:
         """Stable merge of runs stored in separate buffers: runs = [(keys_buf,
         vals_buf or None, offset, length), ...] (earlier runs win ties)."""
         r = len(runs)
+        _require_cuda(out_keys, "out_keys")
+        if out_vals is not None:
+            _require_cuda(out_vals, "out_vals")
+        for k, v, off, ln in runs:
+            _require_cuda(k, "run keys")
+            if off < 0 or ln < 0 or off + ln > k.numel():
+                raise ValueError("run outside its buffer")
+            if out_vals is not None and (v is None or v.numel() < off + ln):
+                raise ValueError("run values missing or too short")
         kp = (_P * r)(*[t[0].data_ptr() for t in runs])
         vp = (_P * r)(*[t[1].data_ptr() for t in runs]) if out_vals is not None else None
         bound = (_I64 * r)(*[t[0].numel() for t in runs])
@@ -520,6 +569,13 @@ class Plan:
                       out_keys: torch.Tensor, out_vals: torch.Tensor | None, run_len: list[int],
                       key_type: str | None = None) -> torch.Tensor:
         """Stable merge of back-to-back sorted runs (earlier runs win ties)."""
+        total = sum(run_len)
+        for name, t in (("in_keys", in_keys), ("in_vals", in_vals), ("out_keys", out_keys),
+                        ("out_vals", out_vals)):
+            if t is not None:
+                _require_cuda(t, name)
+                if t.numel() < total:
+                    raise ValueError(f"{name} holds fewer than sum(run_len) elements")
         lens = (_I64 * len(run_len))(*run_len)
         self._bind_stream(in_keys)
         _check(lib().dc_mg_merge_runs(self._h, _key_type(in_keys, key_type), in_keys.data_ptr(),

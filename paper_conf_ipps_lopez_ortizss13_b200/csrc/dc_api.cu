@@ -13,6 +13,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <algorithm>
+#include <atomic>
 #include <new>
 #include <string>
 #include <vector>
@@ -272,11 +273,49 @@ struct TimedScope {
 
 bool aligned16(const void* ptr) { return ((uintptr_t)ptr & 15u) == 0; }
 
+// Captured sort graphs embed the plan's scratch / staging / slot pointers, so
+// every reallocation of one of them drops the cache (a graph
+// replayed after a larger run reallocated scratch read freed memory).
+void drop_graphs(dc_plan_t p) {
+    for (auto& gc : p->graphs) {
+        if (gc.exec) cudaGraphExecDestroy(gc.exec);
+        if (gc.graph) cudaGraphDestroy(gc.graph);
+    }
+    p->graphs.clear();
+}
+
+// Per-device, thread-safe one-time setup (kernel attributes, occupancy
+// grids): the dynamic shared-memory attribute and the occupancy are
+// properties of (function, device), so a cache keyed only by the
+// instantiation would skip the attribute on a second GPU of the process.
+constexpr int kMaxDevices = 64;
+int current_device() {
+    int d = 0;
+    cudaGetDevice(&d);
+    return d < 0 ? 0 : (d >= kMaxDevices ? kMaxDevices - 1 : d);
+}
+struct PerDevice {
+    std::atomic<int> v[kMaxDevices];
+    int get() const { return v[current_device()].load(std::memory_order_acquire); }
+    void set(int x) { v[current_device()].store(x, std::memory_order_release); }
+};
+
+// Orders a run on the plan stream after every host-buffer sort submitted
+// before it (those run on p->comp and share the plan scratch).
+dc_status join_host_sorts(dc_plan_t p) {
+    if (p->comp && p->comp_done && p->stream != p->comp) {
+        cudaError_t e = cudaStreamWaitEvent(p->stream, p->comp_done, 0);
+        if (e != cudaSuccess) return cuda_fail(p, e, "cudaStreamWaitEvent(host sorts)");
+    }
+    return DC_OK;
+}
+
 dc_status ensure_scratch(dc_plan_t p, bool vals) {
     size_t need = scratch_needed(p->n, vals);
     if (p->scratch && p->scratch_bytes >= need) return DC_OK;
     if (p->scratch && !p->own_scratch)
         return fail(DC_ERR_INVALID_ARG, "caller scratch too small for this run");
+    drop_graphs(p);
     if (p->scratch) {
         cudaFree(p->scratch);
         p->scratch = nullptr;
@@ -326,8 +365,8 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     auto* k1 = dc::nk1_blocksort<C.nt1, C.it1, K, V>;
     auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
     auto* k3sp = dc::nk3_merge_sp<C.nt3, C.it, K, V>;   // partition fused (SMALL)
-    static bool attr_done = false;   // per key/value instantiation
-    if (!attr_done) {
+    static PerDevice attr_done;   // per instantiation and device
+    if (!attr_done.get()) {
         DC_CUDA(p, cudaFuncSetAttribute(k1, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         nk1_smem_bytes(C, hv)));
         DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -335,7 +374,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         if (SMALL)
             DC_CUDA(p, cudaFuncSetAttribute(k3sp, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                             nk3_smem_bytes(C, hv)));
-        attr_done = true;
+        attr_done.set(1);
     }
 
     // Levels over HBM: P = ceil(log2(ceil(n/tile))).  Keys-only sorts fold
@@ -460,7 +499,8 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
             constexpr bool fused_sel = !K::kNeedStable && TC.nsel > 0;
             constexpr int thr2 = fused_sel ? TC.threads() : TC.nt + 64;
             constexpr int smem2 = dc::m4_smem_bytes(TC.T(), TC.it, V);
-            static int grid2 = 0;                        // per instantiation
+            static PerDevice grid2_dev;                  // per instantiation and device
+            int grid2 = grid2_dev.get();
             if (!grid2) {
                 DC_CUDA(p, cudaFuncSetAttribute(k32, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                 smem2));
@@ -469,6 +509,7 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
                 cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
                 cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, thr2, smem2);
                 grid2 = sms * (occ > 0 ? occ : 1);
+                grid2_dev.set(grid2);
             }
             for (; w < n; w *= 4) {
                 const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), TC.T());
@@ -527,6 +568,8 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
         ok = keys;
         ov = vals;
     }
+    dc_status js = join_host_sorts(p);
+    if (js != DC_OK) return js;
     if (!p->use_graphs || p->timing) return sort_direct(p, kt, keys, vals, ok, ov);
     for (auto& gc : p->graphs) {
         if (gc.keys == keys && gc.vals == vals && gc.out == ok && gc.kt == kt) {
@@ -585,7 +628,8 @@ constexpr int ms_tma_smem() { return kMsS * kMsTNT * kMsP * 4; }   // S x NW x 3
 // Max-subarray grid: about one wave of resident CTAs (occupancy x SMs),
 // never more CTAs than there is work for.
 int ms_grid(dc_plan_t p) {
-    static int grid = 0;
+    static PerDevice grid_dev;
+    int grid = grid_dev.get();
     if (!grid) {
         int dev = 0, sms = 148, occ = 1;
         cudaGetDevice(&dev);
@@ -599,6 +643,7 @@ int ms_grid(dc_plan_t p) {
                 &occ, dc::nk4_maxsub<kNK4Threads, kNK4Chunk>, kNK4Threads, 0);
         }
         grid = sms * (occ > 0 ? occ : 1);
+        grid_dev.set(grid);
     }
     const int64_t units = DC_MS_TMA ? num_tiles(p->n, (int64_t)kMsTNT * kMsP)   // >= 1 segment/warp
                                     : num_tiles(p->n, kMsTile);
@@ -643,6 +688,7 @@ dc_status maxsub_launch(dc_plan_t p, const int32_t* d_x, int64_t off, int mode,
 
 dc_status ensure_stage(dc_plan_t p, size_t bytes) {
     if (p->d_stage && p->d_stage_bytes >= bytes) return DC_OK;
+    drop_graphs(p);
     if (p->d_stage) cudaFree(p->d_stage);
     p->d_stage = nullptr;
     if (cudaMalloc(&p->d_stage, bytes) != cudaSuccess) {
@@ -665,7 +711,9 @@ dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* 
     int64_t total = 0;
     for (int64_t r : runs) total += r;
     if (total > p->n) return fail(DC_ERR_INVALID_ARG, "runs exceed the plan size");
-    dc_status st = ensure_scratch(p, V);
+    dc_status st = join_host_sorts(p);
+    if (st != DC_OK) return st;
+    st = ensure_scratch(p, V);
     if (st != DC_OK) return st;
     const size_t kb = align_up((size_t)p->n * 4, 256);
     uint32_t* sk = (uint32_t*)p->scratch;
@@ -673,11 +721,11 @@ dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* 
     int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
     constexpr SortCfg C = cfg_for<K, V, false>();
     auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
-    static bool attr_done = false;
-    if (!attr_done) {
+    static PerDevice attr_done;
+    if (!attr_done.get()) {
         DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         nk3_smem_bytes(C, V)));
-        attr_done = true;
+        attr_done.set(1);
     }
     int rounds = 0;
     for (size_t c = runs.size(); c > 1; c = (c + 1) / 2) ++rounds;
@@ -727,17 +775,19 @@ dc_status mg_merge_peers_typed(dc_plan_t p, const uint32_t* const* rk, const uin
     int64_t total = 0;
     for (int r = 0; r < runs; ++r) total += len[r];
     if (total > p->n) return fail(DC_ERR_INVALID_ARG, "runs exceed the plan size");
-    dc_status st = ensure_scratch(p, V);
+    dc_status st = join_host_sorts(p);
+    if (st != DC_OK) return st;
+    st = ensure_scratch(p, V);
     if (st != DC_OK) return st;
     const size_t kb = align_up((size_t)p->n * 4, 256);
     int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
     constexpr SortCfg C = cfg_for<K, V, false>();
     auto* k3 = dc::nk3_merge_ab<C.nt3, C.it, K, V>;
-    static bool attr_done = false;
-    if (!attr_done) {
+    static PerDevice attr_done;
+    if (!attr_done.get()) {
         DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         nk3_smem_bytes(C, V)));
-        attr_done = true;
+        attr_done.set(1);
     }
     const bool one_round = runs <= 2;
     uint32_t* dk = one_round ? out_k : tmp_k;
@@ -909,14 +959,6 @@ dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32
     return DC_OK;
 }
 
-static void drop_graphs(dc_plan_t p) {
-    for (auto& gc : p->graphs) {
-        if (gc.exec) cudaGraphExecDestroy(gc.exec);
-        if (gc.graph) cudaGraphDestroy(gc.graph);
-    }
-    p->graphs.clear();
-}
-
 dc_status dc_plan_set_two_level(dc_plan_t p, int32_t enable) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     p->two_level = enable != 0;
@@ -990,6 +1032,7 @@ dc_status dc_free(dc_plan_t p) {
     }
     if (p->join_in) cudaEventDestroy(p->join_in);
     if (p->join_out) cudaEventDestroy(p->join_out);
+    if (p->comp_done) cudaEventDestroy(p->comp_done);
     if (p->h2d) cudaStreamDestroy(p->h2d);
     if (p->d2h) cudaStreamDestroy(p->d2h);
     if (p->comp) cudaStreamDestroy(p->comp);
@@ -1411,6 +1454,7 @@ dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys
         DC_CUDA(p, cudaStreamCreateWithFlags(&p->comp, cudaStreamNonBlocking));
         DC_CUDA(p, cudaEventCreateWithFlags(&p->join_in, cudaEventDisableTiming));
         DC_CUDA(p, cudaEventCreateWithFlags(&p->join_out, cudaEventDisableTiming));
+        DC_CUDA(p, cudaEventCreateWithFlags(&p->comp_done, cudaEventDisableTiming));
         for (auto& hs : p->hslot) {
             DC_CUDA(p, cudaEventCreateWithFlags(&hs.in_done, cudaEventDisableTiming));
             DC_CUDA(p, cudaEventCreateWithFlags(&hs.sort_done, cudaEventDisableTiming));
@@ -1423,6 +1467,7 @@ dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys
     const size_t need = h_in_vals ? 2 * kb : kb;
     if (hs.bytes < need) {
         DC_CUDA(p, cudaEventSynchronize(hs.out_done));
+        drop_graphs(p);
         if (hs.d) cudaFree(hs.d);
         hs.d = nullptr;
         if (cudaMalloc(&hs.d, need) != cudaSuccess) {
@@ -1451,6 +1496,7 @@ dc_status dc_sort_host_submit(dc_plan_t p, dc_key_type kt, const void* h_in_keys
     p->stream = user;
     if (st != DC_OK) return st;
     DC_CUDA(p, cudaEventRecord(hs.sort_done, p->comp));
+    DC_CUDA(p, cudaEventRecord(p->comp_done, p->comp));
     // copy out
     DC_CUDA(p, cudaStreamWaitEvent(p->d2h, hs.sort_done, 0));
     DC_CUDA(p, cudaMemcpyAsync(h_out_keys, dk, bytes, cudaMemcpyDeviceToHost, p->d2h));

@@ -92,9 +92,12 @@ __global__ void mg_brackets(const int64_t* __restrict__ R, long long cands, int 
 
 // Send-buffer layout of one rank (uint32 words): for d = 1..G-1 a header of
 // three int64 {lo, len, t} at words [6(d-1), 6d), then the window keys of
-// boundary d at words hdr + (d-1)*wcap, hdr = 6(G-1).
+// boundary d at words hdr + (d-1)*wcap, hdr = 6(G-1).  The total is rounded
+// up to a multiple of 4 words, so every rank's buffer in the all-gathered
+// array starts 16-byte aligned and its int64 headers are aligned loads for
+// any stride (an odd stride with G even used to misalign every odd rank).
 __host__ __device__ constexpr long long mg_sendbuf_words(int G, long long wcap) {
-    return 6LL * (G - 1) + (long long)(G - 1) * wcap;
+    return (6LL * (G - 1) + (long long)(G - 1) * wcap + 3) / 4 * 4;
 }
 
 // a7 (3/4b): one CTA per boundary d.  This rank's elements strictly between

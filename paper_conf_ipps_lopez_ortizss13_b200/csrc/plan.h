@@ -87,6 +87,7 @@ struct dc_plan_s {
     HostSlot hslot[kHostSlots];
     cudaStream_t h2d = nullptr, d2h = nullptr, comp = nullptr;
     cudaEvent_t join_in = nullptr, join_out = nullptr;   // order against the plan stream
+    cudaEvent_t comp_done = nullptr;   // last host-slot sort on comp (scratch users wait on it)
     int64_t submits = 0;
     // library-owned communicator (dc_plan_set_comm / dc_plan_set_loopback):
     // n above is then this rank's shard, n_global the whole problem

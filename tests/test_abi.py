@@ -172,3 +172,55 @@ def test_mg_stride_range():
     assert dc.lib().dc_plan_set_mg_stride(p._h, 1 << 21) == 1
     assert dc.lib().dc_plan_set_mg_stride(p._h, 1024) == 0
     assert dc.lib().dc_loopback_free(None) == 0
+
+
+# ------------------------------------------------ binding argument checks
+
+def test_sendbuf_words_keep_every_rank_aligned():
+    """Back-to-back send buffers of all ranks stay 16-byte aligned for any
+    stride (the int64 headers of rank r sit at r * words * 4 bytes)."""
+    for world in (2, 3, 4, 8):
+        for wcap in (1, 63, 333, 1000, 1001, 4096):
+            w = dc.lib().dc_mg_sendbuf_words(world, wcap)
+            assert w % 4 == 0
+            assert w >= 6 * (world - 1) + (world - 1) * wcap
+            assert w < 6 * (world - 1) + (world - 1) * wcap + 4
+    assert dc.lib().dc_mg_sendbuf_words(1, 100) == 0
+
+
+def _host(n, dtype=None):
+    import torch
+    return torch.zeros(n, dtype=dtype or torch.int32)
+
+
+@pytest.mark.parametrize("call", [
+    lambda p: p.sort_host_(_host(99)),
+    lambda p: p.sort_host_(_host(100), _host(99)),
+    lambda p: p.sort_host_(_host(100, __import__("torch").int64)),
+    lambda p: p.sort_host_submit(_host(100), _host(99)),
+    lambda p: p.sort_host_submit(_host(100), _host(100), _host(100), None),
+    lambda p: p.max_subarray_host(_host(99)),
+    lambda p: p.max_subarray_host(_host(200)[::2]),
+])
+def test_host_entry_points_check_sizes_before_the_c_call(call):
+    """Host buffers the C side copies n*4 bytes into or out of are checked for
+    length, element size and contiguity first (a short tensor used to
+    overflow the host heap)."""
+    p = dc.Plan(100)
+    with pytest.raises(ValueError):
+        call(p)
+
+
+@pytest.mark.parametrize("call", [
+    lambda p: p.max_subarray(_host(100)),
+    lambda p: p.max_subarray_async(_host(100), _host(3, __import__("torch").int64)),
+    lambda p: p.max_subarray_tuple_async(_host(100), _host(8, __import__("torch").int64)),
+    lambda p: p.sum(_host(100)),
+    lambda p: p.sum_async(_host(100), _host(1, __import__("torch").int64)),
+    lambda p: p.sum_alg5(_host(100, __import__("torch").int64)),
+    lambda p: p.sort_(_host(100)),
+])
+def test_device_entry_points_reject_host_tensors(call):
+    p = dc.Plan(100)
+    with pytest.raises(ValueError):
+        call(p)

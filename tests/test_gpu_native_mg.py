@@ -119,6 +119,14 @@ def test_loopback_keys_only(dc, oracle_mod, key_type, stride):
     sort_case(dc, oracle_mod, 4 * 250_001, 4, "paper", key_type, False, stride)
 
 
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("stride", [1001, 333])
+def test_loopback_odd_stride(dc, oracle_mod, world, stride):
+    """odd sample strides with an even world size: every rank's
+    send buffer (int64 headers) must stay aligned in the all-gathered array."""
+    sort_case(dc, oracle_mod, world * 120_007, world, "uniform", "u32", True, stride)
+
+
 @pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
 def test_loopback_large_shards(dc, oracle_mod, p2p):
     """2^25 keys over 2 ranks: 16M-key shards use the full-size tile config."""

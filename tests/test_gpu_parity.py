@@ -155,6 +155,105 @@ def test_sort_max_key_values_and_pads(dc, oracle_mod):
     assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)
 
 
+@pytest.mark.parametrize("n", [(1 << 23) + 7, 4 * TILE * 128 + TILE * 5 + 3])
+@pytest.mark.parametrize("with_vals", [False, True])
+def test_sort_i32_pad_valued_keys_two_level(dc, oracle_mod, n, with_vals):
+    """i32 keys equal to KeyI32::kPad (INT32_MAX) -- the value the pad-safe
+    4-way merges put behind every piece -- mixed with INT32_MIN and ordinary
+    keys, on the two-level schedule (keys-only pad-safe path and the stable
+    key-value path)."""
+    keys = dcgen.sort_keys(n, "few", seed=31, key_type="i32", device="cuda")
+    sel = torch.arange(n, device="cuda")
+    keys[sel % 3 == 0] = 2**31 - 1
+    keys[sel % 7 == 1] = -2**31
+    vals = dcgen.sort_vals(n, device="cuda") if with_vals else None
+    k_in = _np_keys(keys, "i32").copy()
+    plan = dc.Plan(n)
+    assert plan.schedule("i32", with_vals)["hbm_passes"] < plan.schedule("i32", with_vals)["global_passes"]
+    plan.sort_(keys, vals, key_type="i32")
+    if with_vals:
+        ek, ev = oracle_mod.mergesort(k_in, np.arange(n, dtype=np.uint32), key_type="i32")
+        assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)
+    else:
+        ek = oracle_mod.mergesort(k_in, key_type="i32")
+    assert np.array_equal(_np_keys(keys, "i32"), ek)
+
+
+@pytest.mark.parametrize("n", [TILE * 3 + 11, (1 << 20) + 3, (1 << 23) + 7])
+@pytest.mark.parametrize("with_vals", [False, True])
+def test_sort_f32_infinities_and_signed_zeros(dc, oracle_mod, n, with_vals):
+    """f32 keys include +inf (== KeyF32::kPad, the pad of ragged tiles and of
+    the 4-way pieces), -inf, +0.0 and -0.0 (equal keys with distinct bits,
+    which must keep their input order), on the small, one-level and two-level
+    schedules, keys only and with values."""
+    keys = dcgen.sort_keys(n, "uniform", seed=33, key_type="f32", device="cuda")
+    sel = torch.arange(n, device="cuda")
+    keys[sel % 5 == 0] = float("inf")
+    keys[sel % 11 == 2] = float("-inf")
+    keys[sel % 13 == 3] = 0.0
+    keys[sel % 17 == 4] = -0.0
+    vals = dcgen.sort_vals(n, device="cuda") if with_vals else None
+    k_in = _np_keys(keys, "f32").copy()
+    dc.Plan(n).sort_(keys, vals, key_type="f32")
+    if with_vals:
+        ek, ev = oracle_mod.mergesort(k_in, np.arange(n, dtype=np.uint32), key_type="f32")
+        assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)
+    else:
+        ek = oracle_mod.mergesort(k_in, key_type="f32")
+    assert np.array_equal(_np_keys(keys, "f32").view(np.uint32), ek.view(np.uint32))
+
+
+@pytest.mark.parametrize("n", [1 << 20, (1 << 23) + 5])
+def test_graph_cache_survives_scratch_reallocation(dc, oracle_mod, n):
+    """a keys-only sort is captured as a CUDA graph; a key-value
+    sort on other buffers then needs a larger scratch (reallocated); replaying
+    keys-only on the first buffers must not touch the freed scratch."""
+    plan = dc.Plan(n)
+    keys = torch.empty(n, dtype=torch.int32, device="cuda")
+    for seed in range(3):            # eager, capture, replay
+        keys.copy_(dcgen.sort_keys(n, "uniform", seed=60 + seed, device="cuda"))
+        k_in = _np_keys(keys, "u32").copy()
+        plan.sort_(keys, key_type="u32")
+        assert np.array_equal(_np_keys(keys, "u32"), oracle_mod.mergesort(k_in)), seed
+    k2 = dcgen.sort_keys(n, "few", seed=64, device="cuda")
+    v2 = dcgen.sort_vals(n, device="cuda")
+    k2_in = _np_keys(k2, "u32").copy()
+    plan.sort_(k2, v2, key_type="u32")                 # reallocates the scratch
+    ek, ev = oracle_mod.mergesort(k2_in, np.arange(n, dtype=np.uint32))
+    assert np.array_equal(_np_keys(k2, "u32"), ek)
+    assert np.array_equal(v2.cpu().numpy().view(np.uint32), ev)
+    del k2, v2
+    torch.cuda.empty_cache()
+    junk = torch.full((2 * n,), 7, dtype=torch.int32, device="cuda")   # reuse freed memory
+    for seed in range(2):
+        keys.copy_(dcgen.sort_keys(n, "reverse", seed=70 + seed, device="cuda"))
+        k_in = _np_keys(keys, "u32").copy()
+        plan.sort_(keys, key_type="u32")
+        assert np.array_equal(_np_keys(keys, "u32"), oracle_mod.mergesort(k_in)), seed
+    assert bool((junk == 7).all())
+
+
+def test_host_submit_then_device_sort_ordering(dc, oracle_mod):
+    """host-slot sorts run on their own stream with the plan
+    scratch; a device sort enqueued right after them on the plan stream must
+    wait for them (dc.h: later scratch users are ordered after submissions)."""
+    n = (1 << 23) + 77
+    plan = dc.Plan(n)
+    ins = [dcgen.sort_keys(n, d, seed=80 + i).pin_memory()
+           for i, d in enumerate(["uniform", "few", "reverse"])]
+    outs = [torch.empty_like(t).pin_memory() for t in ins]
+    dev_keys = dcgen.sort_keys(n, "uniform", seed=90, device="cuda")
+    dk_in = _np_keys(dev_keys, "u32").copy()
+    for t, o in zip(ins, outs):
+        plan.sort_host_submit(t, o, key_type="u32")
+    plan.sort_(dev_keys, key_type="u32")                # same scratch, plan stream
+    plan.sort_host_wait()
+    torch.cuda.synchronize()
+    assert np.array_equal(_np_keys(dev_keys, "u32"), oracle_mod.mergesort(dk_in))
+    for t, o in zip(ins, outs):
+        assert np.array_equal(_np_keys(o, "u32"), oracle_mod.mergesort(_np_keys(t, "u32")))
+
+
 SMALL_TILE = 128 * 51        # keys-only tile below 2^23 keys
 
 
@@ -336,13 +435,24 @@ def _assert_sorted_permutation_u32(k_in, k_out, samples=12, seed=0):
 
 
 @pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "few"])
-def test_full_size_2pow28_keys(dc, dist):
+def test_full_size_2pow28_keys_exact(dc, oracle_mod, dist):
+    """BASELINE configs[2] at its full size, in the launch configuration bench.py
+    times (the default plan: 512 x 49 fused tiles, 7 two-level HBM passes):
+    every one of the 2^28 outputs equals the oracle's Alg 6 mergesort of the
+    same input (seed 3, as bench.py), element by element."""
     n = 1 << 28
     keys = dcgen.sort_keys(n, dist, seed=3, device="cuda")
-    k_in = keys.clone()
-    dc.Plan(n).sort_(keys, key_type="u32")
+    k_in = _np_keys(keys, "u32").copy()
+    plan = dc.Plan(n)
+    assert plan.schedule("u32")["hbm_passes"] == 7
+    plan.sort_(keys, key_type="u32")
     torch.cuda.synchronize()
-    _assert_sorted_permutation_u32(k_in, keys)
+    got = _np_keys(keys, "u32")
+    del keys
+    plan.close()
+    torch.cuda.empty_cache()
+    expect = oracle_mod.mergesort(k_in)
+    assert np.array_equal(got, expect)
 
 
 def test_max_size_keys(dc):
