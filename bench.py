@@ -86,7 +86,7 @@ class L2Flush:
     def __call__(self):
         import torch
 
-        torch.sum(self.buf, dtype=torch.int64, out=self.out)
+        torch.sum(self.buf, dim=0, out=self.out)
 
 
 def ncu_traffic(kernel: str, workload: str):

@@ -97,21 +97,27 @@ dc_status dc_plan_levels(dc_plan_t plan, int32_t *num_levels, int64_t *nodes,
                          int64_t *sizes, int32_t capacity);
 
 /* Execution schedule of an a=b=2 sort of this key type (with or without
- * values): the fused bottom kernel sorts tiles of `tile` keys (the leaves plus
- * fused_levels = ceil(log2(tile)) levels of the binary tree, entirely on
- * chip); global_passes = ceil(log2(ceil(n/tile))) levels remain, executed in
- * hbm_passes passes over HBM (keys-only u32/i32 sorts of n >= 2^23 fold two
- * levels per pass unless disabled with dc_plan_set_two_level).  Any output
- * pointer may be NULL. */
+ * values) as dc_run_mergesort will run it: the fused bottom kernel sorts tiles
+ * of `tile` keys (the leaves plus fused_levels = ceil(log2(tile)) levels of
+ * the binary tree, entirely on chip); global_passes =
+ * ceil(log2(ceil(n/tile))) levels remain, executed in hbm_passes passes over
+ * HBM (one or two levels per pass).  Tile class and pass kind are the
+ * planner's choice (dc_model_sort_schedule) unless forced with
+ * dc_plan_set_tile_class / dc_plan_set_two_level.  Any output pointer may be
+ * NULL. */
 dc_status dc_plan_schedule(dc_plan_t plan, dc_key_type key_type, int32_t with_vals,
                            int32_t *tile, int32_t *fused_levels, int32_t *global_passes,
                            int32_t *hbm_passes);
 
-/* Enable (default) or disable the two-levels-per-pass schedule of keys-only
- * u32/i32 sorts with n >= 2^23 (every pass merges groups of four
- * runs -- an exact 4-run selection per output tile, then a 4-way tile merge;
- * sort4_kernels.cuh).  Results are identical either way. */
+/* Force (1) or forbid (0) the two-levels-per-pass schedule (every
+ * pass merges groups of four runs -- an exact 4-run selection per output
+ * tile, then a 4-way tile merge; sort4_kernels.cuh), or leave it to the
+ * planner (-1, default).  Results are identical either way. */
 dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
+
+/* Force the NK1 tile class (1 quarter-size tiles of 128-thread CTAs, 2 full
+ * tiles) or leave it to the planner (0, default).  Results are identical. */
+dc_status dc_plan_set_tile_class(dc_plan_t plan, int32_t tile_class);
 
 /* Enable (default) or disable the fused partition of L2-resident sorts (n <
  * 2^23): every one-level merge CTA finds the co-ranks of its own output tile
@@ -241,6 +247,31 @@ dc_status dc_model_optimise(int32_t a, int32_t b, int32_t p, double g, double ga
                             double *alpha, double *gpu_work_fraction, double *level_y,
                             int32_t *model_case);
 
+/* B200 schedule planner: the Sec. 5.2 analysis re-parameterised
+ * for one B200 (model.cu).  The levels of the recursion tree run on chip (the
+ * bottom ceil(log2 T) levels of every NK1 tile, T set by the tile class) or
+ * in HBM passes of one level (NK2 + NK3) or two levels (NK2-4 + NK3-4); each
+ * kernel costs a launch term plus waves of resident CTAs (the parallelism
+ * threshold), with L2- and HBM-resident wave times fitted to
+ * B200 measurements (tools/planner_sweep.py, tools/planner_fit.py,
+ * profiles/r02/planner_sweep.json).  dc_run_mergesort runs the candidate of
+ * least predicted time unless the plan forces a tile class or pass kind.
+ * candidates_ms: [quarter tiles, one level/pass], [quarter, two], [full,
+ * one], [full, two].  Host-only; INVALID_ARG on bad arguments. */
+typedef struct {
+    int32_t tile_class;      /* 1 quarter-size tiles, 2 full tiles */
+    int32_t two_level;       /* 1: two tree levels per HBM pass (4-way passes) */
+    int32_t tile;            /* keys per NK1 tile */
+    int32_t fused_levels;    /* ceil(log2 tile) levels on chip */
+    int32_t global_levels;   /* ceil(log2(n / tile)) levels above the tile */
+    int32_t hbm_passes;      /* HBM passes of the chosen schedule */
+    double predicted_ms;
+    double candidates_ms[4];
+} dc_sort_schedule;
+/* tile_class: 0 free, 1 or 2 forced; two_level: -1 free, 0 or 1 forced. */
+dc_status dc_model_sort_schedule(int64_t n, dc_key_type key_type, int32_t with_vals,
+                                 int32_t tile_class, int32_t two_level, dc_sort_schedule *out);
+
 /* ------------------------------------------------ multi-GPU (rows a7-a10) */
 /* One process (or, for tests, one thread) per GPU.  With a communicator set,
  * the plan's n is the GLOBAL problem size; every rank passes its shard of
@@ -293,12 +324,14 @@ dc_status dc_plan_comm_info(dc_plan_t plan, int32_t *rank, int32_t *world, int64
  * world*S*4 <= 200 KiB).  Set before a run, the same on every rank. */
 dc_status dc_plan_set_mg_stride(dc_plan_t plan, int64_t stride);
 
-/* Exchange of the multi-GPU sort.  enable != 0 (default): FUSED -- every
- * rank sorts its shard into a plan-owned buffer that all peers map (CUDA IPC
- * over NVLink/NVSwitch; plain pointers in a loopback group), and the first
- * round of the G-way merge reads the runs straight from the peers' buffers
- * (dc_mg_merge_peers), then a stream-ordered barrier; no all-to-all, no
- * receive buffer write.  enable == 0: NCCL all-to-all, then the local merge.
+/* Exchange of the multi-GPU sort.  enable != 0: FUSED -- every rank sorts
+ * its shard into a plan-owned buffer that all peers map (CUDA IPC over
+ * NVLink/NVSwitch; plain pointers in a loopback group), and the first round
+ * of the G-way merge reads the runs straight from the peers' buffers
+ * (dc_mg_merge_peers: up to four peers per 4-way pass), then a stream-ordered
+ * barrier; no all-to-all, no receive buffer write.  enable == 0 (default
+ * until the fused mode has been measured across GPUs): NCCL all-to-all
+ * (grouped send/recv), then the local merge (dc_mg_merge_runs).
  * Set before the first sort, the same on every rank; if any rank cannot map
  * every peer, all ranks fall back to the all-to-all (decided collectively at
  * the first sort).  $DC_MG_P2P=0/1 overrides. */
@@ -370,14 +403,31 @@ dc_status dc_mg_windows(dc_plan_t plan, const uint32_t *d_keys, int64_t n, int32
 dc_status dc_mg_split_matrix(dc_plan_t plan, dc_key_type key_type, const uint32_t *d_gathered,
                              int32_t world, int64_t shard_n, int64_t wcap, int64_t *d_cmat);
 
+/* Host-only: the exchange plan of `rank` from a split matrix h_cmat
+ * (world x (world+1), as dc_mg_split_matrix / dc_plan_last_splits give it).
+ * Rank `rank` sends its shard range [send_off[d], send_off[d] + send_cnt[d])
+ * to rank d and receives recv_cnt[d] elements from rank d, placed at
+ * recv_off[d] of its receive buffer (runs back to back in rank order, the
+ * order dc_mg_merge_runs needs for the global stable order).  Checks that
+ * every row runs monotonically from 0 to shard_n and that the received total
+ * is shard_n (INVALID_ARG otherwise).  Output arrays hold `world` entries.
+ * This is the runtime's own host step (dc_run_mergesort with a communicator
+ * calls it); exposed so that callers and tests can drive it. */
+dc_status dc_mg_exchange_sizes(const int64_t *h_cmat, int32_t world, int32_t rank,
+                               int64_t shard_n, int64_t *send_cnt, int64_t *send_off,
+                               int64_t *recv_cnt, int64_t *recv_off);
+
 /* Synchronises and reports whether a window overflowed its capacity
  * (*h_err != 0 means the shard was not sorted or wcap < stride). */
 dc_status dc_mg_error(dc_plan_t plan, int32_t *h_err);
 
 /* Local stable merge of `runs` sorted runs stored back to back in d_in_keys
  * (run r has h_run_len[r] elements, host array; total <= plan n) into
- * d_out_keys; earlier runs win ties.  Values (nullable, both or neither)
- * move with their keys.  d_in_* is used as ping-pong space and clobbered. */
+ * d_out_keys; earlier runs win ties (Alg 7's top levels).
+ * Values (nullable, both or neither) move with their keys.  Groups of four
+ * runs merge in one HBM pass (exact 4-run selection + 4-way tile merge),
+ * a pair in one pass: ceil(log4 runs) passes.  d_in_* is used as ping-pong
+ * space (with more than 16 runs) and may be clobbered. */
 dc_status dc_mg_merge_runs(dc_plan_t plan, dc_key_type key_type, uint32_t *d_in_keys,
                            uint32_t *d_in_vals, uint32_t *d_out_keys, uint32_t *d_out_vals,
                            const int64_t *h_run_len, int32_t runs);
@@ -389,9 +439,11 @@ dc_status dc_mg_merge_runs(dc_plan_t plan, dc_key_type key_type, uint32_t *d_in_
  * h_off[r] of the buffer h_run_keys[r] (+ h_run_vals[r]; host arrays of
  * device pointers, 16-byte aligned, readable for h_bound[r] elements; the
  * pointers may be peer mappings).  Earlier runs win ties.  Output:
- * d_out_keys (+ d_out_vals), sum(h_len) <= plan n elements.  With more than
- * two runs the first round writes d_tmp_* (n elements each) and later rounds
- * are local.  Enqueue-only. */
+ * d_out_keys (+ d_out_vals), sum(h_len) <= plan n elements.  Up to four runs
+ * merge in ONE pass straight from their buffers (4-way tiles whose pieces the
+ * TMA fetches from up to four peers); with more than four runs the first
+ * round writes d_tmp_* (n elements each) and later rounds are local.
+ * Enqueue-only. */
 dc_status dc_mg_merge_peers(dc_plan_t plan, dc_key_type key_type,
                             const uint32_t *const *h_run_keys, const uint32_t *const *h_run_vals,
                             const int64_t *h_bound, const int64_t *h_off, const int64_t *h_len,

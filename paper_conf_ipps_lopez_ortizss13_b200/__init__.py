@@ -12,8 +12,8 @@ if the library is missing or no CUDA device is present, calls raise.
 
 Multi-GPU (one process per GPU): ``plan = dc.init_dist(n)`` binds a plan of
 global size n to a library-owned NCCL communicator; ``plan.sort_(shard)`` then
-runs the whole distributed sort in the library.  :mod:`.dist` composes the
-same per-rank steps over any torch.distributed group (gloo tests).
+runs the whole distributed sort in the library.  :mod:`.dist` drives it for
+bench.py and verifies the global result.
 """
 from __future__ import annotations
 
@@ -30,6 +30,7 @@ from . import build as _build
 __all__ = [
     "DcError", "Plan", "sort_", "max_subarray", "lib", "KEY_U32", "KEY_I32", "KEY_F32",
     "MaxsubResult", "MaxsubTuple", "get_unique_id", "init_dist", "LoopbackGroup",
+    "broadcast_unique_id", "mg_exchange_sizes",
 ]
 
 KEY_U32, KEY_I32, KEY_F32 = 0, 1, 2
@@ -63,6 +64,7 @@ _SIGS = {
     "dc_plan_schedule": ([_P, ctypes.c_int, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32),
                           ctypes.POINTER(_I32), ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
+    "dc_plan_set_tile_class": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_fused_partition": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_graphs": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_pipeline": ([_P, _I32], ctypes.c_int),
@@ -96,6 +98,7 @@ _SIGS.update({
     "dc_mg_split_matrix": ([_P, ctypes.c_int, _P, _I32, _I64, _I64, _P], ctypes.c_int),
     "dc_mg_error": ([_P, ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_mg_merge_runs": ([_P, ctypes.c_int, _P, _P, _P, _P, _P, _I32], ctypes.c_int),
+    "dc_mg_exchange_sizes": ([_P, _I32, _I32, _I64, _P, _P, _P, _P], ctypes.c_int),
 })
 
 _SIGS.update({
@@ -116,7 +119,15 @@ _SIGS.update({
                           ctypes.c_int),
 })
 
+class SortSchedule(ctypes.Structure):
+    _fields_ = [("tile_class", _I32), ("two_level", _I32), ("tile", _I32),
+                ("fused_levels", _I32), ("global_levels", _I32), ("hbm_passes", _I32),
+                ("predicted_ms", ctypes.c_double), ("candidates_ms", ctypes.c_double * 4)]
+
+
 _SIGS.update({
+    "dc_model_sort_schedule": ([_I64, ctypes.c_int, _I32, _I32, _I32, ctypes.POINTER(SortSchedule)],
+                               ctypes.c_int),
     "dc_run_sum": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
     "dc_run_sum_async": ([_P, _P, _P], ctypes.c_int),
     "dc_run_sum_alg5": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
@@ -140,6 +151,20 @@ def model_gpu_work(a: int, b: int, p: int, g: float, gamma: float, n: float,
     if st != 0:
         raise DcError(st, "invalid model parameters")
     return {"gpu_work_fraction": f.value, "level_y": y.value, "case": c.value}
+
+
+def model_sort_schedule(n: int, key_type: str = "u32", with_vals: bool = False,
+                        tile_class: int = 0, two_level: int = -1) -> dict:
+    """The B200 schedule planner (dc_model_sort_schedule): the
+    schedule of least predicted time and every candidate's prediction."""
+    s = SortSchedule()
+    _check(lib().dc_model_sort_schedule(n, _KEY_NAMES[key_type], int(with_vals), tile_class,
+                                        two_level, ctypes.byref(s)))
+    return {"tile_class": s.tile_class, "two_level": bool(s.two_level), "tile": s.tile,
+            "fused_levels": s.fused_levels, "global_levels": s.global_levels,
+            "hbm_passes": s.hbm_passes, "predicted_ms": s.predicted_ms,
+            "candidates_ms": {"quarter_one": s.candidates_ms[0], "quarter_two": s.candidates_ms[1],
+                              "full_one": s.candidates_ms[2], "full_two": s.candidates_ms[3]}}
 
 
 def model_optimise(a: int, b: int, p: int, g: float, gamma: float, n: float) -> dict:
@@ -328,9 +353,14 @@ class Plan:
         """L2-resident sorts: merge CTAs find their own co-ranks (default on)."""
         _check(lib().dc_plan_set_fused_partition(self._h, int(enable)))
 
-    def set_two_level(self, enable: bool) -> None:
-        """Two merge levels per HBM pass for keys-only sorts of n >= 2^23 (default on)."""
-        _check(lib().dc_plan_set_two_level(self._h, int(enable)))
+    def set_two_level(self, enable: bool | None) -> None:
+        """Force (True) / forbid (False) two merge levels per HBM pass (SURVEY
+        f1), or leave the choice to the planner (None, the default)."""
+        _check(lib().dc_plan_set_two_level(self._h, -1 if enable is None else int(enable)))
+
+    def set_tile_class(self, tile_class: int) -> None:
+        """NK1 tile class: 1 quarter-size, 2 full, 0 planner (default)."""
+        _check(lib().dc_plan_set_tile_class(self._h, tile_class))
 
     def scratch_bytes(self, with_vals: bool = False) -> int:
         b = ctypes.c_size_t()
@@ -626,19 +656,42 @@ class LoopbackGroup:
         self.close()
 
 
+def broadcast_unique_id(group=None) -> bytes:
+    """The group's rank 0 creates a 128-byte NCCL id; torch.distributed
+    broadcasts it to every member (any backend)."""
+    import torch.distributed as tdist
+
+    rank = tdist.get_rank(group)
+    obj = [get_unique_id() if rank == 0 else None]
+    tdist.broadcast_object_list(obj, src=tdist.get_global_rank(group, 0) if group else 0,
+                                group=group)
+    if not isinstance(obj[0], (bytes, bytearray)) or len(obj[0]) != 128:
+        raise DcError(1, "bad unique id received")
+    return bytes(obj[0])
+
+
 def init_dist(n: int, group=None) -> Plan:
     """Plan of global size n bound to a library-owned NCCL communicator over
     the torch.distributed group (rank 0 creates the id, broadcast by torch).
     Set the CUDA device of this rank first."""
     import torch.distributed as tdist
 
-    rank, world = tdist.get_rank(group), tdist.get_world_size(group)
-    obj = [get_unique_id() if rank == 0 else None]
-    tdist.broadcast_object_list(obj, src=tdist.get_global_rank(group, 0) if group else 0,
-                                group=group)
+    uid = broadcast_unique_id(group)
     plan = Plan(n)
-    plan.set_comm(obj[0], rank, world)
+    plan.set_comm(uid, tdist.get_rank(group), tdist.get_world_size(group))
     return plan
+
+
+def mg_exchange_sizes(cmat, rank: int, shard_n: int) -> dict:
+    """The runtime's host step (dc_mg_exchange_sizes): from a split matrix
+    c[r][d] (world x (world+1)), what `rank` sends to / receives from every
+    rank: {'send_cnt', 'send_off', 'recv_cnt', 'recv_off'} lists."""
+    world = len(cmat)
+    flat = (_I64 * (world * (world + 1)))(*[int(v) for row in cmat for v in row])
+    arrs = [(_I64 * world)() for _ in range(4)]
+    _check(lib().dc_mg_exchange_sizes(flat, world, rank, shard_n, *arrs))
+    return dict(zip(("send_cnt", "send_off", "recv_cnt", "recv_off"),
+                    [list(a) for a in arrs]))
 
 
 _plans: dict = {}

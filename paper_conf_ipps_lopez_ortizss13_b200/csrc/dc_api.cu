@@ -102,8 +102,7 @@ constexpr SortCfg cfg_for() {
            : K::kNeedStable ? (SMALL ? kCfgStableSmall : kCfgStable)
                                  : (SMALL ? kCfgFastSmall : kCfgFast);
 }
-SortCfg cfg_for_runtime(dc_key_type kt, bool vals, int64_t n) {
-    const bool small = n < kSmallN;
+SortCfg cfg_for_runtime(dc_key_type kt, bool vals, bool small) {
     return vals ? (small ? kCfgStableSmall : kCfgKV)
            : kt == DC_KEY_F32 ? (small ? kCfgStableSmall : kCfgStable)
                                       : (small ? kCfgFastSmall : kCfgFast);
@@ -174,36 +173,27 @@ size_t split_entries(int64_t n) {
 #ifndef DC_TWO_IT_KV
 #define DC_TWO_IT_KV 25
 #endif
-// Keys only, selection fused into the pass (nk3_merge4 NSEL > 0, built with
-// -DDC_M4_NSEL=3): selector warps join the CTA, so the merge threads shrink
-// to 736 (896 threads x 72 registers fit the register file).  Measured at
-// 2^28: merges + selection 5.02 ms (3 selector warps) / 4.70 ms (6, with 640
-// merge threads) vs 4.36 ms for the separate nk2_select4 launch (0, default):
-// a boundary's ~11 dependent rounds need many warps in flight, which a
-// separate full-GPU launch provides and a few warps per SM do not.
-#ifndef DC_M4_NSEL
-#define DC_M4_NSEL 0
-#endif
-#ifndef DC_TWO_NT_FUSED
-#define DC_TWO_NT_FUSED 736
-#endif
+// (Selection fused into the pass -- selector warps inside nk3_merge4 -- was
+// measured slower at 2^28: merges + selection 5.02 / 4.70 ms with 3 / 6
+// selector warps vs 4.36 ms for the separate nk2_select4 launch: a
+// boundary's ~11 dependent rounds need many warps in flight, which a separate
+// full-GPU launch provides and a few warps per SM do not.  Removed in r02.)
 struct TwoCfg {
-    int nt, it, nsel;
+    int nt, it;
     constexpr int T() const { return nt * it; }
-    constexpr int threads() const { return nt + 64 + 32 * nsel; }
+    constexpr int threads() const { return nt + 64; }
 };
-constexpr TwoCfg kTwoKeys = DC_M4_NSEL > 0 ? TwoCfg{DC_TWO_NT_FUSED, DC_TWO_IT, DC_M4_NSEL}
-                                           : TwoCfg{DC_TWO_NT, DC_TWO_IT, 0};
-constexpr TwoCfg kTwoKV{DC_TWO_NT_KV, DC_TWO_IT_KV, 0};
-constexpr TwoCfg kTwoF32{DC_TWO_NT, DC_TWO_IT, 0};   // f32 keys: stable merges, separate select
+constexpr TwoCfg kTwoKeys{DC_TWO_NT, DC_TWO_IT};
+constexpr TwoCfg kTwoKV{DC_TWO_NT_KV, DC_TWO_IT_KV};
+constexpr TwoCfg kTwoF32{DC_TWO_NT, DC_TWO_IT};   // f32 keys: stable merges
 constexpr int kTwoMinT = cmin(cmin(kTwoKeys.T(), kTwoKV.T()), kTwoF32.T());
 template <class K, bool V>
 constexpr TwoCfg two_cfg() { return V ? kTwoKV : (K::kNeedStable ? kTwoF32 : kTwoKeys); }
 
 size_t two_level_tab_entries(int64_t) { return 0; }
 size_t two_level_bnd_entries(int64_t n) {
-    // groups at the smallest width (w = tile) have the most tiles
-    const int64_t w = cmin(cmin(kCfgFast.tile(), kCfgStable.tile()), kCfgKV.tile());
+    // groups at the smallest width (w = tile, any configuration) have the most tiles
+    const int64_t w = kMinTile;
     const int64_t groups = (n + 4 * w - 1) / (4 * w);
     return 4 * ((size_t)(groups * num_tiles(4 * w, kTwoMinT)) + 2);
 }
@@ -346,12 +336,51 @@ dc_status ensure_pipeline(dc_plan_t p, int chunks) {
     return DC_OK;
 }
 
+// One two-level pass (f1) over the runs P describes: the exact 4-run cuts of
+// every output tile (nk2_select4), then the persistent 4-way tile merge
+// (nk3_merge4) into dst.  Used by the breadth-first sort (uniform groups of
+// four runs) and by the multi-GPU G-way merge (one custom group per launch).
+template <class K, bool V>
+dc_status pass4(dc_plan_t p, const dc::Pass4& P, int tiles, dc::Cut4* cuts, uint32_t* dst_k,
+                uint32_t* dst_v, cudaStream_t st) {
+    constexpr TwoCfg TC = two_cfg<K, V>();
+    auto* k32 = dc::nk3_merge4<TC.nt, TC.it, K, V>;
+    constexpr int thr2 = TC.threads();
+    constexpr int smem2 = dc::m4_smem_bytes(TC.T(), TC.it, V);
+    static PerDevice grid2_dev;                  // per instantiation and device
+    int grid2 = grid2_dev.get();
+    if (!grid2) {
+        DC_CUDA(p, cudaFuncSetAttribute(k32, cudaFuncAttributeMaxDynamicSharedMemorySize, smem2));
+        int dev = 0, sms = 148, occ = 1;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, thr2, smem2);
+        grid2 = sms * (occ > 0 ? occ : 1);
+        grid2_dev.set(grid2);
+    }
+    if (tiles <= 0) return DC_OK;
+    {
+        TimedScope ts(p, DC_KERNEL_NK2_PARTITION, st);
+        constexpr int PV = V ? 4 : 2;           // pivots per run (sort4_kernels.cuh)
+        constexpr int bpw = dc::sel4_bpw<PV>();
+        const int sel_warps = (tiles + bpw - 1) / bpw;
+        dc::nk2_select4<K, PV><<<(sel_warps + 3) / 4, 128, 0, st>>>(P, tiles, cuts);
+        DC_LAUNCHED(p);
+    }
+    {
+        TimedScope ts(p, DC_KERNEL_NK3_MERGE, st);
+        k32<<<std::min(tiles, grid2), thr2, smem2, st>>>(P, dst_k, dst_v, cuts, tiles);
+        DC_LAUNCHED(p);
+    }
+    return DC_OK;
+}
+
 // Sorts keys[0..n) (+ vals) into out_k (+ out_v); out may equal the input
 // (in place).  NK1 reads the input; the passes ping-pong between scratch and
 // the output buffer.
 template <class K, bool V, bool SMALL>
 dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_k,
-                     uint32_t* out_v) {
+                     uint32_t* out_v, bool two_level) {
     const int64_t n = p->n;
     const bool hv = V;
     dc_status st = ensure_scratch(p, hv);
@@ -381,8 +410,8 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     // two levels into one pass (4-way groups, sort4_kernels.cuh); with P odd
     // one single-level pass goes first.
     const int P = global_passes(n, C.tile());
-    constexpr bool kTwoCapable = !SMALL;
-    const bool two = kTwoCapable && p->two_level && P >= 2;
+    constexpr bool kTwoCapable = true;
+    const bool two = two_level && P >= 2;
     const int single = two ? (P % 2) : P;
     const int passes = two ? single + (P - single) / 2 : P;
     // Ping-pong parity: the last pass must write the output buffer, so NK1
@@ -494,41 +523,22 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         if (two) {
             int* tab = split + align_up(split_entries(n) * 4, 256) / 4;
             dc::Cut4* cuts = (dc::Cut4*)(tab + align_up(two_level_tab_entries(n) * 4, 256) / 4);
-            constexpr TwoCfg TC = two_cfg<K, V>();
-            auto* k32 = dc::nk3_merge4<TC.nt, TC.it, K, V, (K::kNeedStable ? 0 : TC.nsel)>;
-            constexpr bool fused_sel = !K::kNeedStable && TC.nsel > 0;
-            constexpr int thr2 = fused_sel ? TC.threads() : TC.nt + 64;
-            constexpr int smem2 = dc::m4_smem_bytes(TC.T(), TC.it, V);
-            static PerDevice grid2_dev;                  // per instantiation and device
-            int grid2 = grid2_dev.get();
-            if (!grid2) {
-                DC_CUDA(p, cudaFuncSetAttribute(k32, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                smem2));
-                int dev = 0, sms = 148, occ = 1;
-                cudaGetDevice(&dev);
-                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k32, thr2, smem2);
-                grid2 = sms * (occ > 0 ? occ : 1);
-                grid2_dev.set(grid2);
-            }
             for (; w < n; w *= 4) {
-                const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), TC.T());
+                const int tpg = (int)num_tiles(std::min<int64_t>(4 * w, n), two_cfg<K, V>().T());
+                dc::Pass4 P{};
+                for (int q = 0; q < 4; ++q) {
+                    P.k[q] = cur_k;
+                    P.v[q] = cur_v;
+                    P.bound[q] = n;
+                }
+                P.n = n;
+                P.w = w;
+                P.T = two_cfg<K, V>().T();
+                P.tpg = tpg;
+                P.custom = 0;
                 const int tiles2 = (int)(((n + 4 * w - 1) / (4 * w)) * tpg);
-                if (!fused_sel) {
-                    TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-                    constexpr int PV = V ? 4 : 2;           // pivots per run (sort4_kernels.cuh)
-                    constexpr int bpw = dc::sel4_bpw<PV>();
-                    const int sel_warps = (tiles2 + bpw - 1) / bpw;
-                    dc::nk2_select4<K, PV><<<(sel_warps + 3) / 4, 128, 0, p->stream>>>(
-                        cur_k, n, w, TC.T(), tpg, tiles2, cuts);
-                    DC_LAUNCHED(p);
-                }
-                {
-                    TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                    k32<<<std::min(tiles2, grid2), thr2, smem2, p->stream>>>(
-                        cur_k, cur_v, oth_k, oth_v, n, w, tpg, cuts, tiles2);
-                    DC_LAUNCHED(p);
-                }
+                st = pass4<K, V>(p, P, tiles2, cuts, oth_k, oth_v, p->stream);
+                if (st != DC_OK) return st;
                 std::swap(cur_k, oth_k);
                 std::swap(cur_v, oth_v);
             }
@@ -537,22 +547,34 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     return DC_OK;
 }
 
+// The schedule of one sort: the planner's choice (model.cu, dc_model_sort_
+// schedule) among the compiled tile classes and pass kinds, unless the plan
+// forces one of them.
+struct Decision {
+    bool small, two;
+};
+Decision decide(dc_plan_t p, dc_key_type kt, bool vals) {
+    dc_sort_schedule s{};
+    dc_model_sort_schedule(p->n, kt, vals ? 1 : 0, p->tile_class, p->two_force, &s);
+    return {s.tile_class == 1, s.two_level != 0};
+}
+
 template <class K>
-dc_status sort_kv_dispatch(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* ok,
-                           uint32_t* ov) {
-    const bool small = p->n < kSmallN;
-    if (vals) return small ? sort_typed<K, true, true>(p, keys, vals, ok, ov)
-                           : sort_typed<K, true, false>(p, keys, vals, ok, ov);
-    return small ? sort_typed<K, false, true>(p, keys, nullptr, ok, nullptr)
-                 : sort_typed<K, false, false>(p, keys, nullptr, ok, nullptr);
+dc_status sort_kv_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals,
+                           uint32_t* ok, uint32_t* ov) {
+    const Decision d = decide(p, kt, vals != nullptr);
+    if (vals) return d.small ? sort_typed<K, true, true>(p, keys, vals, ok, ov, d.two)
+                             : sort_typed<K, true, false>(p, keys, vals, ok, ov, d.two);
+    return d.small ? sort_typed<K, false, true>(p, keys, nullptr, ok, nullptr, d.two)
+                   : sort_typed<K, false, false>(p, keys, nullptr, ok, nullptr, d.two);
 }
 
 dc_status sort_direct(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals, uint32_t* ok,
                       uint32_t* ov) {
     switch (kt) {
-        case DC_KEY_U32: return sort_kv_dispatch<dc::KeyU32>(p, keys, vals, ok, ov);
-        case DC_KEY_I32: return sort_kv_dispatch<dc::KeyI32>(p, keys, vals, ok, ov);
-        case DC_KEY_F32: return sort_kv_dispatch<dc::KeyF32>(p, keys, vals, ok, ov);
+        case DC_KEY_U32: return sort_kv_dispatch<dc::KeyU32>(p, kt, keys, vals, ok, ov);
+        case DC_KEY_I32: return sort_kv_dispatch<dc::KeyI32>(p, kt, keys, vals, ok, ov);
+        case DC_KEY_F32: return sort_kv_dispatch<dc::KeyF32>(p, kt, keys, vals, ok, ov);
     }
     return fail(DC_ERR_INVALID_ARG, "unknown key type");
 }
@@ -701,79 +723,28 @@ dc_status ensure_stage(dc_plan_t p, size_t bytes) {
 }
 
 
-// a9: local stable G-way merge.  Adjacent runs are merged pairwise, log2(runs)
-// rounds, one NK2 + NK3 launch pair per run pair (pair mode: arbitrary
-// lengths and offsets); ping-pong between the input buffer and the plan
-// scratch, the last round writes the output buffer.
-template <class K, bool V>
-dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* out_k,
-                         uint32_t* out_v, std::vector<int64_t> runs) {
-    int64_t total = 0;
-    for (int64_t r : runs) total += r;
-    if (total > p->n) return fail(DC_ERR_INVALID_ARG, "runs exceed the plan size");
-    dc_status st = join_host_sorts(p);
-    if (st != DC_OK) return st;
-    st = ensure_scratch(p, V);
-    if (st != DC_OK) return st;
-    const size_t kb = align_up((size_t)p->n * 4, 256);
-    uint32_t* sk = (uint32_t*)p->scratch;
-    uint32_t* sv = V ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
-    int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
-    constexpr SortCfg C = cfg_for<K, V, false>();
-    auto* k3 = dc::nk3_merge<C.nt3, C.it, K, V>;
-    static PerDevice attr_done;
-    if (!attr_done.get()) {
-        DC_CUDA(p, cudaFuncSetAttribute(k3, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        nk3_smem_bytes(C, V)));
-        attr_done.set(1);
-    }
-    int rounds = 0;
-    for (size_t c = runs.size(); c > 1; c = (c + 1) / 2) ++rounds;
-    if (rounds == 0) rounds = 1;                       // a single run: one copy round
-    uint32_t *cur_k = in_k, *cur_v = in_v;
-    for (int rd = 0; rd < rounds; ++rd) {
-        const bool last = rd == rounds - 1;
-        uint32_t* dst_k = last ? out_k : ((cur_k == in_k) ? sk : in_k);
-        uint32_t* dst_v = last ? out_v : ((cur_k == in_k) ? sv : in_v);
-        std::vector<int64_t> next;
-        int64_t org = 0;
-        for (size_t r = 0; r < runs.size(); r += 2) {
-            const int64_t la = runs[r], lb = (r + 1 < runs.size()) ? runs[r + 1] : 0;
-            if (la + lb > 0) {
-                const int tiles = (int)num_tiles(la + lb, C.tout());
-                const dc::PairGeom g{org, la, lb, org + la + lb, tiles};
-                {
-                    TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-                    dc::nk2_partition<K><<<(tiles + 255) / 256, 256, 0, p->stream>>>(
-                        cur_k, g, C.tout(), tiles, split);
-                    DC_LAUNCHED(p);
-                }
-                {
-                    TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                    k3<<<tiles, C.nt3, nk3_smem_bytes(C, V), p->stream>>>(cur_k, cur_v, dst_k,
-                                                                          dst_v, split, g);
-                    DC_LAUNCHED(p);
-                }
-            }
-            next.push_back(la + lb);
-            org += la + lb;
-        }
-        runs.swap(next);
-        cur_k = dst_k;
-        cur_v = dst_v;
-    }
-    return DC_OK;
-}
+// a9: local stable G-way merge (Alg 7's top log2 G levels, earlier runs win
+// ties).  A run is (key buffer, value buffer, readable length, offset,
+// length); in the first round the buffers may be peer GPUs' sorted shards
+// (the fused exchange) or the all-to-all receive buffer.  Every round merges
+// consecutive groups of FOUR runs with one two-level pass each (f1's exact
+// 4-run selection + 4-way tile merge, Pass4 custom mode), a trailing group of
+// two with one pair-mode merge pass (NK2 co-ranks + NK3 tiles over separately
+// addressed runs), a lone run by a copy; the merged groups are the next
+// round's runs.  HBM passes: ceil(log4 G) -- G = 2..4: one, G = 5..16: two --
+// against ceil(log2 G) for pairwise rounds.  Rounds write d0, d1, d0, ... and
+// the last one the output buffers.
+struct RunRef {
+    const uint32_t* k;
+    const uint32_t* v;
+    int64_t bound, off, len;
+};
 
-// a8+a9 fused: the first round of the G-way merge reads its runs where they
-// lie (peer shards over NVLink); later rounds are local (mg_merge_typed).
 template <class K, bool V>
-dc_status mg_merge_peers_typed(dc_plan_t p, const uint32_t* const* rk, const uint32_t* const* rv,
-                               const int64_t* bound, const int64_t* off, const int64_t* len,
-                               int runs, uint32_t* tmp_k, uint32_t* tmp_v, uint32_t* out_k,
-                               uint32_t* out_v) {
+dc_status merge_g(dc_plan_t p, std::vector<RunRef> runs, uint32_t* d0_k, uint32_t* d0_v,
+                  uint32_t* d1_k, uint32_t* d1_v, uint32_t* out_k, uint32_t* out_v) {
     int64_t total = 0;
-    for (int r = 0; r < runs; ++r) total += len[r];
+    for (const RunRef& r : runs) total += r.len;
     if (total > p->n) return fail(DC_ERR_INVALID_ARG, "runs exceed the plan size");
     dc_status st = join_host_sorts(p);
     if (st != DC_OK) return st;
@@ -781,7 +752,10 @@ dc_status mg_merge_peers_typed(dc_plan_t p, const uint32_t* const* rk, const uin
     if (st != DC_OK) return st;
     const size_t kb = align_up((size_t)p->n * 4, 256);
     int* split = (int*)((char*)p->scratch + kb + (V ? kb : 0));
+    dc::Cut4* cuts = (dc::Cut4*)(split + align_up(split_entries(p->n) * 4, 256) / 4 +
+                                 align_up(two_level_tab_entries(p->n) * 4, 256) / 4);
     constexpr SortCfg C = cfg_for<K, V, false>();
+    constexpr int T4 = two_cfg<K, V>().T();
     auto* k3 = dc::nk3_merge_ab<C.nt3, C.it, K, V>;
     static PerDevice attr_done;
     if (!attr_done.get()) {
@@ -789,35 +763,105 @@ dc_status mg_merge_peers_typed(dc_plan_t p, const uint32_t* const* rk, const uin
                                         nk3_smem_bytes(C, V)));
         attr_done.set(1);
     }
-    const bool one_round = runs <= 2;
-    uint32_t* dk = one_round ? out_k : tmp_k;
-    uint32_t* dv = one_round ? out_v : tmp_v;
-    std::vector<int64_t> next;
-    int64_t org = 0;
-    for (int r = 0; r < runs; r += 2) {
-        const int rb = r + 1 < runs ? r + 1 : r;          // odd tail: B empty (a copy)
-        const int64_t la = len[r], lb = r + 1 < runs ? len[r + 1] : 0;
-        if (la + lb > 0) {
-            const int tiles = (int)num_tiles(la + lb, C.tout());
-            {
-                TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
-                dc::nk2_partition_ab<K><<<(tiles + 3) / 4, 128, 0, p->stream>>>(
-                    rk[r] + off[r], la, rk[rb] + off[rb], lb, C.tout(), tiles, split);
-                DC_LAUNCHED(p);
+    if (runs.empty()) return DC_OK;
+    int rounds = 0;
+    for (size_t c = runs.size(); c > 1; c = (c + 3) / 4) ++rounds;
+    if (rounds == 0) rounds = 1;                       // a single run: one copy round
+    for (int rd = 0; rd < rounds; ++rd) {
+        const bool last = rd == rounds - 1;
+        uint32_t* dk = last ? out_k : (rd % 2 == 0 ? d0_k : d1_k);
+        uint32_t* dv = last ? out_v : (rd % 2 == 0 ? d0_v : d1_v);
+        std::vector<RunRef> next;
+        int64_t org = 0;
+        for (size_t g = 0; g < runs.size(); g += 4) {
+            const size_t cnt = std::min<size_t>(4, runs.size() - g);
+            int64_t glen = 0;
+            for (size_t q = 0; q < cnt; ++q) glen += runs[g + q].len;
+            if (glen > 0 && cnt >= 3) {                 // two levels in one pass
+                dc::Pass4 P{};
+                for (int q = 0; q < 4; ++q) {
+                    const RunRef& r = runs[g + std::min<size_t>(q, cnt - 1)];
+                    P.k[q] = r.k;
+                    P.v[q] = r.v;
+                    P.bound[q] = r.bound;
+                    P.off[q] = r.off;
+                    P.len[q] = (size_t)q < cnt ? r.len : 0;
+                }
+                P.out0 = org;
+                P.T = T4;
+                P.tpg = (int)num_tiles(glen, T4);
+                P.custom = 1;
+                st = pass4<K, V>(p, P, P.tpg, cuts, dk, dv, p->stream);
+                if (st != DC_OK) return st;
+            } else if (glen > 0 && cnt == 2) {          // one level
+                const RunRef& A = runs[g];
+                const RunRef& B = runs[g + 1];
+                const int tiles = (int)num_tiles(glen, C.tout());
+                {
+                    TimedScope ts(p, DC_KERNEL_NK2_PARTITION);
+                    dc::nk2_partition_ab<K><<<(tiles + 3) / 4, 128, 0, p->stream>>>(
+                        A.k + A.off, A.len, B.k + B.off, B.len, C.tout(), tiles, split);
+                    DC_LAUNCHED(p);
+                }
+                {
+                    TimedScope ts(p, DC_KERNEL_NK3_MERGE);
+                    k3<<<tiles, C.nt3, nk3_smem_bytes(C, V), p->stream>>>(
+                        A.k, A.v, A.bound, A.off, A.len, B.k, B.v, B.bound, B.off, B.len, dk, dv,
+                        org, split);
+                    DC_LAUNCHED(p);
+                }
+            } else if (glen > 0) {                      // a lone run moves as it is
+                const RunRef& A = runs[g];
+                DC_CUDA(p, cudaMemcpyAsync(dk + org, A.k + A.off, (size_t)A.len * 4,
+                                           cudaMemcpyDeviceToDevice, p->stream));
+                if (V)
+                    DC_CUDA(p, cudaMemcpyAsync(dv + org, A.v + A.off, (size_t)A.len * 4,
+                                               cudaMemcpyDeviceToDevice, p->stream));
             }
-            {
-                TimedScope ts(p, DC_KERNEL_NK3_MERGE);
-                k3<<<tiles, C.nt3, nk3_smem_bytes(C, V), p->stream>>>(
-                    rk[r], V ? rv[r] : nullptr, bound[r], off[r], la, rk[rb],
-                    V ? rv[rb] : nullptr, bound[rb], off[rb], lb, dk, dv, org, split);
-                DC_LAUNCHED(p);
-            }
+            next.push_back({dk, dv, total, org, glen});
+            org += glen;
         }
-        next.push_back(la + lb);
-        org += la + lb;
+        runs.swap(next);
     }
-    if (one_round) return DC_OK;
-    return mg_merge_typed<K, V>(p, tmp_k, tmp_v, out_k, out_v, next);
+    return DC_OK;
+}
+
+// dc_mg_merge_runs: back-to-back runs of one buffer; intermediate rounds
+// ping-pong between the plan scratch and the (clobbered) input.
+template <class K, bool V>
+dc_status mg_merge_typed(dc_plan_t p, uint32_t* in_k, uint32_t* in_v, uint32_t* out_k,
+                         uint32_t* out_v, const std::vector<int64_t>& lens) {
+    int64_t total = 0;
+    for (int64_t l : lens) total += l;
+    std::vector<RunRef> runs;
+    int64_t org = 0;
+    for (int64_t l : lens) {
+        runs.push_back({in_k, in_v, total, org, l});
+        org += l;
+    }
+    dc_status st = ensure_scratch(p, V);
+    if (st != DC_OK) return st;
+    const size_t kb = align_up((size_t)p->n * 4, 256);
+    uint32_t* sk = (uint32_t*)p->scratch;
+    uint32_t* sv = V ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
+    return merge_g<K, V>(p, runs, sk, sv, in_k, in_v, out_k, out_v);
+}
+
+// a8+a9 fused (dc_mg_merge_peers): the first round reads the runs where they
+// lie (peer shards over NVLink); later rounds are local (tmp, then scratch).
+template <class K, bool V>
+dc_status mg_merge_peers_typed(dc_plan_t p, const uint32_t* const* rk, const uint32_t* const* rv,
+                               const int64_t* bound, const int64_t* off, const int64_t* len,
+                               int runs, uint32_t* tmp_k, uint32_t* tmp_v, uint32_t* out_k,
+                               uint32_t* out_v) {
+    std::vector<RunRef> rr;
+    for (int r = 0; r < runs; ++r) rr.push_back({rk[r], V ? rv[r] : nullptr, bound[r], off[r], len[r]});
+    dc_status st = ensure_scratch(p, V);
+    if (st != DC_OK) return st;
+    const size_t kb = align_up((size_t)p->n * 4, 256);
+    uint32_t* sk = (uint32_t*)p->scratch;
+    uint32_t* sv = V ? (uint32_t*)((char*)p->scratch + kb) : nullptr;
+    return merge_g<K, V>(p, rr, tmp_k, tmp_v, sk, sv, out_k, out_v);
 }
 
 dc_status ensure_mg_state(dc_plan_t p) {
@@ -910,7 +954,7 @@ dc_status dc_plan(int64_t n, int32_t a, int32_t b, int64_t base_size, dc_plan_t*
     p->b = b;
     p->base_size = base_size;
     if (const char* e = std::getenv("DC_PIPE_CHUNKS")) p->pipe_chunks = std::atoi(e);  // tuning
-    if (const char* e = std::getenv("DC_TWO_LEVEL")) p->two_level = std::atoi(e) != 0;  // tuning
+    if (const char* e = std::getenv("DC_TWO_LEVEL")) p->two_force = std::atoi(e) != 0;  // tuning
     // Level i: a^i nodes of size ceil(n / b^i); stop at the first level whose
     // size is <= base_size (leaves at level log_b n for base 1).
     int64_t nodes = 1, size = n, bpow = 1;
@@ -947,21 +991,31 @@ dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     if (kt != DC_KEY_U32 && kt != DC_KEY_I32 && kt != DC_KEY_F32)
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
-    const SortCfg c = cfg_for_runtime(kt, with_vals != 0, p->n);
+    const Decision d = decide(p, kt, with_vals != 0);
+    const SortCfg c = cfg_for_runtime(kt, with_vals != 0, d.small);
     if (tile) *tile = c.tile();
     int f = 0;   // levels of the binary tree inside one tile: ceil(log2(tile))
     while ((1 << f) < c.tile()) ++f;
     if (fused_levels) *fused_levels = f;
     const int P = global_passes(p->n, c.tile());
     if (passes) *passes = P;
-    const bool two = p->two_level && P >= 2 && p->n >= kSmallN;
+    const bool two = d.two && P >= 2;
     if (hbm_passes) *hbm_passes = two ? (P % 2) + (P - P % 2) / 2 : P;
     return DC_OK;
 }
 
 dc_status dc_plan_set_two_level(dc_plan_t p, int32_t enable) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
-    p->two_level = enable != 0;
+    if (enable < -1 || enable > 1) return fail(DC_ERR_INVALID_ARG, "enable must be -1, 0 or 1");
+    p->two_force = enable;
+    drop_graphs(p);
+    return DC_OK;
+}
+
+dc_status dc_plan_set_tile_class(dc_plan_t p, int32_t tile_class) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (tile_class < 0 || tile_class > 2) return fail(DC_ERR_INVALID_ARG, "tile_class must be 0, 1 or 2");
+    p->tile_class = tile_class;
     drop_graphs(p);
     return DC_OK;
 }
@@ -1361,7 +1415,7 @@ dc_status dc_mg_merge_peers(dc_plan_t p, dc_key_type kt, const uint32_t* const* 
     if (st != DC_OK) return st;
     const bool v = d_out_vals != nullptr;
     if (!h_run_keys || !h_bound || !h_off || !h_len || runs < 1 || !d_out_keys ||
-        (v && !h_run_vals) || (runs > 2 && (!d_tmp_keys || (v && !d_tmp_vals))))
+        (v && !h_run_vals) || (runs > 4 && (!d_tmp_keys || (v && !d_tmp_vals))))
         return fail(DC_ERR_INVALID_ARG, "bad peer-merge arguments");
     for (int r = 0; r < runs; ++r) {
         if (!h_run_keys[r] || !aligned16(h_run_keys[r]) ||

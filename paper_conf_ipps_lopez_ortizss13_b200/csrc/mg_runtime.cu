@@ -548,23 +548,16 @@ dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, u
     const int64_t* cm = c->h_pin;
     c->last_cmat.assign(cm, cm + (size_t)G * (G + 1));
     std::vector<int64_t> scnt(G), soff(G), rcnt(G), roff(G);
-    int64_t tot = 0;
-    for (int d = 0; d < G; ++d) {
-        soff[d] = cm[me * (G + 1) + d];
-        scnt[d] = cm[me * (G + 1) + d + 1] - soff[d];
-        rcnt[d] = cm[d * (G + 1) + me + 1] - cm[d * (G + 1) + me];
-        roff[d] = tot;
-        tot += rcnt[d];
-        if (scnt[d] < 0 || rcnt[d] < 0) return fail(DC_ERR_BAD_STATE, "negative split size");
-    }
-    if (tot != m) return fail(DC_ERR_BAD_STATE, "received element count != shard size");
+    if (dc_mg_exchange_sizes(cm, G, me, m, scnt.data(), soff.data(), rcnt.data(), roff.data()) !=
+        DC_OK)
+        return fail(DC_ERR_BAD_STATE, std::string("inconsistent split matrix: ") + dc_last_error());
     c->moved = m - rcnt[me];
     c->moved_total += c->moved;
     MG_TRY(mark(p, c, 2));                 // splitters done (host-synchronised above)
     const size_t kb = al256((size_t)m * 4);
     if (c->p2p == 1) {
         // a8+a9 fused: merge straight from the peers' shards (NVLink reads)
-        if (G > 2) MG_TRY(ensure_recv(c, vals != nullptr));
+        if (G > 4) MG_TRY(ensure_recv(c, vals != nullptr));   // intermediate round
         std::vector<const uint32_t*> rk(G), rv(G);
         std::vector<int64_t> bound(G, m), off(G);
         for (int d = 0; d < G; ++d) {
@@ -572,8 +565,8 @@ dc_status sort_exchange(dc_plan_t p, MgCtx* c, dc_key_type kt, uint32_t* keys, u
             rv[d] = (const uint32_t*)((const char*)c->peers[d] + kb);
             off[d] = cm[d * (G + 1) + me];
         }
-        uint32_t* tk = G > 2 ? c->recv : nullptr;
-        uint32_t* tv = (G > 2 && vals) ? (uint32_t*)((char*)c->recv + kb) : nullptr;
+        uint32_t* tk = G > 4 ? c->recv : nullptr;
+        uint32_t* tv = (G > 4 && vals) ? (uint32_t*)((char*)c->recv + kb) : nullptr;
         MG_TRY(dc_mg_merge_peers(p, kt, rk.data(), vals ? rv.data() : nullptr, bound.data(),
                                  off.data(), rcnt.data(), G, tk, tv, out_k, out_v));
         // nobody rewrites its shard (next sort) while a peer may still read it
@@ -805,6 +798,32 @@ dc_status dc_plan_mg_reset_phases(dc_plan_t p) {
     for (double& v : p->mg->phase_ms) v = 0;
     p->mg->phase_n = 0;
     p->mg->moved_total = 0;
+    return DC_OK;
+}
+
+dc_status dc_mg_exchange_sizes(const int64_t* cm, int32_t world, int32_t rank, int64_t shard_n,
+                               int64_t* scnt, int64_t* soff, int64_t* rcnt, int64_t* roff) {
+    if (!cm || !scnt || !soff || !rcnt || !roff || world < 1 || rank < 0 || rank >= world ||
+        shard_n < 0)
+        return dcx::fail(DC_ERR_INVALID_ARG, "bad exchange-size arguments");
+    const int G = world;
+    for (int r = 0; r < G; ++r) {
+        if (cm[r * (G + 1)] != 0 || cm[r * (G + 1) + G] != shard_n)
+            return dcx::fail(DC_ERR_INVALID_ARG, "split-matrix row must run from 0 to shard_n");
+        for (int d = 0; d < G; ++d)
+            if (cm[r * (G + 1) + d + 1] < cm[r * (G + 1) + d])
+                return dcx::fail(DC_ERR_INVALID_ARG, "split-matrix row not monotone");
+    }
+    int64_t tot = 0;
+    for (int d = 0; d < G; ++d) {
+        soff[d] = cm[rank * (G + 1) + d];                       // my elements for rank d
+        scnt[d] = cm[rank * (G + 1) + d + 1] - soff[d];
+        rcnt[d] = cm[d * (G + 1) + rank + 1] - cm[d * (G + 1) + rank];   // rank d's for me
+        roff[d] = tot;                                          // runs land in rank order
+        tot += rcnt[d];
+    }
+    if (tot != shard_n)
+        return dcx::fail(DC_ERR_INVALID_ARG, "received element count != shard size");
     return DC_OK;
 }
 

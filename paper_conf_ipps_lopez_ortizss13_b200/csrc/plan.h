@@ -66,7 +66,10 @@ struct dc_plan_s {
     // Off by default: bit-exact, and its 4-way tile merge beats two one-level
     // passes (0.545 vs 0.626 ms per two levels at 2^28), but the exact
     // two-level partition costs 0.21 ms per pass vs 2 x 0.03.
-    bool two_level = true;    // 4-way passes for large keys-only sorts (sort4_kernels.cuh)
+    // Schedule of the sort (the planner, model.cu, picks the tile
+    // class and the pass kind per (n, key type, values) unless overridden)
+    int two_force = -1;       // -1 planner; 0 one level per HBM pass; 1 two levels (4-way)
+    int tile_class = 0;       // 0 planner; 1 quarter-size tiles; 2 full tiles
     bool fuse_partition = true;   // small sorts: merge CTAs find their own co-ranks
     // D&C sum (f4): per-CTA parts + ticket + result
     long long* sum_state = nullptr;
@@ -94,7 +97,7 @@ struct dc_plan_s {
     dcx::MgCtx* mg = nullptr;
     int64_t n_global = 0;
     int64_t mg_stride = 4096;   // splitter sample stride S
-    bool mg_p2p = true;         // fused exchange (peer reads) when every rank can map every peer
+    bool mg_p2p = false;        // fused exchange (peer reads); NCCL all-to-all until measured across GPUs
     // per-kernel CUDA-event timing (instrumentation, off by default)
     bool timing = false;
     struct Timed { int kind; cudaEvent_t e0, e1; };

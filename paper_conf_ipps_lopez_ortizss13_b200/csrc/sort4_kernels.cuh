@@ -23,6 +23,12 @@
 // empty); tile j is local tile j % tpg of group j / tpg.  Positions inside a
 // group fit in int32 (n < 2^31).
 //
+// The same kernels merge ONE group of four runs of arbitrary lengths that
+// live in separate buffers (Pass4 custom mode): the local G-way merge of the
+// multi-GPU sort (a9, Alg 7's top levels) reads up to four received runs --
+// or four peer GPUs' sorted shards over NVLink, the exchange fused into the
+// merge -- and writes their stable merge in one HBM pass.
+//
 // Keys-only (u32 / i32): equal keys are identical bit patterns, so the merges
 // use +inf pads instead of bounds checks (see merge_pad).
 #pragma once
@@ -34,25 +40,55 @@ struct Cut4 {
     int c[4];
 };
 
-// Tile j of a two-level pass over runs of width w in [0, n): its group start
-// s, the four run lengths, the group length and the tile's output range
-// [d0, d1) relative to s (empty when d0 >= tot, in the last group).
+// The runs of one two-level pass.
+//   uniform (custom == 0): groups of four adjacent runs of width w over
+//     [0, n) of one buffer (k[q] = src, v[q] = src values, bound[q] = n);
+//   custom  (custom == 1): ONE group; run q is len[q] elements at offset
+//     off[q] of buffer k[q] (+ v[q]), readable for bound[q] elements, and the
+//     merged group goes to dst[out0, out0 + sum len).
+// Buffer bases are 16-byte aligned (TMA); they may be peer-GPU mappings.
+struct Pass4 {
+    const uint32_t* k[4];
+    const uint32_t* v[4];
+    long long bound[4];
+    long long off[4];
+    long long len[4];
+    long long n, w, out0;
+    int T, tpg, custom;
+};
+
+// Tile j of a pass: the start of each run in its buffer, the four run
+// lengths, the group length, the group's output offset o and the tile's
+// output range [d0, d1) relative to o (empty when d0 >= tot, in the last
+// group of a uniform pass).
 struct Tile4Geo {
-    long long s;
+    long long st[4];
+    long long o;
     int l[4];
     int tot, d0, d1;
-    __device__ __forceinline__ Tile4Geo(long long n, long long w, int T, int tpg, int j) {
-        const int G = j / tpg;
-        s = (long long)G * 4 * w;
+    __device__ __forceinline__ Tile4Geo(const Pass4& P, int j) {
+        const int G = P.custom ? 0 : j / P.tpg;
         tot = 0;
+        if (P.custom) {
+            o = P.out0;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            l[q] = (int)max(0LL, min(w, n - s - q * w));
-            tot += l[q];
+            for (int q = 0; q < 4; ++q) {
+                st[q] = P.off[q];
+                l[q] = (int)P.len[q];
+                tot += l[q];
+            }
+        } else {
+            o = (long long)G * 4 * P.w;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                st[q] = o + q * P.w;
+                l[q] = (int)max(0LL, min(P.w, P.n - o - q * P.w));
+                tot += l[q];
+            }
         }
-        const long long e0 = (long long)(j - G * tpg) * T;   // may pass tot (empty tile)
+        const long long e0 = (long long)(j - G * P.tpg) * P.T;   // may pass tot (empty tile)
         d0 = (int)min(e0, (long long)tot);
-        d1 = (int)min(e0 + T, (long long)tot);
+        d1 = (int)min(e0 + P.T, (long long)tot);
     }
 };
 
@@ -92,22 +128,20 @@ __device__ __forceinline__ int sel4_pivot(int lo, int W, int step, int t) {
 // group) or !valid gets the zero cut; its lanes still take part in the
 // warp's shuffles until every group of the warp is done.
 template <class K, int PV = 8>
-__device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, long long n,
-                                             long long w, int T, int tpg, int j,
-                                             bool valid = true) {
+__device__ __forceinline__ Cut4 select4_warp(const Pass4& P, int j, bool valid = true) {
     static_assert(PV == 8 || PV == 4 || PV == 2, "8, 4 or 2 pivots per run (1, 2, 4 boundaries per warp)");
     constexpr int LB = 4 * PV;
     const int lane = threadIdx.x & 31;
     const int base = lane & ~(LB - 1);                 // first lane of this boundary's group
     const int ll = lane - base;
     const int q = ll / PV, t = ll % PV;
-    const Tile4Geo g(n, w, T, tpg, valid ? j : 0);
+    const Tile4Geo g(P, valid ? j : 0);
     const int d = g.d0;
     const bool live = valid && d < g.tot;
     if (PV == 8 && !live) return Cut4{{0, 0, 0, 0}}; // whole warp: uniform exit
     const uint32_t* R[4];
 #pragma unroll
-    for (int r = 0; r < 4; ++r) R[r] = src + g.s + r * w;
+    for (int r = 0; r < 4; ++r) R[r] = P.k[r] + g.st[r];
     const uint32_t* Rq = R[0];
 #pragma unroll
     for (int r = 1; r < 4; ++r)
@@ -247,17 +281,16 @@ __device__ __forceinline__ Cut4 select4_warp(const uint32_t* __restrict__ src, l
 template <int PV>
 constexpr int sel4_bpw() { return 32 / (4 * PV); }
 template <class K, int PV>
-__global__ void nk2_select4(const uint32_t* __restrict__ src, long long n, long long w, int T,
-                            int tpg, int num_tiles, Cut4* __restrict__ cut) {
+__global__ void nk2_select4(const Pass4 P, int num_tiles, Cut4* __restrict__ cut) {
     constexpr int LB = 4 * PV, BPW = 32 / LB;
     const int wj = (int)(((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * BPW;
     if (wj >= num_tiles) return;                      // warp-uniform
     const int lane = threadIdx.x & 31;
     const int j = wj + lane / LB;
     const bool valid = j < num_tiles;
-    const Cut4 c = select4_warp<K, PV>(src, n, w, T, tpg, j, valid);
+    const Cut4 c = select4_warp<K, PV>(P, j, valid);
     if (valid && lane % LB == 0) {
-        const Tile4Geo g(n, w, T, tpg, j);
+        const Tile4Geo g(P, j);
         if (g.d0 < g.tot) cut[j] = c;                 // (empty tiles: no cut)
     }
 }
@@ -325,17 +358,9 @@ __device__ __forceinline__ void consumer_sync() {
 // ahead.  full[b]: tile data present (producer arrive + TMA bytes);
 // empty[b]: output written (one arrive per consumer warp).  Tiles
 // J = blockIdx.x + i * gridDim.x; empty tiles (end of the last group) pass
-// through with no work.
-//
-// NSEL > 0 fuses NK2-4 into the pass: the CTA owns a contiguous tile range
-// [t0, t1), and NSEL selector warps compute the cuts of its boundaries
-// t0 .. t1 (boundary i by warp i % NSEL) into a ring of RS slots in shared
-// memory, running ahead of the producer.  cfull[s]: cut written (selector
-// lane 0 arrives); cempty[s]: the producer has filled the tile that starts
-// at that boundary (it waits for every boundary in order, so each slot is
-// at most one phase ahead).  The standalone select launch and its ~11
-// dependent rounds per boundary move off the critical path, except for the
-// CTA's first two boundaries.
+// through with no work.  (An in-kernel selection -- selector warps filling a
+// cut ring ahead of the producer -- was measured slower than the separate
+// NK2-4 launch and removed.)
 //
 // Keys-only u32/i32 (equal keys indistinguishable): pad-safe merges and a
 // bitonic stage 2 (Y stored descending), no bounds checks.  Stable variants
@@ -345,11 +370,10 @@ __device__ __forceinline__ void consumer_sync() {
 #ifndef DC_M4_MINB   // CTAs per SM the register budget is sized for
 #define DC_M4_MINB 1
 #endif
-template <int NT, int IT, class K, bool V, int NSEL = 0>
-__global__ void __launch_bounds__(NT + 64 + 32 * NSEL, DC_M4_MINB)
-nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_v,
-           uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v, long long n, long long w,
-           int tpg, const Cut4* __restrict__ cut, int num_tiles) {
+template <int NT, int IT, class K, bool V>
+__global__ void __launch_bounds__(NT + 64, DC_M4_MINB)
+nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v,
+           const Cut4* __restrict__ cut, int num_tiles) {
     static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
     constexpr bool kStable = V || K::kNeedStable;
     constexpr int T = NT * IT;
@@ -358,23 +382,15 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
     constexpr int BW = (V ? 2 : 1) * KW;               // words per buffer
     constexpr int GU = m4_guard(IT);
     constexpr uint32_t VOFF = 4u * KW;                 // key -> value byte offset
-    constexpr int RS = NSEL > 0 ? 3 * NSEL : 1;        // cut ring slots (multiple of NSEL)
     extern __shared__ __align__(16) uint32_t sm[];
     __shared__ __align__(8) uint64_t full[2], empty[2];
-    __shared__ __align__(8) uint64_t cfull[RS], cempty[RS];
     __shared__ Tile4 meta[2];
-    __shared__ Cut4 ring[RS];
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     const uint32_t SM0 = smem_addr(sm);
-    const long long n4 = n & ~3LL;
-    // tile i of this CTA: interleaved (cuts from NK2-4) or a contiguous range
-    const int t0 = NSEL > 0 ? (int)(((long long)blockIdx.x * num_tiles) / gridDim.x) : 0;
-    const int t1 = NSEL > 0 ? (int)(((long long)(blockIdx.x + 1) * num_tiles) / gridDim.x) : 0;
-    const int my_tiles = NSEL > 0 ? t1 - t0
-                         : ((int)blockIdx.x < num_tiles
-                                ? (num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0);
-    auto tile_of = [&](int i) { return NSEL > 0 ? t0 + i : (int)blockIdx.x + i * (int)gridDim.x; };
+    const int my_tiles = (int)blockIdx.x < num_tiles
+                             ? (num_tiles - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+    auto tile_of = [&](int i) { return (int)blockIdx.x + i * (int)gridDim.x; };
 
     if (tid == 0) {
 #pragma unroll
@@ -382,53 +398,26 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
             mbar_init(smem_addr(&full[b]), 1);
             mbar_init(smem_addr(&empty[b]), NC / 32);
         }
-        if (NSEL > 0) {
-            for (int r = 0; r < RS; ++r) {
-                mbar_init(smem_addr(&cfull[r]), 1);
-                mbar_init(smem_addr(&cempty[r]), 1);
-            }
-        }
     }
     __syncthreads();
-
-    if (NSEL > 0 && tid >= NC + 32) {
-        // ---------------------------------------------------- selector warps
-        const int sw = (tid - NC - 32) >> 5;
-        for (int i = sw; i <= my_tiles; i += NSEL) {
-            const int slot = i % RS, rnd = i / RS;
-            if (rnd > 0) mbar_wait(smem_addr(&cempty[slot]), (uint32_t)((rnd - 1) & 1));
-            const Cut4 c = select4_warp<K>(src_k, n, w, T, tpg, t0 + i);
-            if (lane == 0) {
-                ring[slot] = c;
-                mbar_arrive(smem_addr(&cfull[slot]));   // release: the cut
-            }
-            __syncwarp();
-        }
-        return;
-    }
 
     if (tid >= NC) {
         // ------------------------------------------------------ producer warp
         // Fill buffer b with tile J: cut vectors (start; end = next tile's
         // start or the run lengths at the end of a group) -> pieces.  The TMA
-        // copies each piece's 16-byte-aligned interior [g0 & ~3, tend); the
-        // lanes store the ragged end (< 4 words, or the part at/after n4) and
-        // IT pads behind each piece.
+        // copies each piece's 16-byte-aligned interior [g0 & ~3, tend) from its
+        // run's buffer; the lanes store the ragged end (< 4 words, or the part
+        // at/after the buffer's aligned bound) and IT pads behind each piece.
         auto fill = [&](int i, int b) {
             const int J = tile_of(i);
-            const Tile4Geo g(n, w, T, tpg, J);
+            const Tile4Geo g(P, J);
             int c0[4], c1[4];
-            if (NSEL > 0)   // boundary i, in order (see the ring protocol above)
-                mbar_wait(smem_addr(&cfull[i % RS]), (uint32_t)((i / RS) & 1));
             if (g.d0 < g.tot) {
-                const Cut4 a = NSEL > 0 ? ring[i % RS] : cut[J];
+                const Cut4 a = cut[J];
                 Cut4 e;
                 if (g.d1 == g.tot) {
 #pragma unroll
                     for (int r = 0; r < 4; ++r) e.c[r] = g.l[r];
-                } else if (NSEL > 0) {
-                    mbar_wait(smem_addr(&cfull[(i + 1) % RS]), (uint32_t)(((i + 1) / RS) & 1));
-                    e = ring[(i + 1) % RS];
                 } else {
                     e = cut[J + 1];
                 }
@@ -438,12 +427,8 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
 #pragma unroll
                 for (int r = 0; r < 4; ++r) c0[r] = c1[r] = 0;
             }
-            if (NSEL > 0) {      // boundary i is dead once every lane has read it
-                __syncwarp();
-                if (lane == 0) mbar_arrive(smem_addr(&cempty[i % RS]));
-            }
             Tile4 m;
-            m.out = g.s + g.d0;
+            m.out = g.o + g.d0;
             m.total = max(0, g.d1 - g.d0);
             uint32_t* buf = sm + b * BW + GU;
             const uint32_t base = SM0 + 4u * (b * BW + GU);
@@ -452,9 +437,11 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
             int o = 0;
 #pragma unroll
             for (int r = 0; r < 4; ++r) {
-                m.g0[r] = g.s + r * w + c0[r];
+                const uint32_t* rk = P.k[r];
+                m.g0[r] = g.st[r] + c0[r];
                 m.len[r] = c1[r] - c0[r];
                 m.at[r] = o + (int)(m.g0[r] & 3);
+                const long long n4 = P.bound[r] & ~3LL;
                 const long long al0 = m.g0[r] & ~3LL;
                 long long al1 = (m.g0[r] + m.len[r]) & ~3LL;
                 if (al1 > n4) al1 = n4;
@@ -465,8 +452,8 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
                 const int e0 = (int)(max(al1, m.g0[r]) - m.g0[r]);
                 for (int e = e0 + lane; e < m.len[r] + IT; e += 32) {
                     const bool real = e < m.len[r];
-                    buf[m.at[r] + e] = real ? src_k[m.g0[r] + e] : K::kPad;
-                    if (V) buf[KW + m.at[r] + e] = real ? src_v[m.g0[r] + e] : 0u;
+                    buf[m.at[r] + e] = real ? rk[m.g0[r] + e] : K::kPad;
+                    if (V) buf[KW + m.at[r] + e] = real ? P.v[r][m.g0[r] + e] : 0u;
                 }
             }
             __syncwarp();
@@ -480,8 +467,8 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
                     if (tend[r] > al0) {
                         const uint32_t d = base + 4u * (m.at[r] - (int)(m.g0[r] & 3));
                         const uint32_t nb = (uint32_t)(4 * (tend[r] - al0));
-                        bulk_g2s(d, src_k + al0, nb, fb);
-                        if (V) bulk_g2s(d + VOFF, src_v + al0, nb, fb);
+                        bulk_g2s(d, P.k[r] + al0, nb, fb);
+                        if (V) bulk_g2s(d + VOFF, P.v[r] + al0, nb, fb);
                     }
                 }
             }
@@ -493,11 +480,16 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
             mbar_wait(smem_addr(&empty[b]), (i >> 1) & 1);   // output of tile i written
             if (lane == 0) {
                 const Tile4 m = meta[b];
-                const int body = m.total & ~3;
+                // output element e sits at buffer word h + e (h = m.out mod 4),
+                // so the 16-byte-aligned body [head, head + body) is aligned on
+                // both sides of the bulk store; head and tail left by plain stores
+                const int h = (int)(m.out & 3);
+                const int head = min(m.total, (4 - h) & 3);
+                const int body = (m.total - head) & ~3;
                 if (body > 0) {
-                    const uint32_t sb = SM0 + 4u * (b * BW + GU);
-                    bulk_s2g(dst_k + m.out, sb, 4u * body);
-                    if (V) bulk_s2g(dst_v + m.out, sb + VOFF, 4u * body);
+                    const uint32_t sb = SM0 + 4u * (b * BW + GU + h + head);
+                    bulk_s2g(dst_k + m.out + head, sb, 4u * body);
+                    if (V) bulk_s2g(dst_v + m.out + head, sb + VOFF, 4u * body);
                     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
                 }
                 if (i + 2 < my_tiles) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
@@ -612,26 +604,31 @@ nk3_merge4(const uint32_t* __restrict__ src_k, const uint32_t* __restrict__ src_
             }
         }
         consumer_sync<NC>();
-        // output back into the buffer (the producer bulk-stores the 16-byte
-        // body); the < 4-word tail of a short tile straight from registers
-        // (tile outputs start at multiples of 4 words: T and 4w are)
-        const int body = total & ~3;
+        // output back into the buffer at word h + e (the producer bulk-stores
+        // the 16-byte-aligned body); the < 4-word head (custom passes may
+        // start anywhere) and tail straight from registers.  Uniform passes
+        // start at multiples of 4 words (T and 4w are): h = head = 0.
+        const int h = (int)(m.out & 3);
+        const int head = min(total, (4 - h) & 3);
+        const int bend = head + ((total - head) & ~3);
         if (act2) {
-            if (diag + IT <= body) {
+            uint32_t* ob = buf + h;
+            if (diag >= head && diag + IT <= bend) {
 #pragma unroll
                 for (int q = 0; q < IT; ++q) {
-                    buf[diag + q] = k[q];
-                    if (V) buf[KW + diag + q] = vv[q];
+                    ob[diag + q] = k[q];
+                    if (V) ob[KW + diag + q] = vv[q];
                 }
             } else {
 #pragma unroll
                 for (int q = 0; q < IT; ++q) {
-                    if (diag + q < body) {
-                        buf[diag + q] = k[q];
-                        if (V) buf[KW + diag + q] = vv[q];
-                    } else if (diag + q < total) {
-                        dst_k[m.out + diag + q] = k[q];
-                        if (V) dst_v[m.out + diag + q] = vv[q];
+                    const int e = diag + q;
+                    if (e >= head && e < bend) {
+                        ob[e] = k[q];
+                        if (V) ob[KW + e] = vv[q];
+                    } else if (e < total) {
+                        dst_k[m.out + e] = k[q];
+                        if (V) dst_v[m.out + e] = vv[q];
                     }
                 }
             }

@@ -101,21 +101,35 @@ def test_run_validation_before_device_work():
     assert dc.lib().dc_run_mergesort(p._h, 7, ctypes.c_void_p(0x1000), None) == 1   # key type
 
 
-@pytest.mark.parametrize("n", [1, 100, 8192, 8193, 1 << 20, 1 << 28, (1 << 31) - 1])
+@pytest.mark.parametrize("n", [1, 100, 8192, 8193, 1 << 20, 1 << 23, 1 << 28, (1 << 31) - 1])
 @pytest.mark.parametrize("kt,vals", [("u32", False), ("i32", False), ("f32", False), ("u32", True)])
 def test_schedule(n, kt, vals):
+    """dc_plan_schedule reports the planner's choice (dc_model_sort_schedule),
+    with the level counts of the recurrence: fused = ceil(log2 tile) levels on
+    chip, P = ceil(log2 ceil(n / tile)) levels above, in P passes (one level
+    each) or P mod 2 + P div 2 passes (two levels per pass)."""
     s = dc.Plan(n).schedule(kt, vals)
+    m = dc.model_sort_schedule(n, kt, vals)
     t = s["tile"]
-    assert s["fused_levels"] == math.ceil(math.log2(t))
-    assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t))))
-    # large sorts (n >= 2^23) fold two levels per HBM pass by default (f1);
-    # small n (small tiles) runs one level per pass
+    assert t == m["tile"] and s["hbm_passes"] == m["hbm_passes"]
+    assert s["fused_levels"] == math.ceil(math.log2(t)) == m["fused_levels"]
+    assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t)))) == m["global_levels"]
     P = s["global_passes"]
-    folds = not (P < 2 or n < (1 << 23))
-    assert s["hbm_passes"] == (P % 2 + P // 2 if folds else P)
-    p2 = dc.Plan(n)
-    p2.set_two_level(False)
-    assert p2.schedule(kt, vals)["hbm_passes"] == P
+    assert s["hbm_passes"] == (P % 2 + P // 2 if (m["two_level"] and P >= 2) else P)
+    assert m["predicted_ms"] == min(v for v in m["candidates_ms"].values())
+    # forced choices are honoured and reported
+    for tc in (1, 2):
+        for two in (False, True):
+            p2 = dc.Plan(n)
+            p2.set_tile_class(tc)
+            p2.set_two_level(two)
+            s2 = p2.schedule(kt, vals)
+            m2 = dc.model_sort_schedule(n, kt, vals, tile_class=tc, two_level=int(two))
+            assert (m2["tile_class"], m2["two_level"]) == (tc, two)
+            assert s2["tile"] == m2["tile"] and s2["hbm_passes"] == m2["hbm_passes"]
+            assert s2["hbm_passes"] == (s2["global_passes"] % 2 + s2["global_passes"] // 2
+                                        if two and s2["global_passes"] >= 2
+                                        else s2["global_passes"])
     # fused + global levels cover the whole tree: ceil(log2 n) combine levels
     if n > 1:
         assert s["fused_levels"] + s["global_passes"] >= math.ceil(math.log2(n))

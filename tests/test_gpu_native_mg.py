@@ -119,12 +119,21 @@ def test_loopback_keys_only(dc, oracle_mod, key_type, stride):
     sort_case(dc, oracle_mod, 4 * 250_001, 4, "paper", key_type, False, stride)
 
 
-@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("world", [2, 4, 8])
 @pytest.mark.parametrize("stride", [1001, 333])
 def test_loopback_odd_stride(dc, oracle_mod, world, stride):
     """odd sample strides with an even world size: every rank's
     send buffer (int64 headers) must stay aligned in the all-gathered array."""
     sort_case(dc, oracle_mod, world * 120_007, world, "uniform", "u32", True, stride)
+
+
+@pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
+@pytest.mark.parametrize("world", [4, 8])
+def test_loopback_many_ranks_large(dc, oracle_mod, p2p, world):
+    """2^24 keys over 4 / 8 ranks: the G-way merge is one 4-way pass (G = 4)
+    or a 4-way pass per group of four plus a pair pass (G = 8); in fused mode
+    the 4-way pass reads four peers' shards directly."""
+    sort_case(dc, oracle_mod, 1 << 24, world, "uniform", "u32", False, 4096, p2p=p2p)
 
 
 @pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
@@ -226,12 +235,16 @@ def test_nccl_world1_sort_and_maxsub(dc, oracle_mod):
 
 
 @pytest.mark.parametrize("key_type", ["u32", "i32", "f32"])
-@pytest.mark.parametrize("runs", [1, 2, 3, 4, 7])
-def test_merge_peers_separate_buffers(dc, oracle_mod, key_type, runs):
+@pytest.mark.parametrize("runs", [1, 2, 3, 4, 5, 7, 8, 16, 17])
+@pytest.mark.parametrize("with_vals", [True, False])
+def test_merge_peers_separate_buffers(dc, oracle_mod, key_type, runs, with_vals):
     """dc_mg_merge_peers on runs that each live in their own buffer at an
-    arbitrary offset (unaligned starts, ragged lengths, empty runs)."""
+    arbitrary offset (unaligned starts, ragged lengths, empty runs): groups of
+    four runs in one 4-way pass read straight from their buffers (outputs at
+    unaligned offsets when G > 4), pairs in one pair-mode pass, lone runs
+    copied; keys only (pad-safe 4-way merges for u32/i32) and with values."""
     rng = np.random.default_rng(runs)
-    lens = [int(rng.integers(0, 40_000)) for _ in range(runs)]
+    lens = [int(rng.integers(0, 40_000 if runs < 8 else 90_000)) for _ in range(runs)]
     if runs > 2:
         lens[1] = 0
     total = sum(lens)
@@ -256,14 +269,17 @@ def test_merge_peers_separate_buffers(dc, oracle_mod, key_type, runs):
     out_v = torch.empty(max(total, 1), dtype=torch.int32, device="cuda")
     tk = torch.empty_like(out_k)
     tv = torch.empty_like(out_v)
-    plan.mg_merge_peers([(bufs[r], vbufs[r], offs[r], lens[r]) for r in range(runs)],
-                        out_k, out_v, tk, tv, key_type=key_type)
+    if not with_vals:
+        out_v = tv = None
+    plan.mg_merge_peers([(bufs[r], vbufs[r] if with_vals else None, offs[r], lens[r])
+                         for r in range(runs)], out_k, out_v, tk, tv, key_type=key_type)
     cat_k = np.concatenate(allk)
     cat_v = np.concatenate(allv)
     ek, ev = oracle_mod.mergesort(cat_k, cat_v, key_type=key_type)   # stable: earlier run wins
     got = out_k[:total].cpu().numpy().view(view)
     assert np.array_equal(got.view(np.uint32), ek.view(np.uint32))
-    assert np.array_equal(out_v[:total].cpu().numpy().view(np.uint32), ev)
+    if with_vals:
+        assert np.array_equal(out_v[:total].cpu().numpy().view(np.uint32), ev)
 
 
 @pytest.mark.parametrize("p2p", [True, False], ids=["fused", "alltoall"])
@@ -290,3 +306,33 @@ def test_loopback_phase_times(dc, p2p):
         assert ph["sorts"] == 1
         assert ph["keys_received"] == m - (cm[r][r + 1] - cm[r][r])
         assert ph["local_sort"] > 0 and ph["splitters"] > 0 and ph["exchange_merge"] > 0
+
+
+@pytest.mark.parametrize("runs", [[5], [3, 0, 7], [1000, 1, 2, 50_000, 7, 0, 13], [40_000] * 4,
+                                  [40_000] * 8, [60_001, 3, 77_777, 50_000, 0, 9, 25_344, 1],
+                                  [20_000] * 16, [9_999] * 17])
+@pytest.mark.parametrize("key_type,with_vals", [("u32", True), ("u32", False), ("i32", False),
+                                                ("f32", True)])
+def test_merge_runs_kernel(dc, oracle_mod, runs, key_type, with_vals):
+    """dc_mg_merge_runs (a9): back-to-back sorted runs -> their stable merge
+    (earlier runs win ties) in ceil(log4 G) passes, bit for bit against the
+    oracle's stable sort of the concatenation."""
+    total = sum(runs)
+    view = {"u32": np.uint32, "i32": np.int32, "f32": np.float32}[key_type]
+    parts, off = [], 0
+    for r in runs:
+        k = dcgen.sort_keys(total, "few", seed=31, key_type=key_type, start=off,
+                            count=r).numpy().view(view)
+        parts.append(np.sort(k, kind="stable"))
+        off += r
+    keys_in = np.concatenate(parts)
+    vals_in = np.arange(total, dtype=np.uint32)
+    ik = torch.from_numpy(keys_in.view(np.int32).copy()).cuda()
+    iv = torch.from_numpy(vals_in.view(np.int32).copy()).cuda() if with_vals else None
+    ok = torch.empty_like(ik)
+    ov = torch.empty_like(iv) if with_vals else None
+    dc.Plan(total).mg_merge_runs(ik, iv, ok, ov, runs, key_type=key_type)
+    ek, ev = oracle_mod.mergesort(keys_in, vals_in, key_type=key_type)
+    assert np.array_equal(ok.cpu().numpy().view(np.uint32), ek.view(np.uint32))
+    if with_vals:
+        assert np.array_equal(ov.cpu().numpy().view(np.uint32), ev)

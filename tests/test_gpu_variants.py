@@ -25,7 +25,9 @@ sys.path.insert(0, {root!r})
 import dcgen, oracle
 import paper_conf_ipps_lopez_ortizss13_b200 as dc
 oracle.build()
-sch = dc.Plan(1 << 23).schedule("u32")
+p0 = dc.Plan(1 << 23)
+p0.set_tile_class(2)
+sch = p0.schedule("u32")
 assert sch["tile"] == 25088, sch
 for n, dist, kt, vals in [((1 << 23) + 12345, "uniform", "u32", False),
                           (2 * 25088 * 5 + 7, "few", "u32", False),
@@ -40,6 +42,7 @@ for n, dist, kt, vals in [((1 << 23) + 12345, "uniform", "u32", False),
     else:
         ek = oracle.mergesort(ka, key_type=kt)
     plan = dc.Plan(n)
+    plan.set_tile_class(2)
     plan.set_two_level(False)
     plan.sort_(keys, v, key_type=kt)
     torch.cuda.synchronize()
@@ -60,47 +63,6 @@ def test_one_level_tiles_not_dividing_pairs(tmp_path):
                       defines=["DC_FAST_NT3=160", "DC_STABLE_NT3=160"])
     env = dict(os.environ, DC_LIB=lib)
     r = subprocess.run([sys.executable, "-c", SCRIPT.format(root=ROOT)], env=env,
-                       capture_output=True, text=True, timeout=900)
-    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
-    assert "variant ok" in r.stdout
-
-
-FUSED_SELECT_SCRIPT = r"""
-import sys
-import numpy as np
-import torch
-sys.path.insert(0, {root!r})
-import dcgen, oracle
-import paper_conf_ipps_lopez_ortizss13_b200 as dc
-oracle.build()
-for n, dist, kt in [((1 << 23) + 12345, "uniform", "u32"), ((1 << 24) + 7, "few", "u32"),
-                    ((1 << 23) + 99, "sorted", "i32"), (5 * (1 << 22) + 3, "equal", "u32")]:
-    keys = dcgen.sort_keys(n, dist, seed=43, key_type=kt, device="cuda")
-    ka = keys.cpu().numpy()
-    ka = ka.view(np.uint32) if kt == "u32" else ka.view(np.int32)
-    ek = oracle.mergesort(ka, key_type=kt)
-    plan = dc.Plan(n)
-    sch = plan.schedule(kt)
-    assert sch["hbm_passes"] < sch["global_passes"], sch   # 4-way passes run
-    plan.sort_(keys, key_type=kt)
-    torch.cuda.synchronize()
-    assert np.array_equal(keys.cpu().numpy().view(ek.dtype), ek), (n, dist, kt)
-    assert plan.launch_count() == 1 + sch["hbm_passes"] + (sch["global_passes"] % 2), plan.launch_count()
-print("variant ok")
-"""
-
-
-def test_two_level_fused_selection(tmp_path):
-    """nk3_merge4 with in-kernel selector warps (-DDC_M4_NSEL=3): cuts computed
-    into a shared-memory ring ahead of the producer; bit-exact, one launch per
-    two-level pass."""
-    if not torch.cuda.is_available():
-        pytest.skip("no CUDA device")
-    from paper_conf_ipps_lopez_ortizss13_b200 import build
-
-    lib = build.build(out=str(tmp_path / "libdc_nsel3.so"), defines=["DC_M4_NSEL=3"])
-    env = dict(os.environ, DC_LIB=lib)
-    r = subprocess.run([sys.executable, "-c", FUSED_SELECT_SCRIPT.format(root=ROOT)], env=env,
                        capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     assert "variant ok" in r.stdout

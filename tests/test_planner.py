@@ -1,0 +1,89 @@
+"""The B200 schedule planner (model.cu dc_model_sort_schedule).
+
+Host-only.  The planner re-parameterises the paper's Sec. 5.2 work-division
+analysis for one B200: tree levels run on chip (NK1 tile) or in
+HBM passes of one or two levels, each kernel costing launch + waves of
+resident CTAs, coefficients fitted to the measured sweep committed at
+profiles/r02/planner_sweep.jsonl.  Checks: the library's predictions equal the
+fit tool's model term by term (the C code and the fitted model are the same
+function); the planner's choice is, at every measured size and key class, the
+fastest measured schedule or within 3 % of it (one recorded exception, 3.7 %,
+f32 keys at 3 * 2^23); and it beats or matches the round-1 hand rule
+(quarter tiles below 2^23, full tiles + two-level passes above)."""
+import importlib.util
+import json
+import os
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_lopez_ortizss13_b200 as dc
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SWEEP = os.path.join(ROOT, "profiles", "r02", "planner_sweep.jsonl")
+FIT = os.path.join(ROOT, "profiles", "r02", "planner_fit.json")
+KT = {"u32": ("u32", False), "f32": ("f32", False), "u32_kv": ("u32", True)}
+
+
+def _fit_tool():
+    spec = importlib.util.spec_from_file_location("planner_fit",
+                                                  os.path.join(ROOT, "tools", "planner_fit.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    return m
+
+
+def _rows():
+    return [json.loads(line) for line in open(SWEEP) if line.strip()]
+
+
+def test_library_prediction_is_the_fitted_model():
+    pf = _fit_tool()
+    coef = json.load(open(FIT))
+    for r in _rows():
+        kt, vals = KT[r["class"]]
+        c = np.array([coef[r["class"]]["coefficients"][p] for p in pf.PARAMS])
+        expect = float(pf.features(r["class"], r["n"], r["tile_class"] == 1, r["two_level"]) @ c)
+        m = dc.model_sort_schedule(r["n"], kt, vals, tile_class=r["tile_class"],
+                                   two_level=int(r["two_level"]))
+        assert m["predicted_ms"] == pytest.approx(expect, rel=1e-5, abs=1e-7), r
+
+
+def test_choice_is_fastest_measured_within_3_percent():
+    by = {}
+    for r in _rows():
+        by.setdefault((r["class"], r["n"]), {})[(r["tile_class"], r["two_level"])] = r["ms"]
+    worst = {}
+    for (cls, n), ms in by.items():
+        kt, vals = KT[cls]
+        m = dc.model_sort_schedule(n, kt, vals)
+        chosen = ms[(m["tile_class"], m["two_level"])]
+        ratio = chosen / min(ms.values())
+        worst[(cls, n)] = ratio
+        limit = 1.04 if (cls, n) == ("f32", 3 << 23) else 1.03
+        assert ratio <= limit, (cls, n, m, ms)
+        # the round-1 hand rule: quarter tiles below 2^23, else full tiles + two-level
+        rule = ms[(1, False)] if n < (1 << 23) else ms[(2, True)]
+        assert chosen <= rule * 1.03, (cls, n)
+    assert sum(1 for v in worst.values() if v > 1.03) <= 1
+
+
+def test_planner_picks_the_measured_winners_at_the_bench_configs():
+    # 2^28 u32 (configs[2]): full tiles, two levels per HBM pass -> 7 passes
+    m = dc.model_sort_schedule(1 << 28, "u32", False)
+    assert (m["tile_class"], m["two_level"], m["hbm_passes"]) == (2, True, 7)
+    # 2^20 u32 (configs[0]): quarter tiles, one level per pass
+    m = dc.model_sort_schedule(1 << 20, "u32", False)
+    assert (m["tile_class"], m["two_level"]) == (1, False)
+    # f32 keys at 2^28: quarter tiles + two-level passes (the full f32 NK1 is slow)
+    m = dc.model_sort_schedule(1 << 28, "f32", False)
+    assert (m["tile_class"], m["two_level"]) == (1, True)
+
+
+def test_schedule_model_validation():
+    with pytest.raises(dc.DcError):
+        dc.model_sort_schedule(0)
+    with pytest.raises(dc.DcError):
+        dc.model_sort_schedule(100, tile_class=3)
+    with pytest.raises(dc.DcError):
+        dc.model_sort_schedule(100, two_level=2)

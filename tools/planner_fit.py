@@ -1,0 +1,163 @@
+"""Fit the schedule planner's B200 coefficients (model.cu) to a measured sweep.
+
+    python tools/planner_fit.py profiles/r02/planner_sweep.jsonl [--write]
+
+The planner predicts a sort's time as a sum over its kernels of a launch term
+plus (waves of resident CTAs) x (wave time, L2- or HBM-resident); for a fixed
+schedule that is LINEAR in the coefficients, so they are fitted by
+non-negative least squares on relative error (every measured sort weighted by
+1 / its time).  Reports, per key class and size, the planner's choice against
+the fastest measured schedule; --write regenerates csrc/planner_coeffs.inc.
+"""
+import json
+import math
+import os
+import sys
+
+import numpy as np
+from scipy.optimize import nnls
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+L2_BYTES = 96.0 * (1 << 20)   # working sets within this are L2-resident (126 MB L2)
+
+# compiled shapes (dc_api.cu): NK1 tile, NK1 slots, one-level merge tile, slots,
+# 4-way tile (persistent, 148 CTAs); slots = SMs x resident CTAs per SM
+SHAPES = {
+    "u32": {"nk1": [(128 * 51, 1184), (512 * 49, 296)], "p1": [(128 * 51, 1184), (256 * 51, 592)],
+            "m4": (768 * 33, 148)},
+    "f32": {"nk1": [(128 * 33, 1184), (512 * 33, 296)], "p1": [(128 * 33, 1184), (256 * 33, 592)],
+            "m4": (768 * 33, 148)},
+    "u32_kv": {"nk1": [(128 * 33, 592), (256 * 33, 296)], "p1": [(128 * 33, 592), (256 * 33, 296)],
+               "m4": (512 * 25, 148)},
+}
+PARAMS = ["nk1_q_0", "nk1_q_l2", "nk1_q_hbm", "nk1_f_0", "nk1_f_l2", "nk1_f_hbm", "p1_q_0",
+          "p1_q_l2", "p1_q_hbm", "p1_f_0", "p1_f_l2", "p1_f_hbm", "nk2_0", "nk2_t", "m4_0",
+          "m4_l2", "m4_hbm", "sel_0", "sel_t"]
+
+
+def cdiv(a, b):
+    return -(-a // b)
+
+
+def levels(n, tile):
+    p, w = 0, tile
+    while w < n:
+        w *= 2
+        p += 1
+    return p
+
+
+def features(cls, n, small, two):
+    """Coefficient multipliers of one sort (model.cu predict(), term by term)."""
+    sh = SHAPES[cls]
+    s = 0 if small else 1
+    f = dict.fromkeys(PARAMS, 0.0)
+    l2 = 8.0 * n * (2.0 if cls.endswith("kv") else 1.0) <= L2_BYTES
+    reg = "l2" if l2 else "hbm"
+    q = "q" if small else "f"
+    tile, slots = sh["nk1"][s]
+    P = levels(n, tile)
+    use_two = two and P >= 2
+    single = P % 2 if use_two else P
+    doubles = (P - single) // 2 if use_two else 0
+    f[f"nk1_{q}_0"] += 1
+    f[f"nk1_{q}_{reg}"] += cdiv(cdiv(n, tile), slots)
+    pt, ps = sh["p1"][s]
+    for _ in range(single):
+        f[f"p1_{q}_0"] += 1
+        f[f"p1_{q}_{reg}"] += cdiv(cdiv(n, pt), ps)
+        if not small:
+            f["nk2_0"] += 1
+            f["nk2_t"] += cdiv(n, pt)
+    mt, ms = sh["m4"]
+    t4 = cdiv(n, mt)
+    for _ in range(doubles):
+        f["m4_0"] += 1
+        f[f"m4_{reg}"] += cdiv(t4, ms)
+        f["sel_0"] += 1
+        f["sel_t"] += t4
+    return np.array([f[p] for p in PARAMS])
+
+
+def main():
+    rows = [json.loads(l) for l in open(sys.argv[1]) if l.strip().startswith("{")]
+    bad = [r for r in rows if not r.get("sorted_ok", True)]
+    if bad:
+        print("WARNING: unsorted outputs in the sweep:", [(r["class"], r["n"]) for r in bad])
+    fits, report = {}, {}
+    for cls in SHAPES:
+        rs = [r for r in rows if r["class"] == cls]
+        if not rs:
+            continue
+        A = np.array([features(cls, r["n"], r["tile_class"] == 1, r["two_level"]) for r in rs])
+        y = np.array([r["ms"] for r in rs])
+        w = 1.0 / y
+        coef, _ = nnls(A * w[:, None], y * w)
+        fits[cls] = dict(zip(PARAMS, coef))
+        pred = A @ coef
+        err = np.abs(pred - y) / y
+        # planner choice vs fastest measured, per n
+        by_n = {}
+        for r, p in zip(rs, pred):
+            by_n.setdefault(r["n"], []).append((p, r["ms"], r["tile_class"], r["two_level"]))
+        table = []
+        worst = 1.0
+        for n in sorted(by_n):
+            cand = by_n[n]
+            chosen = min(cand, key=lambda c: c[0])
+            best = min(cand, key=lambda c: c[1])
+            ratio = chosen[1] / best[1]
+            worst = max(worst, ratio)
+            table.append({"n": n, "chosen": [chosen[2], chosen[3]], "chosen_ms": chosen[1],
+                          "best": [best[2], best[3]], "best_ms": best[1], "ratio": ratio,
+                          "predicted_ms": chosen[0]})
+        report[cls] = {"coefficients": fits[cls], "median_rel_err": float(np.median(err)),
+                       "max_rel_err": float(err.max()), "worst_choice_ratio": worst,
+                       "table": table}
+        print(f"{cls}: median rel err {np.median(err):.3f}, max {err.max():.3f}, "
+              f"worst choice / best measured = {worst:.4f}")
+        for t in table:
+            flag = "" if t["ratio"] <= 1.03 else "  <-- over 3 %"
+            print(f"  n=2^{math.log2(t['n']):5.2f} chosen {t['chosen']} {t['chosen_ms']:.4f} ms"
+                  f"  best {t['best']} {t['best_ms']:.4f} ms  x{t['ratio']:.3f}{flag}")
+    out = os.path.join(os.path.dirname(sys.argv[1]), "planner_fit.json")
+    json.dump(report, open(out, "w"), indent=1)
+    if "--write" in sys.argv:
+        write_inc(fits)
+
+
+def write_inc(fits):
+    def kc(c0, l2, hbm, slots, tile):
+        return f"{{{c0:.7g}, {l2:.7g}, {hbm:.7g}, {slots}, {tile}}}"
+
+    blocks = []
+    for cls in ("u32", "f32", "u32_kv"):
+        c, sh = fits[cls], SHAPES[cls]
+        (tq, sq), (tf, sf) = sh["nk1"]
+        (pq, psq), (pf, psf) = sh["p1"]
+        mt, ms = sh["m4"]
+        blocks.append(
+            f"    // {cls}\n"
+            f"    {{{{{kc(c['nk1_q_0'], c['nk1_q_l2'], c['nk1_q_hbm'], sq, tq)},\n"
+            f"      {kc(c['nk1_f_0'], c['nk1_f_l2'], c['nk1_f_hbm'], sf, tf)}}},\n"
+            f"     {{{kc(c['p1_q_0'], c['p1_q_l2'], c['p1_q_hbm'], psq, pq)},\n"
+            f"      {kc(c['p1_f_0'], c['p1_f_l2'], c['p1_f_hbm'], psf, pf)}}},\n"
+            f"     {c['nk2_0']:.7g}, {c['nk2_t']:.7g},\n"
+            f"     {kc(c['m4_0'], c['m4_l2'], c['m4_hbm'], ms, mt)},\n"
+            f"     {c['sel_0']:.7g}, {c['sel_t']:.7g}}},")
+    text = ("// planner_coeffs.inc -- B200 cost coefficients of the schedule planner\n"
+            "// (model.cu), generated by tools/planner_fit.py from the measured sweep\n"
+            "// profiles/r02/planner_sweep.jsonl (whole sorts, graph replay, L2 flushed by\n"
+            "// a read; non-negative least squares on relative error).  Per key class:\n"
+            "// NK1 and one-level pass {c0 ms, wave ms L2, wave ms HBM, slots, tile} for\n"
+            "// quarter and full tiles, NK2 {c0, per tile}, 4-way pass wave, select\n"
+            "// {c0, per 4-way tile}.  Do not edit by hand.\n"
+            "static const ClassCost kPlannerCost[3] = {\n" + "\n".join(blocks) + "\n};\n"
+            f"static const double kPlannerL2Bytes = {L2_BYTES:.1f};\n")
+    path = os.path.join(ROOT, "paper_conf_ipps_lopez_ortizss13_b200", "csrc", "planner_coeffs.inc")
+    open(path, "w").write(text)
+    print("wrote", path)
+
+
+if __name__ == "__main__":
+    main()

@@ -16,7 +16,7 @@ import torch  # noqa: E402
 import dcgen  # noqa: E402
 import oracle  # noqa: E402
 import paper_conf_ipps_lopez_ortizss13_b200 as dc  # noqa: E402
-from paper_conf_ipps_lopez_ortizss13_b200 import dist  # noqa: E402
+import threading  # noqa: E402
 
 
 def check_sort(n, key_type="u32", vals=False, graphs=False, dist_name="few"):
@@ -55,18 +55,38 @@ def main():
         x = dcgen.maxsub_input(n, "small", seed=2, device="cuda")
         assert dc.Plan(n).max_subarray(x) == oracle.maxsub(x.cpu().numpy())
         assert dc.Plan(n).sum(x) == oracle.dc_sum(x.cpu().numpy())
-    # multi-GPU protocol, loopback ranks
+    # multi-GPU runtime (library), loopback ranks sharing this GPU, both exchanges
     n, G = 4 * 20_011, 4
-
-    def rank_fn(comm):
-        m = n // G
-        k = dcgen.sort_keys(n, "few", seed=7, start=comm.rank * m, count=m, device="cuda")
-        dist.sort_(k, None, comm, "u32", stride=256)
-        return k.cpu()
-
-    res = dist.run_loopback(G, rank_fn)
     full = dcgen.sort_keys(n, "few", seed=7).numpy().view(np.uint32)
-    assert np.array_equal(torch.cat(res).numpy().view(np.uint32), oracle.mergesort(full))
+    for p2p in (False, True):
+        group = dc.LoopbackGroup(G)
+        plans = []
+        for r in range(G):
+            p = dc.Plan(n)
+            p.set_mg_p2p(p2p)
+            p.set_mg_stride(256)
+            p.set_loopback(group, r)
+            plans.append(p)
+        out = [None] * G
+
+        def body(r):
+            m = n // G
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                k = dcgen.sort_keys(n, "few", seed=7, start=r * m, count=m, device="cuda")
+                plans[r].sort_(k, key_type="u32")
+                s.synchronize()
+                out[r] = k.cpu()
+
+        ts = [threading.Thread(target=body, args=(r,)) for r in range(G)]
+        for t in ts:
+            t.start()
+        for t in ts:
+            t.join()
+        assert np.array_equal(torch.cat(out).numpy().view(np.uint32), oracle.mergesort(full)), p2p
+        for p in plans:
+            p.close()
+        group.close()
     print("sanitize_run ok")
 
 

@@ -83,7 +83,18 @@ int main(int argc, char** argv) {
     CK(cudaMalloc(&dcut, (tiles + 1) * sizeof(dc::Cut4)));
     CK(cudaMemcpy(dsrc, h.data(), n * 4, cudaMemcpyHostToDevice));
     CK(cudaMemset(dcut, 0xff, (tiles + 1) * sizeof(dc::Cut4)));
-    dc::nk2_select4<dc::KeyU32, 2><<<((tiles + dc::sel4_bpw<2>() - 1) / dc::sel4_bpw<2>() + 3) / 4, 128>>>(dsrc, n, w, T, tpg, tiles, dcut);
+    dc::Pass4 P{};
+    for (int q = 0; q < 4; ++q) {
+        P.k[q] = dsrc;
+        P.v[q] = nullptr;
+        P.bound[q] = n;
+    }
+    P.n = n;
+    P.w = w;
+    P.T = T;
+    P.tpg = tpg;
+    P.custom = 0;
+    dc::nk2_select4<dc::KeyU32, 2><<<((tiles + dc::sel4_bpw<2>() - 1) / dc::sel4_bpw<2>() + 3) / 4, 128>>>(P, tiles, dcut);
     CK(cudaGetLastError());
     CK(cudaDeviceSynchronize());
     printf("select4 done\n");
@@ -105,7 +116,7 @@ int main(int argc, char** argv) {
     int grid = std::min(tiles, sms * occ);
     if (max_grid > 0) grid = std::min(grid, max_grid);
     printf("merge4: smem %d B, occupancy %d CTAs/SM, grid %d\n", smem, occ, grid);
-    k<<<grid, NT + 64, smem>>>(dsrc, nullptr, ddst, nullptr, n, w, tpg, dcut, tiles);
+    k<<<grid, NT + 64, smem>>>(P, ddst, nullptr, dcut, tiles);
     CK(cudaGetLastError());
     CK(cudaDeviceSynchronize());
     std::vector<uint32_t> out(n), ref(h);
@@ -122,13 +133,13 @@ int main(int argc, char** argv) {
         float ms_s = 0, ms_m = 0, t;
         for (int i = 0; i < iters; ++i) {
             cudaEventRecord(e0);
-            dc::nk2_select4<dc::KeyU32, 2><<<((tiles + dc::sel4_bpw<2>() - 1) / dc::sel4_bpw<2>() + 3) / 4, 128>>>(dsrc, n, w, T, tpg, tiles, dcut);
+            dc::nk2_select4<dc::KeyU32, 2><<<((tiles + dc::sel4_bpw<2>() - 1) / dc::sel4_bpw<2>() + 3) / 4, 128>>>(P, tiles, dcut);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
             cudaEventElapsedTime(&t, e0, e1);
             if (i) ms_s += t;
             cudaEventRecord(e0);
-            k<<<grid, NT + 64, smem>>>(dsrc, nullptr, ddst, nullptr, n, w, tpg, dcut, tiles);
+            k<<<grid, NT + 64, smem>>>(P, ddst, nullptr, dcut, tiles);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
             cudaEventElapsedTime(&t, e0, e1);

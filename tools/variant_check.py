@@ -1,7 +1,10 @@
 """Exact oracle parity of a tuning variant of the library (DC_LIB=<variant.so>)
 at sizes that cross its tile shapes, both schedules (diagnostic; the shipped
 library is covered by tests/)."""
+import os
 import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 import numpy as np
 import torch
