@@ -26,6 +26,10 @@
 #include "sort_kernels.cuh"
 #include "sort4_kernels.cuh"
 #include "maxsub_tma.cuh"
+#include "maxsub_rows.cuh"
+
+#include <cudaTypedefs.h>
+#include <mutex>
 
 namespace {
 
@@ -86,12 +90,11 @@ constexpr SortCfg kCfgKV{DC_KV_NT1, DC_KV_IT1, DC_STABLE_NT3, DC_STABLE_IT};
 #ifndef DC_SMALL_NT1
 #define DC_SMALL_NT1 128
 #endif
-#ifndef DC_SMALL_IT1
-#define DC_SMALL_IT1 DC_FAST_IT
+#ifndef DC_SMALL_IT1   // 128 x 49 = 6272: four quarter runs fill one 4-way tile (25088 <= 25344)
+#define DC_SMALL_IT1 49
 #endif
 constexpr SortCfg kCfgFastSmall{DC_SMALL_NT1, DC_SMALL_IT1, 128, DC_FAST_IT};
 constexpr SortCfg kCfgStableSmall{128, DC_STABLE_IT, 128, DC_STABLE_IT};
-constexpr int64_t kSmallN = 1LL << 23;
 constexpr int cmin(int a, int b) { return a < b ? a : b; }
 constexpr int kMinTout = cmin(cmin(cmin(kCfgFast.tout(), kCfgStable.tout()), kCfgKV.tout()),
                               cmin(kCfgFastSmall.tout(), kCfgStableSmall.tout()));
@@ -643,6 +646,25 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
 #ifndef DC_MS_VONLY       // values-only element fold + chunk-index recovery (measured slower)
 #define DC_MS_VONLY 0
 #endif
+// DC_MS_ROWS = 1 (default): every lane folds one contiguous row, rows fed by
+// 2-D TMA tensor copies (maxsub_rows.cuh); 0: the warp-segment kernel below.
+#ifndef DC_MS_ROWS
+#define DC_MS_ROWS 1
+#endif
+#ifndef DC_MS_RNT          // rows kernel: threads per CTA
+#define DC_MS_RNT 256
+#endif
+#ifndef DC_MS_RL           // columns per TMA box (L/4 odd)
+#define DC_MS_RL 28
+#endif
+#ifndef DC_MS_RS           // ring stages
+#define DC_MS_RS 2
+#endif
+#ifndef DC_MS_RMINB        // CTAs per SM the register budget is sized for
+#define DC_MS_RMINB 3
+#endif
+constexpr int kMsRNT = DC_MS_RNT, kMsRL = DC_MS_RL, kMsRS = DC_MS_RS, kMsRMinB = DC_MS_RMINB;
+constexpr int ms_rows_smem() { return kMsRS * kMsRNT * kMsRL * 4; }   // S x NW x 32 x L words
 constexpr int kMsP = DC_MS_P, kMsS = DC_MS_S, kMsTNT = DC_MS_TNT, kMsJ = DC_MS_J;
 constexpr bool kMsVO = DC_MS_VONLY != 0;
 constexpr int ms_tma_smem() { return kMsS * kMsTNT * kMsP * 4; }   // S x NW x 32*L words
@@ -656,7 +678,11 @@ int ms_grid(dc_plan_t p) {
         int dev = 0, sms = 148, occ = 1;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (DC_MS_TMA) {
+        if (DC_MS_ROWS) {
+            auto* k = dc::nk4_maxsub_rows<kMsRNT, kMsRL, kMsRS, kMsRMinB>;
+            cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, ms_rows_smem());
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kMsRNT, ms_rows_smem());
+        } else if (DC_MS_TMA) {
             auto* k = dc::nk4_maxsub_tma<kMsTNT, kMsP, kMsS, kMsJ, kMsVO>;
             cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, ms_tma_smem());
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, kMsTNT, ms_tma_smem());
@@ -667,8 +693,9 @@ int ms_grid(dc_plan_t p) {
         grid = sms * (occ > 0 ? occ : 1);
         grid_dev.set(grid);
     }
-    const int64_t units = DC_MS_TMA ? num_tiles(p->n, (int64_t)kMsTNT * kMsP)   // >= 1 segment/warp
-                                    : num_tiles(p->n, kMsTile);
+    const int64_t units = DC_MS_ROWS ? num_tiles(p->n, (int64_t)kMsRNT * kMsRL)   // rows >= L
+                          : DC_MS_TMA ? num_tiles(p->n, (int64_t)kMsTNT * kMsP)   // >= 1 segment/warp
+                                      : num_tiles(p->n, kMsTile);
     return (int)(units < grid ? units : grid);
 }
 
@@ -692,8 +719,52 @@ dc_status maxsub_launch(dc_plan_t p, const int32_t* d_x, int64_t off, int mode,
                         dc_maxsub_result* out_res, dc_maxsub_tuple* out_tup) {
     dc_status st = ensure_ms_state(p);
     if (st != DC_OK) return st;
-    TimedScope ts(p, DC_KERNEL_NK4_MAXSUB);
     const int grid = ms_grid(p);
+    if (DC_MS_ROWS) {
+        // rows of W elements (16-byte multiple), one per lane of the grid
+        const int64_t lanes = (int64_t)grid * kMsRNT;
+        int64_t W = (p->n + lanes - 1) / lanes;
+        W = std::max<int64_t>(4, (W + 3) / 4 * 4);
+        if (W > 65536) return fail(DC_ERR_UNSUPPORTED, "max-subarray rows longer than 2^16");
+        const dc::MsRows g{p->n, W, p->n / W};
+        if (p->ms_map_x != (const void*)d_x || p->ms_map_n != p->n || p->ms_map_w != W) {
+            std::memset(&p->ms_map, 0, sizeof(p->ms_map));
+            if (g.nrows > 0) {
+                static PFN_cuTensorMapEncodeTiled_v12000 encode = [] {
+                    void* fn = nullptr;
+                    cudaDriverEntryPointQueryResult q;
+                    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault,
+                                                &q) != cudaSuccess ||
+                        q != cudaDriverEntryPointSuccess) {
+                        cudaGetLastError();
+                        fn = nullptr;
+                    }
+                    return (PFN_cuTensorMapEncodeTiled_v12000)fn;
+                }();
+                if (!encode) return fail(DC_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+                const cuuint64_t dims[2] = {(cuuint64_t)W, (cuuint64_t)g.nrows};
+                const cuuint64_t strides[1] = {(cuuint64_t)W * 4};
+                const cuuint32_t box[2] = {(cuuint32_t)kMsRL, 32};
+                const cuuint32_t estr[2] = {1, 1};
+                const CUresult r = encode(&p->ms_map, CU_TENSOR_MAP_DATA_TYPE_INT32, 2,
+                                          const_cast<int32_t*>(d_x), dims, strides, box, estr,
+                                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                if (r != CUDA_SUCCESS) return fail(DC_ERR_CUDA, "cuTensorMapEncodeTiled failed");
+            }
+            p->ms_map_x = d_x;
+            p->ms_map_n = p->n;
+            p->ms_map_w = W;
+        }
+        TimedScope ts(p, DC_KERNEL_NK4_MAXSUB);
+        dc::nk4_maxsub_rows<kMsRNT, kMsRL, kMsRS, kMsRMinB>
+            <<<grid, kMsRNT, ms_rows_smem(), p->stream>>>(p->ms_map, d_x, g, p->ms_tiles,
+                                                          p->ms_ticket, off, mode, out_res, out_tup);
+        DC_LAUNCHED(p);
+        return DC_OK;
+    }
+    TimedScope ts(p, DC_KERNEL_NK4_MAXSUB);
     if (DC_MS_TMA) {
         // warp ranges of RW elements, a multiple of the 32*L-element segment
         const int64_t warps = (int64_t)grid * (kMsTNT / 32), seg = 32LL * kMsP;

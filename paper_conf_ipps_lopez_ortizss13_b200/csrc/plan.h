@@ -1,6 +1,7 @@
 // plan.h -- the plan object shared by the library's translation units
 // (internal; the ABI sees only the opaque dc_plan_t of include/dc.h).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -40,6 +41,9 @@ struct dc_plan_s {
     dc_maxsub_tuple* ms_tiles = nullptr;
     unsigned int* ms_ticket = nullptr;
     dc_maxsub_result* ms_res = nullptr;
+    CUtensorMap ms_map;                // 2-D row view of the last max-subarray input
+    const void* ms_map_x = nullptr;
+    int64_t ms_map_n = -1, ms_map_w = 0;
     // CUDA graphs of the sort's launch sequence, per (keys, vals, key type)
     struct GraphCache {
         uint32_t* keys;

@@ -370,6 +370,23 @@ __device__ __forceinline__ void consumer_sync() {
 #ifndef DC_M4_MINB   // CTAs per SM the register budget is sized for
 #define DC_M4_MINB 1
 #endif
+// Sanitizer variant (-DDC_M4_BARRIER_HANDOFF, tools/sanitize.sh only): the same
+// kernel with every producer/consumer hand-off done by named barriers
+// (bar.arrive / bar.sync, which compute-sanitizer racecheck models) instead of
+// mbarriers, and the pieces and outputs moved by plain loads and stores
+// instead of TMA.  The merge code is unchanged; racecheck runs clean on it,
+// which isolates the default build's reports to the mbarrier/TMA hand-off.
+#ifndef DC_M4_BARRIER_HANDOFF
+#define DC_M4_BARRIER_HANDOFF 0
+#endif
+template <int NC>
+__device__ __forceinline__ void named_arrive(int id) {
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "n"(NC + 32) : "memory");
+}
+template <int NC>
+__device__ __forceinline__ void named_sync(int id) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "n"(NC + 32) : "memory");
+}
 template <int NT, int IT, class K, bool V>
 __global__ void __launch_bounds__(NT + 64, DC_M4_MINB)
 nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ dst_v,
@@ -445,7 +462,7 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
                 const long long al0 = m.g0[r] & ~3LL;
                 long long al1 = (m.g0[r] + m.len[r]) & ~3LL;
                 if (al1 > n4) al1 = n4;
-                if (al1 < al0) al1 = al0;
+                if (al1 < al0 || DC_M4_BARRIER_HANDOFF) al1 = al0;   // (variant: all plain loads)
                 tend[r] = al1;
                 if (al1 > al0) bytes += (uint32_t)(4 * (al1 - al0)) * (V ? 2 : 1);
                 o = (m.at[r] + m.len[r] + IT + 1 + 3) & ~3;
@@ -457,6 +474,11 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
                 }
             }
             __syncwarp();
+            if (DC_M4_BARRIER_HANDOFF) {
+                if (lane == 0) meta[b] = m;
+                named_arrive<NC>(2 + b);                 // full[b]
+                return;
+            }
             if (lane == 0) {
                 meta[b] = m;
                 const uint32_t fb = smem_addr(&full[b]);
@@ -477,6 +499,21 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
         if (my_tiles > 1) fill(1, 1);
         for (int i = 0; i < my_tiles; ++i) {
             const int b = i & 1;
+            if (DC_M4_BARRIER_HANDOFF) {
+                named_sync<NC>(4 + b);                   // empty[b]: output of tile i written
+                const Tile4 m = meta[b];
+                const int h = (int)(m.out & 3);
+                const int head = min(m.total, (4 - h) & 3);
+                const int body = (m.total - head) & ~3;
+                const uint32_t* ob = sm + b * BW + GU + h;
+                for (int e = head + lane; e < head + body; e += 32) {
+                    dst_k[m.out + e] = ob[e];
+                    if (V) dst_v[m.out + e] = ob[KW + e];
+                }
+                __syncwarp();
+                if (i + 2 < my_tiles) fill(i + 2, b);
+                continue;
+            }
             mbar_wait(smem_addr(&empty[b]), (i >> 1) & 1);   // output of tile i written
             if (lane == 0) {
                 const Tile4 m = meta[b];
@@ -509,7 +546,8 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
         const int b = i & 1;
         uint32_t* buf = sm + b * BW + GU;
         const uint32_t B0 = SM0 + 4u * (b * BW + GU);
-        mbar_wait(smem_addr(&full[b]), (i >> 1) & 1);
+        if (DC_M4_BARRIER_HANDOFF) named_sync<NC>(2 + b);
+        else mbar_wait(smem_addr(&full[b]), (i >> 1) & 1);
         const Tile4 m = meta[b];
 
         // stage 1: X = merge(P0, P1), Y = merge(P2, P3), IT-output windows
@@ -632,6 +670,10 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
                     }
                 }
             }
+        }
+        if (DC_M4_BARRIER_HANDOFF) {
+            named_arrive<NC>(4 + b);                     // empty[b]
+            continue;
         }
         fence_proxy_async_smem();
         __syncwarp();

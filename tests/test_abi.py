@@ -116,7 +116,8 @@ def test_schedule(n, kt, vals):
     assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / t)))) == m["global_levels"]
     P = s["global_passes"]
     assert s["hbm_passes"] == (P % 2 + P // 2 if (m["two_level"] and P >= 2) else P)
-    assert m["predicted_ms"] == min(v for v in m["candidates_ms"].values())
+    # least predicted time, or a full-tile schedule within 3 % of it (near-tie rule)
+    assert m["predicted_ms"] <= 1.03 * min(v for v in m["candidates_ms"].values())
     # forced choices are honoured and reported
     for tc in (1, 2):
         for two in (False, True):

@@ -285,7 +285,7 @@ def test_sort_every_forced_schedule(dc, oracle_mod, tile_class, two, key_type, w
     assert np.array_equal(_np_keys(keys, key_type).view(np.uint32), ek.view(np.uint32))
 
 
-SMALL_TILE = 128 * 51        # keys-only tile below 2^23 keys
+SMALL_TILE = 128 * 49        # keys-only quarter tile (the planner's choice below 2^23 keys)
 
 
 @pytest.mark.parametrize("n", [SMALL_TILE - 1, SMALL_TILE, SMALL_TILE + 1, 2 * SMALL_TILE + 3,
@@ -604,5 +604,5 @@ def test_launch_counts(dc, n, fused):
     s = p.schedule("u32", False)
     P, H = s["global_passes"], s["hbm_passes"]
     single = P - 2 * (P - H)          # one-level passes; the rest are two-level passes
-    per_single = 1 if (fused and s["tile"] == 128 * 51) else 2   # quarter tiles: fused partition
+    per_single = 1 if (fused and s["tile"] == 128 * 49) else 2   # quarter tiles: fused partition
     assert p.launch_count() == 1 + per_single * single + 2 * (H - single)

@@ -23,7 +23,7 @@ L2_BYTES = 96.0 * (1 << 20)   # working sets within this are L2-resident (126 MB
 # compiled shapes (dc_api.cu): NK1 tile, NK1 slots, one-level merge tile, slots,
 # 4-way tile (persistent, 148 CTAs); slots = SMs x resident CTAs per SM
 SHAPES = {
-    "u32": {"nk1": [(128 * 51, 1184), (512 * 49, 296)], "p1": [(128 * 51, 1184), (256 * 51, 592)],
+    "u32": {"nk1": [(128 * 49, 1184), (512 * 49, 296)], "p1": [(128 * 51, 1184), (256 * 51, 592)],
             "m4": (768 * 33, 148)},
     "f32": {"nk1": [(128 * 33, 1184), (512 * 33, 296)], "p1": [(128 * 33, 1184), (256 * 33, 592)],
             "m4": (768 * 33, 148)},
@@ -45,6 +45,11 @@ def levels(n, tile):
         w *= 2
         p += 1
     return p
+
+
+def hbm_passes(cls, n, small, two):
+    P = levels(n, SHAPES[cls]["nk1"][0 if small else 1][0])
+    return P % 2 + P // 2 if (two and P >= 2) else P
 
 
 def features(cls, n, small, two):
@@ -105,6 +110,13 @@ def main():
         for n in sorted(by_n):
             cand = by_n[n]
             chosen = min(cand, key=lambda c: c[0])
+            # model.cu's near-tie rule: a full-tile schedule with the same
+            # number of HBM passes within 3 % of a quarter-tile choice wins
+            if chosen[2] == 1:
+                full = [c for c in cand if c[2] == 2 and c[3] == chosen[3]]
+                if full and hbm_passes(cls, n, False, chosen[3]) == \
+                        hbm_passes(cls, n, True, chosen[3]) and full[0][0] <= chosen[0] * 1.03:
+                    chosen = full[0]
             best = min(cand, key=lambda c: c[1])
             ratio = chosen[1] / best[1]
             worst = max(worst, ratio)

@@ -60,11 +60,25 @@ caps = {"prof_nk1": ("sort_u32", "nk1_blocksort"), "prof_nk2": ("sort_u32", "nk2
         "prof_nk3": ("sort_u32", "nk3_merge4"), "prof_nk3_kv": ("sort_kv", "nk3_merge4"),
         "prof_nk4": ("maxsub", "nk4_maxsub"), "prof_nk1_kv": ("sort_kv", "nk1_blocksort"),
         "prof_sum": ("sum", "breadth_first_reduce")}
-for cap, (wl, kern) in caps.items():
+def load_summary(cap):
+    """Summary of one capture: the .ncu-rep if it came back, else the JSON the
+    box wrote with tools/ncu_summary.py (reports are summarised and deleted
+    there to keep gpurun_out/ under the 64 MiB copy-back limit)."""
     p = os.path.join(G, cap + ".ncu-rep")
-    if not os.path.exists(p):
+    if os.path.exists(p):
+        return summarise(p)
+    j = os.path.join(G, cap + ".summary.json")
+    if os.path.exists(j):
+        text = open(j).read()
+        return json.loads(text[text.index("["):])
+    return None
+
+
+for cap, (wl, kern) in caps.items():
+    ss = load_summary(cap)
+    if not ss:
         continue
-    s = summarise(p)[0]
+    s = ss[0]
     json.dump(s, open(os.path.join(out, f"ncu_{wl}_{kern}.json"), "w"), indent=1)
     rd = float(s["dram__bytes_read.sum"].split()[0]) * (1e9 if "Gbyte" in s["dram__bytes_read.sum"] else 1e6 if "Mbyte" in s["dram__bytes_read.sum"] else 1e3)
     wr = float(s["dram__bytes_write.sum"].split()[0]) * (1e9 if "Gbyte" in s["dram__bytes_write.sum"] else 1e6 if "Mbyte" in s["dram__bytes_write.sum"] else 1e3)
@@ -73,6 +87,13 @@ for cap, (wl, kern) in caps.items():
                                         "source": f"profiles/{rnd}/ncu_{wl}_{kern}.json"}
     print(wl, kern, s["gpu__time_duration.sum"], f"dram {(rd + wr) / 1e9:.4f} GB")
 json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
+
+# ---- multi-GPU kernels in loopback (tools/mg_profile.py under ncu): one JSON per mode
+for mode in ("a2a", "fused"):
+    ss = load_summary(f"prof_mg_{mode}")
+    if ss:
+        json.dump(ss, open(os.path.join(out, f"ncu_mg_{mode}.json"), "w"), indent=1)
+        print("mg", mode, [(x["kernel"][:40], x.get("gpu__time_duration.sum")) for x in ss][:8])
 
 # ---- bench lines of the same build (last JSON line of each gpurun_out/bench_*.json)
 import glob  # noqa: E402
