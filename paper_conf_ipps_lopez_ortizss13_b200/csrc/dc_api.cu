@@ -646,10 +646,14 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
 #ifndef DC_MS_VONLY       // values-only element fold + chunk-index recovery (measured slower)
 #define DC_MS_VONLY 0
 #endif
-// DC_MS_ROWS = 1 (default): every lane folds one contiguous row, rows fed by
-// 2-D TMA tensor copies (maxsub_rows.cuh); 0: the warp-segment kernel below.
+// DC_MS_ROWS = 1: every lane folds one contiguous row, rows fed by 2-D TMA
+// tensor copies, 3 CTAs per SM (maxsub_rows.cuh).  Measured at 2^24 (r02,
+// profiles/r02/nk4_variants.txt): 28.9-33.3 us per launch over five ring
+// shapes against 28.8 us for the warp-segment kernel (0, default): tripling
+// the resident warps did not raise the issue rate (52 %), the per-element fold
+// (~17 instructions, selects on the half-rate ALU pipe) bounds both.
 #ifndef DC_MS_ROWS
-#define DC_MS_ROWS 1
+#define DC_MS_ROWS 0
 #endif
 #ifndef DC_MS_RNT          // rows kernel: threads per CTA
 #define DC_MS_RNT 256
@@ -1404,21 +1408,21 @@ dc_status dc_mg_split_matrix(dc_plan_t p, dc_key_type kt, const uint32_t* d_gath
             auto* k = dc::mg_split_matrix<dc::KeyU32>;
             DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                             (int)smem));
-            k<<<world - 1, 64, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
+            k<<<world - 1, 256, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
             break;
         }
         case DC_KEY_I32: {
             auto* k = dc::mg_split_matrix<dc::KeyI32>;
             DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                             (int)smem));
-            k<<<world - 1, 64, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
+            k<<<world - 1, 256, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
             break;
         }
         case DC_KEY_F32: {
             auto* k = dc::mg_split_matrix<dc::KeyF32>;
             DC_CUDA(p, cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                             (int)smem));
-            k<<<world - 1, 64, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
+            k<<<world - 1, 256, smem, p->stream>>>(d_gathered, world, shard_n, wcap, d_cmat);
             break;
         }
         default:

@@ -1,4 +1,5 @@
-// maxsub_rows.cuh -- NK4 with every lane folding ONE contiguous row (default NK4).
+// maxsub_rows.cuh -- NK4 with every lane folding ONE contiguous row (-DDC_MS_ROWS=1;
+// measured no faster than the warp-segment kernel).
 //
 // Same method as nk4_maxsub / nk4_maxsub_tma: contiguous pieces are folded
 // left to right (the leaves and the bottom levels of the D&C tree, exact by

@@ -22,6 +22,8 @@
 #pragma once
 #include <cstdint>
 
+#include "sort_kernels.cuh"   // warp_first_false
+
 namespace dc {
 
 // a7 (1/4): every stride-th key of a sorted shard.
@@ -76,17 +78,30 @@ __global__ void mg_count(const uint32_t* __restrict__ keys, long long n, int me,
 // of largest global rank < k_d (lo) and smallest global rank >= k_d (hi).
 // Global ranks are distinct (candidates are distinct elements); packed as
 // ((rank + 1) << 24) | c so one 64-bit atomic max / min finds both.
+// Every candidate's packed value is reduced within its warp first (max of
+// the ones below k_d, min of the others), so one lane per warp issues the
+// atomics: the G-1 addresses see cands/32 atomics each instead of cands
+// (ncu, loopback G = 4, 2^25 keys: 12-20 us of contended atomics before).
 __global__ void mg_brackets(const int64_t* __restrict__ R, long long cands, int G, long long m,
                             unsigned long long* __restrict__ lo_pack,
                             unsigned long long* __restrict__ hi_pack) {
     const long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= cands) return;
-    const long long rc = R[c];
+    const bool valid = c < cands;                      // every lane takes part in the shuffles
+    const long long rc = valid ? R[c] : 0;
     const unsigned long long packed = ((unsigned long long)(rc + 1) << 24) | (unsigned long long)c;
     for (int d = 1; d < G; ++d) {
         const long long k = (long long)d * m;
-        if (rc < k) atomicMax(lo_pack + d, packed);
-        else atomicMin(hi_pack + d, packed);
+        unsigned long long lo = (valid && rc < k) ? packed : 0ULL;
+        unsigned long long hi = (valid && rc >= k) ? packed : ~0ULL;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            lo = max(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+            hi = min(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+        }
+        if ((threadIdx.x & 31) == 0) {
+            if (lo != 0ULL) atomicMax(lo_pack + d, lo);
+            if (hi != ~0ULL) atomicMin(hi_pack + d, hi);
+        }
     }
 }
 
@@ -186,17 +201,21 @@ __global__ void mg_split_matrix(const uint32_t* __restrict__ gathered, int G, lo
     }
     __syncthreads();
     const long long t = reinterpret_cast<const long long*>(gathered)[3 * (d - 1) + 2];
-    if (threadIdx.x < G) {
-        const int r = threadIdx.x;
-        long long a = 0, b = len[r];      // cnt = first p with merged_rank(r, p) >= t
-        while (a < b) {
-            const long long mid = (a + b) >> 1;
-            if (merged_rank<K>(win, off, len, G, r, mid) < t) a = mid + 1; else b = mid;
-        }
-        cmat[r * (G + 1) + d] = lo[r] + a;
-        if (d == 1) {
-            cmat[r * (G + 1) + 0] = 0;
-            cmat[r * (G + 1) + G] = m;
+    // one warp per rank r: cnt = first p with merged_rank(r, p) >= t, found by
+    // a 33-ary warp search (32 probes per round, ~3 rounds for a window of
+    // 4096) instead of one thread's binary search (12 dependent probes, each
+    // G-1 inner searches); ncu, loopback G = 4: ~110 us per launch before.
+    const int lane = threadIdx.x & 31;
+    for (int r = threadIdx.x >> 5; r < G; r += blockDim.x >> 5) {
+        const long long cnt = warp_first_false(0, len[r], [&](long long p) {
+            return merged_rank<K>(win, off, len, G, r, p) < t;
+        });
+        if (lane == 0) {
+            cmat[r * (G + 1) + d] = lo[r] + cnt;
+            if (d == 1) {
+                cmat[r * (G + 1) + 0] = 0;
+                cmat[r * (G + 1) + G] = m;
+            }
         }
     }
 }

@@ -114,3 +114,19 @@ def test_maxsub_values_only_fold(tmp_path):
                        capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     assert "variant ok" in r.stdout
+
+
+def test_maxsub_rows_kernel(tmp_path):
+    """NK4 with one contiguous row per lane fed by 2-D TMA tensor copies
+    (-DDC_MS_ROWS=1, maxsub_rows.cuh): bit-exact (sum, start, end) and summary
+    tuple on tie-heavy, degenerate and ragged-tail inputs."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ipps_lopez_ortizss13_b200 import build
+
+    lib = build.build(out=str(tmp_path / "libdc_rows.so"), defines=["DC_MS_ROWS=1"])
+    env = dict(os.environ, DC_LIB=lib)
+    r = subprocess.run([sys.executable, "-c", VONLY_SCRIPT.format(root=ROOT)], env=env,
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert "variant ok" in r.stdout
