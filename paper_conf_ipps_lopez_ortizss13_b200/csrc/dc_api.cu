@@ -39,7 +39,7 @@ namespace {
 // 512 threads x 49 items = tiles of 25088 keys (9 shared-memory merge levels
 // on top of a 49-input register network; 14 global levels at 2^28), one-level
 // merge CTAs of 256 x 51 = 13056 outputs.  49 rather than 51 items: a group of
-// four 25088-key runs splits into four 4-way tiles of <= 25344 keys, where four
+// four 25088-key runs splits into four 4-way tiles of <= 25984 keys, where four
 // 26112-key runs need a fifth 3072-key sliver tile (2^28: 6.08 -> 5.96 ms).
 // (1024 x 51 tiles save a global level at 2^28 but cost more in NK1 than they
 // save: 6.38 vs 6.19 ms.)  f32 keys carry a tile-local index for stability:
@@ -90,7 +90,7 @@ constexpr SortCfg kCfgKV{DC_KV_NT1, DC_KV_IT1, DC_STABLE_NT3, DC_STABLE_IT};
 #ifndef DC_SMALL_NT1
 #define DC_SMALL_NT1 128
 #endif
-#ifndef DC_SMALL_IT1   // 128 x 49 = 6272: four quarter runs fill one 4-way tile (25088 <= 25344)
+#ifndef DC_SMALL_IT1   // 128 x 49 = 6272: four quarter runs fill one 4-way tile (25088 <= 25984)
 #define DC_SMALL_IT1 49
 #endif
 constexpr SortCfg kCfgFastSmall{DC_SMALL_NT1, DC_SMALL_IT1, 128, DC_FAST_IT};
@@ -162,13 +162,16 @@ size_t split_entries(int64_t n) {
 
 // Two-level passes: 4-way output tiles of NT*IT keys, one cut vector (4 ints)
 // per tile; every group of 4 runs is cut into ceil(min(4w, n)/T) tiles.  Keys
-// only: 768 x 33 (T = 25344; one CTA per SM, 2 x 102 KB of buffers); with
+// only: 896 x 29 (T = 25984; one CTA per SM, 2 x 104 KB of buffers); with
 // values the key and value regions share the same budget: 512 x 25.
+// r02: 896 x 29 (T = 25984, 960 threads x 64 registers) 3.708 ms of merges per
+// 2^28 u32 sort vs 768 x 33 3.757; fewer threads with more items are slower
+// (512 x 49 4.03 ... 320 x 79 4.92; profiles/r02/m4_shapes.txt).
 #ifndef DC_TWO_NT
-#define DC_TWO_NT 768
+#define DC_TWO_NT 896
 #endif
 #ifndef DC_TWO_IT
-#define DC_TWO_IT 33
+#define DC_TWO_IT 29
 #endif
 #ifndef DC_TWO_NT_KV
 #define DC_TWO_NT_KV 512

@@ -24,9 +24,9 @@ L2_BYTES = 96.0 * (1 << 20)   # working sets within this are L2-resident (126 MB
 # 4-way tile (persistent, 148 CTAs); slots = SMs x resident CTAs per SM
 SHAPES = {
     "u32": {"nk1": [(128 * 49, 1184), (512 * 49, 296)], "p1": [(128 * 51, 1184), (256 * 51, 592)],
-            "m4": (768 * 33, 148)},
+            "m4": (896 * 29, 148)},
     "f32": {"nk1": [(128 * 33, 1184), (512 * 33, 296)], "p1": [(128 * 33, 1184), (256 * 33, 592)],
-            "m4": (768 * 33, 148)},
+            "m4": (896 * 29, 148)},
     "u32_kv": {"nk1": [(128 * 33, 592), (256 * 33, 296)], "p1": [(128 * 33, 592), (256 * 33, 296)],
                "m4": (512 * 25, 148)},
 }

@@ -22,6 +22,8 @@ import paper_conf_ipps_lopez_ortizss13_b200 as dc  # noqa: E402
 
 K, W = 7, 3
 SIZES = [1 << k for k in range(14, 29)] + [3 << 21, 3 << 23, 3 << 25]
+if os.environ.get("DC_SWEEP_SIZES"):      # e.g. "24,26,28": powers of two only
+    SIZES = [1 << int(k) for k in os.environ["DC_SWEEP_SIZES"].split(",")]
 CLASSES = [("u32", False), ("f32", False), ("u32", True)]
 if len(sys.argv) > 1:
     CLASSES = [c for c in CLASSES if f"{c[0]}{'_kv' if c[1] else ''}" in sys.argv[1].split(",")]
