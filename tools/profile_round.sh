@@ -6,6 +6,8 @@
 # Then, here: python tools/summarize_profiles.py <round>
 mkdir -p gpurun_out
 O=gpurun_out
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1
+timeout 2400 python -m pytest tests -m gpu -q > $O/pytest_gpu.txt 2>&1
 timeout 600 python bench.py > $O/bench_default.json 2> $O/bench_default.err
 for w in sort_kv sort_u32_small maxsub sum; do
   timeout 300 python bench.py --workload $w --steps 10 --warmup 3 > $O/bench_$w.json 2>&1
