@@ -86,52 +86,65 @@ struct MsVal {
     }
 };
 
-// Chunk [c, min(c+L, n)): smallest e maximising sum(x[c..e]) (the prefix end).
+// Chunk [c, min(c+L, n)) staged at s[0..): smallest e maximising sum(x[c..e])
+// (the prefix end).
 template <int L>
-__device__ long long ms_first_max_prefix(const int* __restrict__ x, long long n, long long c) {
-    const long long e1 = min(n, c + L);
-    long long P = 0, m = kMsNeg, k = c;
-    for (long long j = c; j < e1; ++j) {
-        P += x[j];
+__device__ long long ms_first_max_prefix(const int* s, long long n, long long c) {
+    const int len = (int)min((long long)L, n - c);
+    long long P = 0, m = kMsNeg;
+    int k = 0;
+    for (int j = 0; j < len; ++j) {
+        P += s[j];
         if (P > m) { m = P; k = j; }
     }
-    return k;
+    return c + k;
 }
-// Chunk [c, e1): smallest s maximising sum(x[s..e1-1]) (the suffix start).
+// Chunk [c, c+len) staged at s: smallest start maximising the suffix sum.
 template <int L>
-__device__ long long ms_first_max_suffix(const int* __restrict__ x, long long n, long long c) {
-    const long long e1 = min(n, c + L);
-    long long P = 0, m = 0, k = c;
-    for (long long j = c; j + 1 < e1; ++j) {
-        P += x[j];
+__device__ long long ms_first_max_suffix(const int* s, long long n, long long c) {
+    const int len = (int)min((long long)L, n - c);
+    long long P = 0, m = 0;
+    int k = 0;
+    for (int j = 0; j + 1 < len; ++j) {
+        P += s[j];
         if (P < m) { m = P; k = j + 1; }
     }
-    return k;
+    return c + k;
 }
 
-// Exact indices from chunk labels (warp 0 of the last CTA; lanes 0..3 scan
-// one chunk each).  a's pe/ss/bs/be are chunk starts; on return they are
-// element indices.  pe: first prefix maximum inside its chunk; ss: first
-// suffix maximum inside its chunk; best: the in-chunk Kadane when start and
-// end chunk coincide, else the suffix-start / prefix-end scans of the two.
+// Exact indices from chunk labels (warp 0 of the last CTA).  a's pe/ss/bs/be
+// are chunk starts; on return they are element indices.  pe: first prefix
+// maximum inside its chunk; ss: first suffix maximum inside its chunk; best:
+// the in-chunk Kadane when start and end chunk coincide, else the
+// suffix-start / prefix-end scans of the two.  The (at most four) chunks are
+// first staged in shared memory by one coalesced warp load, so the four
+// scanning lanes read shared memory instead of waiting out one global-memory
+// latency per element (r01's serial scans of global memory cost ~17 us).
 template <int L>
 __device__ void ms_recover(const int* __restrict__ x, long long n, MsTupG& a, long long* rec) {
+    __shared__ int stage[4][L];
     const int lane = threadIdx.x & 31;
-    if (lane == 0) rec[0] = ms_first_max_prefix<L>(x, n, a.pe);
-    if (lane == 1) rec[1] = ms_first_max_suffix<L>(x, n, a.ss);
+    const long long cs[4] = {a.pe, a.ss, a.bs, a.be};
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+        for (int e = lane; e < L; e += 32)
+            if (cs[q] + e < n) stage[q][e] = x[cs[q] + e];
+    __syncwarp();
+    if (lane == 0) rec[0] = ms_first_max_prefix<L>(stage[0], n, a.pe);
+    if (lane == 1) rec[1] = ms_first_max_suffix<L>(stage[1], n, a.ss);
     if (lane == 2) {
         if (a.bs == a.be) {
             MsFold f;
             f.init();
-            const long long e1 = min(n, a.bs + L);
-            for (long long j = a.bs; j < e1; ++j) f.step(x[j], (int)(j - a.bs));
+            const int len = (int)min((long long)L, n - a.bs);
+            for (int j = 0; j < len; ++j) f.step(stage[2][j], j);
             rec[2] = a.bs + f.bs;
             rec[3] = a.bs + f.be;
         } else {
-            rec[2] = ms_first_max_suffix<L>(x, n, a.bs);
+            rec[2] = ms_first_max_suffix<L>(stage[2], n, a.bs);
         }
     }
-    if (lane == 3 && a.bs != a.be) rec[3] = ms_first_max_prefix<L>(x, n, a.be);
+    if (lane == 3 && a.bs != a.be) rec[3] = ms_first_max_prefix<L>(stage[3], n, a.be);
     __syncwarp();
     a.pe = rec[0]; a.ss = rec[1]; a.bs = rec[2]; a.be = rec[3];
 }
