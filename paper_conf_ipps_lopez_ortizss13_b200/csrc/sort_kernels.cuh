@@ -287,8 +287,12 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
 #ifndef DC_NK1_STOPW   // measurement knob only: stop the merge levels below this width
 #define DC_NK1_STOPW (1 << 30)
 #endif
+    // w = IT * 2^lg at every level: the run index, the pair's thread group
+    // and the diagonal are shifts and masks (runtime divisions by w compiled
+    // to ~20-instruction float sequences, ~4 % of NK1's issue slots in r01)
+    int lg = 0;
 #pragma unroll 1
-    for (int w = IT; w < TILE && w < DC_NK1_STOPW; w *= 2) {
+    for (int w = IT; w < TILE && w < DC_NK1_STOPW; w *= 2, ++lg) {
         // Levels whose pairs fit in one warp (2w <= 32*IT) only touch that
         // warp's own region: a warp barrier suffices and warps drift apart
         // (search / merge / write phases overlap across warps).
@@ -296,7 +300,7 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
         if (warp_local) __syncwarp(); else __syncthreads();
         {   // write this thread's IT ascending keys: A runs ascending, B runs descending
             const int pos = tid * IT;
-            const int r = pos / w;                        // run index at width w
+            const int r = tid >> lg;                      // run index at width w
             const int o = pos - r * w;                    // offset inside the run
             const int pr = (r >> 1) * (2 * w);            // pair start
             if ((r & 1) == 0) {
@@ -308,9 +312,8 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
             }
         }
         if (warp_local) __syncwarp(); else __syncthreads();
-        const int tpg = (2 * w) / IT;                     // threads per merged pair
-        const int s = (tid / tpg) * (2 * w);              // pair start
-        const int diag = (tid % tpg) * IT;
+        const int s = (tid >> (lg + 1)) * (2 * w);        // pair start (2^(lg+1) threads per pair)
+        const int diag = (tid & ((2 << lg) - 1)) * IT;
         // co-rank: A[m] at s + m, B[diag-1-m] at s + 2w - 1 - (diag-1-m) = s + 2w - diag + m
         const uint32_t Ab = SK + 4u * s, Bb = SK + 4u * (s + 2 * w - diag);
         int lo = max(0, diag - w), hi = min(diag, w);
@@ -402,8 +405,9 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     if constexpr (!V && !K::kNeedStable) {
         merge_levels_bitonic<NT, IT, K>(k, sk);
     } else {
+        int lg = 0;                                    // w = IT * 2^lg (shifts, not divisions)
 #pragma unroll 1
-        for (int w = IT; w < TILE; w *= 2) {
+        for (int w = IT; w < TILE; w *= 2, ++lg) {
             __syncthreads();
 #pragma unroll
             for (int j = 0; j < IT; ++j) {
@@ -411,9 +415,8 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
                 if (V) si[tid * IT + j] = ix[j];
             }
             __syncthreads();
-            const int tpg = (2 * w) / IT;            // threads per merged pair
-            const int s = (tid / tpg) * (2 * w);     // pair start
-            const int diag = (tid % tpg) * IT;
+            const int s = (tid >> (lg + 1)) * (2 * w);   // pair start (2^(lg+1) threads per pair)
+            const int diag = (tid & ((2 << lg) - 1)) * IT;
             const uint32_t A = SK + 4u * s, B = A + 4u * w;
             const int i = corank_smem<K>(A, w, B, w, diag);
             uint32_t src[IT];
