@@ -63,6 +63,20 @@ __device__ __forceinline__ MsTupT<I> ms_combine(const MsTupT<I>& L, const MsTupT
     return c;
 }
 
+// int32 -> FP64.  DC_MS_CVT = 1: 2^52 + 2^31 + x is the double with high word
+// 0x43300000 and low word x ^ 0x80000000, so x = that - (2^52 + 2^31) exactly
+// (one LOP3 + one DADD on the FP64 pipe instead of an I2F.F64 conversion).
+#ifndef DC_MS_CVT
+#define DC_MS_CVT 0
+#endif
+__device__ __forceinline__ double ms_i2d(int x) {
+#if DC_MS_CVT
+    return __hiloint2double(0x43300000, x ^ (int)0x80000000) - 4503601774854144.0;
+#else
+    return (double)x;
+#endif
+}
+
 // Left-to-right fold of one element x at index i: combine(T, leaf(x, i)),
 // which is Kadane's step with the tie rules above.  The running values are
 // kept in FP64: a thread folds at most 2^16 int32 elements, so every real
@@ -78,7 +92,7 @@ struct MsFold {
         pe = ss = bs = be = 0;
     }
     __device__ __forceinline__ void step(int x, int i) {
-        const double xd = (double)x;
+        const double xd = ms_i2d(x);
         tot += xd;
         const bool up = tot > pre;                 // strict: smallest end
         pre = up ? tot : pre;
@@ -134,11 +148,12 @@ __device__ __forceinline__ MsTupT<I> ms_shfl_down(const MsTupT<I>& t, int off) {
 // order); the result is valid in lane 0.
 template <int WIDTH, class I>
 __device__ __forceinline__ MsTupT<I> ms_warp_combine(MsTupT<I> t) {
-    const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int off = 1; off < WIDTH; off <<= 1) {
-        MsTupT<I> r = ms_shfl_down(t, off);
-        if ((lane & (2 * off - 1)) == 0) t = ms_combine(t, r);
+        // branch-free (see ms_fold_warp): lanes that are not multiples of
+        // 2*off compute unused values, and no shuffle is ever divergent
+        const MsTupT<I> r = ms_shfl_down(t, off);
+        t = ms_combine(t, r);
     }
     return t;
 }

@@ -44,12 +44,18 @@ __device__ __forceinline__ MsFold ms_fold_shfl_down(const MsFold& t, int off) {
 }
 
 // Ordered combine of the 32 lanes' folds (lane order = segment order); lane 0.
+// Branch-free: every lane absorbs its partner at every level.  Only lanes
+// with (lane & (2*off - 1)) == 0 hold a meaningful summary afterwards (the
+// partner they read at the next level is again such a lane), the others carry
+// unused values.  A conditional absorb made the next level's full-mask
+// shuffles potentially divergent, and the compiler guarded every level with a
+// WARPSYNC / BRA.DIV fallback path (~45 extra instructions per level, ~30 %
+// of NK4's instructions were the per-segment tree).
 __device__ __forceinline__ MsFold ms_fold_warp(MsFold t) {
-    const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int off = 1; off < 32; off <<= 1) {
         const MsFold r = ms_fold_shfl_down(t, off);
-        if ((lane & (2 * off - 1)) == 0) t.absorb(r);
+        t.absorb(r);
     }
     return t;
 }
@@ -72,7 +78,7 @@ struct MsVal {
         tot = 0.0; pre = (double)kMsNeg; suf = (double)kMsNeg; best = (double)kMsNeg;
     }
     __device__ __forceinline__ void step(int x) {
-        const double xd = (double)x;
+        const double xd = ms_i2d(x);
         tot += xd;
         pre = dmax(pre, tot);
         suf = dmax(suf, 0.0) + xd;
@@ -262,6 +268,7 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
             for (int e = e0; e < min(cnt, e0 + L); ++e)
                 f.step(e < body ? sl[e - e0] : x[g0 + e], i0 + (e - e0));
         }
+        __syncwarp();                                // reconverge before the shuffle tree
         f = ms_fold_warp(f);
         if (lane == 0) acc.absorb(f);
         __syncwarp();                                // every lane is done with stage s
