@@ -415,7 +415,14 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     // Levels over HBM: P = ceil(log2(ceil(n/tile))).  Keys-only sorts fold
     // two levels into one pass (4-way groups, sort4_kernels.cuh); with P odd
     // one single-level pass goes first.
-    const int P = global_passes(n, C.tile());
+    // f2 prototype (-DDC_NK1_CLUSTER=2, keys-only full tiles): NK1 runs one more
+    // level across each cluster of two CTAs, so the fused runs are 2 tiles wide.
+#ifndef DC_NK1_CLUSTER
+#define DC_NK1_CLUSTER 0
+#endif
+    constexpr bool kCl = DC_NK1_CLUSTER == 2 && !V && !K::kNeedStable && !SMALL;
+    const int64_t ftile = kCl ? 2 * (int64_t)C.tile() : (int64_t)C.tile();
+    const int P = global_passes(n, ftile);
     constexpr bool kTwoCapable = true;
     const bool two = two_level && P >= 2;
     const int single = two ? (P % 2) : P;
@@ -460,13 +467,13 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
         return DC_OK;
     };
 
-    int64_t w = C.tile();
+    int64_t w = ftile;
     int lv = 0;
     // Chunked pipeline (one-level schedule, not while timing kernels): the
     // bottom `lc` levels of every chunk of tile*2^lc keys run on the chunk's
     // own stream right after its NK1; chunks overlap each other.
     int lc = 0, chunks = 1;
-    if (!SMALL && !two && !p->timing && p->pipe_chunks > 1) {
+    if (!SMALL && !kCl && !two && !p->timing && p->pipe_chunks > 1) {
         int lt = 0;
         while ((1 << lt) < p->pipe_chunks) ++lt;
         if (single > lt) {
@@ -512,8 +519,20 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     } else {
         // NK1: base cases + fused bottom levels (reads the caller's buffer).
         TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT);
-        k1<<<(unsigned)num_tiles(n, C.tile()), C.nt1, nk1_smem_bytes(C, hv), p->stream>>>(
-            keys, vals, cur_k, cur_v, n);
+        if constexpr (kCl) {
+            auto* kc = dc::nk1_blocksort_cl2<C.nt1, C.it1, K>;
+            const int smem = dc::tile_words(C.tile(), C.it1 + 4) * 4;
+            static PerDevice cl_attr;
+            if (!cl_attr.get()) {
+                DC_CUDA(p, cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+                cl_attr.set(1);
+            }
+            const unsigned grid = (unsigned)(num_tiles(n, 2 * (int64_t)C.tile()) * 2);
+            kc<<<grid, C.nt1, smem, p->stream>>>(keys, cur_k, n);
+        } else {
+            k1<<<(unsigned)num_tiles(n, C.tile()), C.nt1, nk1_smem_bytes(C, hv), p->stream>>>(
+                keys, vals, cur_k, cur_v, n);
+        }
         DC_LAUNCHED(p);
     }
 #ifdef DC_ONLY_NK1   // measurement builds only: time the fused kernel alone

@@ -30,6 +30,21 @@
 
 namespace dc {
 
+// Timeline probe (tools/nk4_trace.cu only): %globaltimer at CTA entry, after
+// each warp's segment loop, after the CTA's ticket, and at the end of the last
+// CTA, into the __device__ array dc::dc_ms_trace the tool defines before
+// including this header.
+#ifdef DC_MS_TRACE
+#define DC_MS_TRACE_AT(slot)                                                      \
+    do {                                                                          \
+        unsigned long long t_;                                                    \
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                    \
+        dc_ms_trace[slot] = t_;                                                   \
+    } while (0)
+#else
+#define DC_MS_TRACE_AT(slot) do { } while (0)
+#endif
+
 __device__ __forceinline__ MsFold ms_fold_shfl_down(const MsFold& t, int off) {
     MsFold r;
     r.tot = __shfl_down_sync(0xffffffffu, t.tot, off);
@@ -172,6 +187,7 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
     __shared__ MsTupG redg[NW];
     __shared__ bool am_last;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) DC_MS_TRACE_AT(blockIdx.x * 16 + 0);
 
     // this warp's range [wbeg, wend) (RW is a multiple of SEG); CTA-local indices
     const long long cbase = min(n, (long long)blockIdx.x * NW * RW);
@@ -280,6 +296,7 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
 
     // ---- warps -> CTA summary (thread 0), in order
     if (lane == 0) red[warp] = acc.tup();
+    if (lane == 0) DC_MS_TRACE_AT(blockIdx.x * 16 + 1 + warp);
     __syncthreads();
     if (tid == 0) {
         MsTupG c = ms_empty<long long>();
@@ -289,6 +306,7 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
         am_last = atomicAdd(ticket, 1u) == gridDim.x - 1;
     }
     __syncthreads();
+    if (tid == 0) DC_MS_TRACE_AT(blockIdx.x * 16 + 15);
     if (!am_last) return;
 
     // ---- NK5: ordered combine of the per-CTA summaries (top levels)
@@ -317,6 +335,7 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
             ms_store(out_tup, a, off);
         }
         *ticket = 0u;
+        DC_MS_TRACE_AT(2047 * 16);
     }
 }
 

@@ -441,6 +441,163 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     if (V) store_tile(out_v + base, si, 0, count);
 }
 
+// ------------------------------------------- NK1 + one cluster level (f2)
+// Prototype of SURVEY f2's cluster/DSMEM levels (keys-only u32/i32): a
+// cluster of two CTAs sorts two adjacent tiles exactly like nk1_blocksort,
+// then runs ONE more merge level across the pair on chip: CTA r produces
+// outputs [r*TILE, (r+1)*TILE) of merge(tile 0, tile 1), reading the partner's
+// sorted tile straight out of its shared memory through the cluster window
+// (ld.shared::cluster, distributed shared memory; DC_NK1_CL_SWAP = 1: the two
+// CTAs first exchange the pieces each needs by coalesced DSMEM loads, then merge
+// locally).  The fused run width doubles
+// (2*TILE), so one global level fewer is left for the HBM passes.  Built with
+// -DDC_NK1_CLUSTER=2 (off by default: measured in DESIGN.md Sec. 5).
+#ifndef DC_NK1_CL_SWAP
+#define DC_NK1_CL_SWAP 1
+#endif
+__device__ __forceinline__ uint32_t ldcl(uint32_t addr) {   // shared::cluster address
+    uint32_t v;
+    asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+}
+__device__ __forceinline__ uint32_t cluster_map(uint32_t local_addr, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(local_addr), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+template <int NT, int IT, class K>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NT)
+nk1_blocksort_cl2(const uint32_t* __restrict__ in_k, uint32_t* __restrict__ out_k, long long n) {
+    static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
+    static_assert(!K::kNeedStable, "keys-only (pad-safe merges)");
+    constexpr int TILE = NT * IT;
+    extern __shared__ __align__(16) uint32_t smem[];
+    uint32_t* sk = smem;              // [TILE + IT pads]
+    __shared__ __align__(8) uint64_t bar;
+    const uint32_t SK = smem_addr(sk);
+    const uint32_t BAR = smem_addr(&bar);
+    const int tid = threadIdx.x;
+    const uint32_t rank = cluster_rank();
+    const long long base = (long long)blockIdx.x * TILE;
+    const int count = (int)max(0LL, min((long long)TILE, n - base));
+    const int body = count & ~3;
+
+    if (tid == 0) {
+        mbar_init(BAR, 1);
+        mbar_arrive_expect_tx(BAR, 4u * body);
+        if (body > 0) bulk_g2s(SK, in_k + base, 4u * body, BAR);
+    }
+    for (int e = body + tid; e < TILE; e += NT) sk[e] = e < count ? in_k[base + e] : K::kPad;
+    __syncthreads();
+    mbar_wait(BAR, 0);
+    uint32_t k[IT];
+    uint32_t ix[IT];
+#pragma unroll
+    for (int j = 0; j < IT; ++j) k[j] = sk[tid * IT + j];
+    thread_sort<K, IT, false>(k, ix);
+    merge_levels_bitonic<NT, IT, K>(k, sk);      // this tile sorted, in registers
+
+    // ---- the cluster level: tile 0 (A) and tile 1 (B) -> runs of 2*TILE
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < IT; ++j) sk[tid * IT + j] = k[j];
+    cluster_sync_all();                          // both sorted tiles visible in the cluster
+    const uint32_t A = cluster_map(SK, 0), B = cluster_map(SK, 1);
+#if DC_NK1_CL_SWAP
+    // Exchange, then merge locally.  c = #A among the first TILE outputs; CTA 0
+    // keeps A[0, c) and needs B[0, m), CTA 1 keeps B[m, TILE) and needs A[c, TILE)
+    // (m = TILE - c on both sides).  c by a 33-ary warp search over the
+    // cluster window (every CTA finds the same c), the partner's piece copied
+    // in coalesced DSMEM loads, a cluster barrier, then one local merge level.
+    __shared__ int s_c;
+    if (tid < 32) {
+        int lo = 0, hi = TILE;                   // c in [lo, hi]
+        while (hi > lo) {
+            const int step = (hi - lo + 31) / 32;   // probes lo + (l + 1) * step reach hi
+            const int q = lo + (tid + 1) * step;
+            // predicate(q): q <= c  <=>  A[q - 1] <= B[TILE - q] (A wins ties);
+            // monotone, so the probes that hold are a prefix
+            bool ok = false;
+            if (q <= hi) ok = !K::lt(ldcl(B + 4u * (TILE - q)), ldcl(A + 4u * (q - 1)));
+            const int nt = __popc(__ballot_sync(0xffffffffu, ok));
+            const int nlo = lo + nt * step;
+            hi = min(hi, lo + (nt + 1) * step - 1);
+            lo = nlo;
+        }
+        if (tid == 0) s_c = lo;
+    }
+    __syncthreads();
+    const int c = s_c, m = TILE - c;
+    // CTA 0: [0, c) own A, [c, TILE) <- B[0, m);  CTA 1: [0, m) <- A[c, TILE), [m, TILE) own B
+    const uint32_t src = rank == 0 ? B : A + 4u * c;
+    const int dst0 = rank == 0 ? c : 0;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+        const int e = j * NT + tid;
+        if (e < m) k[j] = ldcl(src + 4u * e);
+    }
+    cluster_sync_all();                          // every read of the partner's tile done
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+        const int e = j * NT + tid;
+        if (e < m) sk[dst0 + e] = k[j];
+    }
+    __syncthreads();
+    {
+        const int l1 = rank == 0 ? c : m;        // first run [0, l1), second [l1, TILE)
+        const int d = tid * IT;
+        const int i1 = corank_smem<K>(SK, l1, SK + 4u * l1, TILE - l1, d);
+        uint32_t srcs[IT];
+        serial_merge<K, IT, false>(SK + 4u * i1, SK + 4u * l1, SK + 4u * (l1 + d - i1),
+                                   SK + 4u * TILE, k, srcs);
+    }
+#else
+    for (int e = tid; e < IT + 1; e += NT) sk[TILE + e] = K::kPad;   // pads behind the run
+    cluster_sync_all();
+    const int d = (int)rank * TILE + tid * IT;
+    int lo = max(0, d - TILE), hi = min(d, TILE);
+    while (lo < hi) {
+        const int m = (lo + hi) >> 1;
+        if (!K::lt(ldcl(B + 4u * (d - 1 - m)), ldcl(A + 4u * m))) lo = m + 1;
+        else hi = m;
+    }
+    {   // pad-safe serial merge (merge_pad) over the cluster window
+        uint32_t ai = A + 4u * lo, bi = B + 4u * (d - lo);
+        uint32_t a = ldcl(ai), b = ldcl(bi);
+        const uint32_t c0 = ai + bi;
+#pragma unroll
+        for (int j = 0; j < IT; ++j) {
+            const bool p = K::lt(b, a);
+            k[j] = p ? b : a;
+            if (!p) ai += 4u;
+            bi = c0 + 4u * (j + 1) - ai;
+            const uint32_t v = ldcl(p ? bi : ai);
+            if (p) b = v; else a = v;
+        }
+    }
+    cluster_sync_all();                          // the partner is done reading this tile
+#endif
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < IT; ++j) sk[tid * IT + j] = k[j];
+    fence_proxy_async_smem();
+    __syncthreads();
+    // the pair's real keys come first (pads are maximum keys)
+    const long long cbase = base - (long long)rank * TILE;
+    const long long tot = max(0LL, min(2LL * TILE, n - cbase));
+    const int cnt = (int)max(0LL, min((long long)TILE, tot - (long long)rank * TILE));
+    if (cnt > 0) store_tile(out_k + cbase + (long long)rank * TILE, sk, 0, cnt);
+}
+
 // ------------------------------------------------------------------ NK2
 // Geometry of one merge level over [org, end) of a buffer: pairs of adjacent
 // runs (A of width wa, then B of width wb) with stride wa + wb starting at
