@@ -653,8 +653,8 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
 #ifndef DC_MS_TMA
 #define DC_MS_TMA 1
 #endif
-#ifndef DC_MS_P            // L: elements per lane per warp segment (L/4 odd)
-#define DC_MS_P 68
+#ifndef DC_MS_P            // L: elements per lane per warp segment (L/4 odd); r02b: 68 -> 76
+#define DC_MS_P 76
 #endif
 #ifndef DC_MS_S
 #define DC_MS_S 2
@@ -665,8 +665,12 @@ dc_status sort_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* v
 #ifndef DC_MS_J
 #define DC_MS_J 2
 #endif
-#ifndef DC_MS_VONLY       // values-only element fold + chunk-index recovery (measured slower)
-#define DC_MS_VONLY 0
+// Values-only element fold + chunk-label index recovery (DESIGN R21).  r02b:
+// default once the recovery became warp-parallel and the trees branch-free
+// (2^24: 26.86 us indexed fold, L = 68 -> 24.93 us values-only, L = 76; 50
+// steps each, profiles/r02b/nk4_sweep.txt); 0 keeps the indexed fold.
+#ifndef DC_MS_VONLY
+#define DC_MS_VONLY 1
 #endif
 // DC_MS_ROWS = 1: every lane folds one contiguous row, rows fed by 2-D TMA
 // tensor copies, 3 CTAs per SM (maxsub_rows.cuh).  Measured at 2^24 (r02,

@@ -14,7 +14,8 @@
 // folds the 32 lane summaries into the warp's running summary.  Warps, then
 // CTAs (atomic ticket, last CTA), are combined in order as before.
 //
-// VO (values-only, opt-in -DDC_MS_VONLY=1; measured slower): the per-element fold keeps only the four
+// VO (values-only, the default since r02b; -DDC_MS_VONLY=0 keeps the indexed
+// fold): the per-element fold keeps only the four
 // values (tot, pre, suf, best: two DADDs and three max) and no indices; each
 // lane's L-element chunk then enters the ordered combine as one leaf labelled
 // by its chunk start.  The combine's tie rules pick the lexicographically
@@ -107,40 +108,141 @@ struct MsVal {
     }
 };
 
-// Chunk [c, min(c+L, n)) staged at s[0..): smallest e maximising sum(x[c..e])
-// (the prefix end).
+// Warp-parallel scans over one staged chunk s[0, len) (len <= L): lane l owns
+// the E = ceil(L/32) elements [l*E, l*E + E).  Prefix sums P_j = s[0] + ...
+// + s[j] in int64 (exact); an exclusive warp scan of the lane totals gives
+// every lane its offset.
 template <int L>
-__device__ long long ms_first_max_prefix(const int* s, long long n, long long c) {
-    const int len = (int)min((long long)L, n - c);
-    long long P = 0, m = kMsNeg;
-    int k = 0;
-    for (int j = 0; j < len; ++j) {
-        P += s[j];
-        if (P > m) { m = P; k = j; }
+struct MsChunkScan {
+    static constexpr int E = (L + 31) / 32;
+    long long p[E];   // P_j of this lane's elements (j < len)
+    int len;
+    __device__ __forceinline__ MsChunkScan(const int* s, int len_) : len(len_) {
+        const int lane = threadIdx.x & 31;
+        long long run = 0;
+#pragma unroll
+        for (int t = 0; t < E; ++t) {
+            const int j = lane * E + t;
+            run += j < len ? s[j] : 0;
+            p[t] = run;
+        }
+        long long inc = run;                       // inclusive scan of lane totals
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const long long u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += u;
+        }
+        const long long off = inc - run;
+#pragma unroll
+        for (int t = 0; t < E; ++t) p[t] += off;
     }
-    return c + k;
+};
+// (value, index) reductions over the warp; ties -> smallest index.
+__device__ __forceinline__ void ms_warp_argmax(long long& v, int& i) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const long long ov = __shfl_xor_sync(0xffffffffu, v, o);
+        const int oi = __shfl_xor_sync(0xffffffffu, i, o);
+        if (ov > v || (ov == v && oi < i)) { v = ov; i = oi; }
+    }
 }
-// Chunk [c, c+len) staged at s: smallest start maximising the suffix sum.
-template <int L>
-__device__ long long ms_first_max_suffix(const int* s, long long n, long long c) {
-    const int len = (int)min((long long)L, n - c);
-    long long P = 0, m = 0;
-    int k = 0;
-    for (int j = 0; j + 1 < len; ++j) {
-        P += s[j];
-        if (P < m) { m = P; k = j + 1; }
+__device__ __forceinline__ void ms_warp_argmin(long long& v, int& i) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        const long long ov = __shfl_xor_sync(0xffffffffu, v, o);
+        const int oi = __shfl_xor_sync(0xffffffffu, i, o);
+        if (ov < v || (ov == v && oi < i)) { v = ov; i = oi; }
     }
-    return c + k;
+}
+// smallest e maximising P_e (the prefix end)
+template <int L>
+__device__ int ms_par_first_max_prefix(const MsChunkScan<L>& c) {
+    const int lane = threadIdx.x & 31;
+    long long v = kMsNeg;
+    int i = 1 << 30;
+#pragma unroll
+    for (int t = 0; t < MsChunkScan<L>::E; ++t) {
+        const int j = lane * MsChunkScan<L>::E + t;
+        if (j < c.len && c.p[t] > v) { v = c.p[t]; i = j; }
+    }
+    ms_warp_argmax(v, i);
+    return i;
+}
+// smallest start k maximising the suffix sum = smallest k minimising P_{k-1}
+// over k - 1 in [-1, len - 2] (P_{-1} = 0)
+template <int L>
+__device__ int ms_par_first_max_suffix(const MsChunkScan<L>& c) {
+    const int lane = threadIdx.x & 31;
+    long long v = 0;                          // P_{-1} = 0 at k = 0 (lane 0 only)
+    int i = lane == 0 ? 0 : (1 << 30);
+    if (lane != 0) v = -kMsNeg;
+#pragma unroll
+    for (int t = 0; t < MsChunkScan<L>::E; ++t) {
+        const int j = lane * MsChunkScan<L>::E + t;
+        if (j + 1 < c.len && (c.p[t] < v || (c.p[t] == v && j + 1 < i))) { v = c.p[t]; i = j + 1; }
+    }
+    ms_warp_argmin(v, i);
+    return i;
+}
+// lexicographically smallest (s, e) maximising sum(s..e) inside the chunk:
+// s_e = first argmin of Q_q = P_{q-1} over q in [0, e], e = first argmax of
+// P_e - Q_{s_e} (R21: that pair is the lexicographic minimum)
+template <int L>
+__device__ void ms_par_kadane(const MsChunkScan<L>& c, const int* s, int& bs, int& be) {
+    constexpr int E = MsChunkScan<L>::E;
+    const int lane = threadIdx.x & 31;
+    long long q[E];
+    int qi[E];
+    long long mn = -kMsNeg;                   // lane-local inclusive prefix min of Q
+    int mi = 1 << 30;
+#pragma unroll
+    for (int t = 0; t < E; ++t) {
+        const int j = lane * E + t;
+        const long long Q = j < c.len ? c.p[t] - s[j] : -kMsNeg;   // P_{j-1}
+        if (Q < mn) { mn = Q; mi = j; }
+        q[t] = mn;
+        qi[t] = mi;
+    }
+    // exclusive warp scan of the lane minima (ties keep the earlier index)
+    long long em = mn;
+    int ei = mi;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const long long um = __shfl_up_sync(0xffffffffu, em, o);
+        const int ui = __shfl_up_sync(0xffffffffu, ei, o);
+        if (lane >= o && (um < em || (um == em && ui < ei))) { em = um; ei = ui; }
+    }
+    long long pm = __shfl_up_sync(0xffffffffu, em, 1);
+    int pi = __shfl_up_sync(0xffffffffu, ei, 1);
+    if (lane == 0) { pm = -kMsNeg; pi = 1 << 30; }
+    long long v = kMsNeg;
+    int e = 1 << 30, sb = 0;
+#pragma unroll
+    for (int t = 0; t < E; ++t) {
+        const int j = lane * E + t;
+        long long m = q[t];
+        int mi2 = qi[t];
+        if (pm < m || (pm == m && pi < mi2)) { m = pm; mi2 = pi; }   // earlier lanes first
+        if (j < c.len) {
+            const long long val = c.p[t] - m;
+            if (val > v) { v = val; e = j; sb = mi2; }
+        }
+    }
+    int ee = e;
+    ms_warp_argmax(v, ee);                     // first e with the maximum value
+    bs = __shfl_sync(0xffffffffu, sb, ee / E);
+    be = ee;
 }
 
 // Exact indices from chunk labels (warp 0 of the last CTA).  a's pe/ss/bs/be
 // are chunk starts; on return they are element indices.  pe: first prefix
 // maximum inside its chunk; ss: first suffix maximum inside its chunk; best:
-// the in-chunk Kadane when start and end chunk coincide, else the
+// the in-chunk maximum subarray when start and end chunk coincide, else the
 // suffix-start / prefix-end scans of the two.  The (at most four) chunks are
-// first staged in shared memory by one coalesced warp load, so the four
-// scanning lanes read shared memory instead of waiting out one global-memory
-// latency per element (r01's serial scans of global memory cost ~17 us).
+// staged in shared memory by coalesced warp loads; every scan is a warp-
+// parallel int64 prefix scan with (value, index) reductions (r01's serial
+// scans of global memory cost ~17 us, r02's serial scans of shared memory
+// ~2-3 us on the critical path).
 template <int L>
 __device__ void ms_recover(const int* __restrict__ x, long long n, MsTupG& a, long long* rec) {
     __shared__ int stage[4][L];
@@ -151,23 +253,27 @@ __device__ void ms_recover(const int* __restrict__ x, long long n, MsTupG& a, lo
         for (int e = lane; e < L; e += 32)
             if (cs[q] + e < n) stage[q][e] = x[cs[q] + e];
     __syncwarp();
-    if (lane == 0) rec[0] = ms_first_max_prefix<L>(stage[0], n, a.pe);
-    if (lane == 1) rec[1] = ms_first_max_suffix<L>(stage[1], n, a.ss);
-    if (lane == 2) {
-        if (a.bs == a.be) {
-            MsFold f;
-            f.init();
-            const int len = (int)min((long long)L, n - a.bs);
-            for (int j = 0; j < len; ++j) f.step(stage[2][j], j);
-            rec[2] = a.bs + f.bs;
-            rec[3] = a.bs + f.be;
-        } else {
-            rec[2] = ms_first_max_suffix<L>(stage[2], n, a.bs);
-        }
+    int len[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) len[q] = (int)min((long long)L, n - cs[q]);
+    const MsChunkScan<L> c0(stage[0], len[0]);
+    const long long pe = a.pe + ms_par_first_max_prefix<L>(c0);
+    const MsChunkScan<L> c1(stage[1], len[1]);
+    const long long ss = a.ss + ms_par_first_max_suffix<L>(c1);
+    const MsChunkScan<L> c2(stage[2], len[2]);
+    long long bs, be;
+    if (a.bs == a.be) {
+        int s0, e0;
+        ms_par_kadane<L>(c2, stage[2], s0, e0);
+        bs = a.bs + s0;
+        be = a.bs + e0;
+    } else {
+        bs = a.bs + ms_par_first_max_suffix<L>(c2);
+        const MsChunkScan<L> c3(stage[3], len[3]);
+        be = a.be + ms_par_first_max_prefix<L>(c3);
     }
-    if (lane == 3 && a.bs != a.be) rec[3] = ms_first_max_prefix<L>(stage[3], n, a.be);
-    __syncwarp();
-    a.pe = rec[0]; a.ss = rec[1]; a.bs = rec[2]; a.be = rec[3];
+    (void)rec;
+    a.pe = pe; a.ss = ss; a.bs = bs; a.be = be;
 }
 
 template <int NT, int L, int S, int J, bool VO>
@@ -184,7 +290,6 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
     extern __shared__ __align__(16) int ms_smem[];            // [S][NW][SEG]
     __shared__ __align__(8) uint64_t bars[S][NW];
     __shared__ MsTup red[NW];
-    __shared__ MsTupG redg[NW];
     __shared__ bool am_last;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) DC_MS_TRACE_AT(blockIdx.x * 16 + 0);
@@ -294,38 +399,52 @@ nk4_maxsub_tma(const int* __restrict__ x, long long n, long long RW,
         }
     }
 
-    // ---- warps -> CTA summary (thread 0), in order
+    // ---- warps -> CTA summary: an ordered branch-free tree over the NW warp
+    // summaries in warp 0; the part is published with a release atomic on the
+    // ticket (acq_rel: the last CTA also acquires every other part)
     if (lane == 0) red[warp] = acc.tup();
     if (lane == 0) DC_MS_TRACE_AT(blockIdx.x * 16 + 1 + warp);
     __syncthreads();
-    if (tid == 0) {
-        MsTupG c = ms_empty<long long>();
-        for (int w = 0; w < NW; ++w) c = ms_combine(c, ms_widen(red[w], cbase));
-        ms_store(&parts[blockIdx.x], c, 0);
-        __threadfence();
-        am_last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+    if (warp == 0) {
+        MsTupG c = lane < NW ? ms_widen(red[lane], cbase) : ms_empty<long long>();
+        c = ms_warp_combine<NW>(c);
+        if (lane == 0) {
+            ms_store(&parts[blockIdx.x], c, 0);
+            unsigned int prev;
+            asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(prev) : "l"(ticket) : "memory");
+            am_last = prev == gridDim.x - 1;
+        }
     }
     __syncthreads();
     if (tid == 0) DC_MS_TRACE_AT(blockIdx.x * 16 + 15);
-    if (!am_last) return;
+    if (!am_last || warp != 0) return;         // (lane 0's acq_rel ticket + the barrier order the loads below)
 
-    // ---- NK5: ordered combine of the per-CTA summaries (top levels)
-    __threadfence();
+    // ---- NK5 (warp 0 of the last CTA): lane l folds the contiguous parts
+    // [l*per, (l+1)*per) (loads issued together), then one ordered warp tree
     const int np = gridDim.x;
-    const int per = (np + NT - 1) / NT;
+    const int per = (np + 31) / 32;
     MsTupG a = ms_empty<long long>();
-    for (int q = tid * per; q < min(np, tid * per + per); ++q) a = ms_combine(a, ms_load_cg(parts + q));
-    a = ms_block_combine<NT>(a, redg);
-    if (VO) {
-        __shared__ MsTupG s_a;
-        __shared__ long long rec[4];
-        if (tid == 0) s_a = a;
-        __syncthreads();
-        if (warp == 0) {
-            a = s_a;
-            ms_recover<L>(x, n, a, rec);
+    constexpr int kPer = 5;                    // parts loaded at once per lane (148 SMs: one round)
+    for (int q0 = 0; q0 < per; q0 += kPer) {
+        MsTupG v[kPer];
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            const int i = lane * per + q0 + q;
+            v[q] = (q0 + q < per && i < np) ? ms_load_cg(parts + i) : ms_empty<long long>();
         }
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) a = ms_combine(a, v[q]);
     }
+    a = ms_warp_combine<32>(a);
+    a.tot = __shfl_sync(0xffffffffu, a.tot, 0);
+    a.pre = __shfl_sync(0xffffffffu, a.pre, 0);
+    a.suf = __shfl_sync(0xffffffffu, a.suf, 0);
+    a.best = __shfl_sync(0xffffffffu, a.best, 0);
+    a.pe = __shfl_sync(0xffffffffu, a.pe, 0);
+    a.ss = __shfl_sync(0xffffffffu, a.ss, 0);
+    a.bs = __shfl_sync(0xffffffffu, a.bs, 0);
+    a.be = __shfl_sync(0xffffffffu, a.be, 0);
+    if (VO) ms_recover<L>(x, n, a, nullptr);
     if (tid == 0) {
         if (mode == 0) {
             out_res->sum = a.best;

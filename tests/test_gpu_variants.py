@@ -101,14 +101,15 @@ print("variant ok")
 
 
 def test_maxsub_values_only_fold(tmp_path):
-    """NK4 with the values-only element fold and chunk-label index recovery
-    (-DDC_MS_VONLY=1, R21): bit-exact (sum, start, end) and summary
+    """NK4 with the indexed element fold (-DDC_MS_VONLY=0, L = 68: the r02
+    default; the default build now folds values only and recovers indices from
+    chunk labels, R21): bit-exact (sum, start, end) and summary
     tuple on tie-heavy and degenerate inputs."""
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     from paper_conf_ipps_lopez_ortizss13_b200 import build
 
-    lib = build.build(out=str(tmp_path / "libdc_vonly.so"), defines=["DC_MS_VONLY=1"])
+    lib = build.build(out=str(tmp_path / "libdc_indexed.so"), defines=["DC_MS_VONLY=0", "DC_MS_P=68"])
     env = dict(os.environ, DC_LIB=lib)
     r = subprocess.run([sys.executable, "-c", VONLY_SCRIPT.format(root=ROOT)], env=env,
                        capture_output=True, text=True, timeout=900)

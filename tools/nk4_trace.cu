@@ -32,7 +32,7 @@ __global__ void empty_kernel(int* sink) {
 }
 
 int main(int argc, char** argv) {
-    constexpr int NT = 256, L = 68, S = 2, J = 2;
+    constexpr int NT = 256, L = 76, S = 2, J = 2;   // the library default
     const long long n = 1ll << 24;
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
@@ -53,7 +53,10 @@ int main(int argc, char** argv) {
     cudaMalloc(&ticket, 4);
     cudaMemset(ticket, 0, 4);
     cudaMalloc(&res, sizeof(dc_maxsub_result));
-    auto k = dc::nk4_maxsub_tma<NT, L, S, J, false>;
+#ifndef DC_MS_VONLY
+#define DC_MS_VONLY 1
+#endif
+    auto k = dc::nk4_maxsub_tma<NT, L, S, J, DC_MS_VONLY != 0>;
     const int smem = S * NT * L * 4;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     const long long warps = (long long)sms * (NT / 32), seg = 32ll * L;
