@@ -42,6 +42,13 @@ __device__ __forceinline__ T reduce_shfl_down(const T& v, int off) {
 
 // Ordered combine of one summary per thread (thread order = segment order);
 // the result is valid in thread 0.  red: NT/32 summaries of shared memory.
+// The shuffle trees are branch-free: every lane combines with its partner at
+// every level, and only lanes that are multiples of 2*off carry a meaningful
+// summary into the next level (a conditional combine makes the following
+// full-mask shuffles potentially divergent, and the compiler then guards each
+// level with a WARPSYNC fallback).  M::combine must therefore be total: it
+// also sees pairs of valid summaries in the wrong order, whose results are
+// discarded.
 template <class M, int NT>
 __device__ __forceinline__ typename M::T reduce_block(typename M::T t, typename M::T* red) {
     using T = typename M::T;
@@ -50,7 +57,7 @@ __device__ __forceinline__ typename M::T reduce_block(typename M::T t, typename 
 #pragma unroll
     for (int off = 1; off < 32; off <<= 1) {
         const T r = reduce_shfl_down(t, off);
-        if ((lane & (2 * off - 1)) == 0) t = M::combine(t, r);
+        t = M::combine(t, r);   // branch-free: only lanes = 0 mod 2*off stay meaningful
     }
     if (lane == 0) red[warp] = t;
     __syncthreads();
@@ -59,7 +66,7 @@ __device__ __forceinline__ typename M::T reduce_block(typename M::T t, typename 
 #pragma unroll
         for (int off = 1; off < NT / 32; off <<= 1) {
             const T r = reduce_shfl_down(t, off);
-            if ((lane & (2 * off - 1)) == 0) t = M::combine(t, r);
+            t = M::combine(t, r);   // branch-free: only lanes = 0 mod 2*off stay meaningful
         }
     }
     __syncthreads();
@@ -234,10 +241,11 @@ breadth_first_reduce_tma(const typename M::In* __restrict__ x, long long n, long
             for (int e = lane * L; e < min(cnt, lane * L + L); ++e)
                 f = M::combine(f, M::leaf(e < body ? seg_ptr(s)[e] : x[g0 + e], g0 + e));
         }
+        __syncwarp();                                           // reconverge before the tree
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {                      // ordered warp tree
             const T r = reduce_shfl_down(f, o);
-            if ((lane & (2 * o - 1)) == 0) f = M::combine(f, r);
+            f = M::combine(f, r);   // branch-free (no divergent shuffles)
         }
         if (lane == 0) acc = M::combine(acc, f);
         __syncwarp();

@@ -539,6 +539,13 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
     }
 
     // ---------------------------------------------------------- consumers
+// Stage-2 co-ranks seeded by one 32-ary warp search per warp (each lane then
+// searches [c(D), c(D) + lane*IT] only).  Measured r02b at 2^28 u32: merges
+// 3.761 vs 3.702 ms per sort (the warp rounds cost more issue slots than the
+// ~5 binary steps per lane they save; profiles/r02b/m4_warp_corank.txt): off.
+#ifndef DC_M4_WARP_CORANK
+#define DC_M4_WARP_CORANK 0
+#endif
 #ifndef DC_M4_SKIP   // measurement knob: bit 0 skips stage 1, bit 1 stage 2
 #define DC_M4_SKIP 0
 #endif
@@ -621,6 +628,28 @@ nk3_merge4(const Pass4 P, uint32_t* __restrict__ dst_k, uint32_t* __restrict__ d
                 // stage 2: bitonic merge of X (ascending) and Y (descending)
                 const uint32_t Ab = B0, Bb = B0 + 4u * (total - diag);
                 int lo = max(0, diag - ny), hi = min(diag, nx);
+#if DC_M4_WARP_CORANK
+                if (__activemask() == 0xffffffffu) {   // (the tile's last warp may be partial)
+                    // The warp's lanes own consecutive diagonals D + l*IT, so
+                    // c(D + l*IT) lies in [c(D), c(D) + l*IT].  c(D) by a 32-ary
+                    // warp search (probes spread over the window, ~3 rounds),
+                    // then every lane's binary search starts from that window.
+                    const int D = diag - lane * IT;
+                    int wlo = max(0, D - ny), whi = min(D, nx);
+                    const uint32_t Bd = B0 + 4u * (total - D);
+                    while (whi > wlo) {
+                        const int step = (whi - wlo + 31) >> 5;
+                        const int q = wlo + (lane + 1) * step - 1;   // P(q): q < c(D)
+                        const bool ok = q < whi && !K::lt(lds(Bd + 4u * q), lds(Ab + 4u * q));
+                        const int nt = __popc(__ballot_sync(0xffffffffu, ok));
+                        const int nlo = wlo + nt * step;
+                        whi = min(whi, wlo + (nt + 1) * step - 1);
+                        wlo = nlo;
+                    }
+                    lo = max(lo, wlo);
+                    hi = min(hi, wlo + lane * IT);
+                }
+#endif
                 while (lo < hi) {
                     const int mid = (lo + hi) >> 1;
                     if (!K::lt(lds(Bb + 4u * mid), lds(Ab + 4u * mid))) lo = mid + 1;
