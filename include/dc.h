@@ -103,8 +103,9 @@ dc_status dc_plan_levels(dc_plan_t plan, int32_t *num_levels, int64_t *nodes,
  * ceil(log2(ceil(n/tile))) levels remain, executed in hbm_passes passes over
  * HBM (one or two levels per pass).  Tile class and pass kind are the
  * planner's choice (dc_model_sort_schedule) unless forced with
- * dc_plan_set_tile_class / dc_plan_set_two_level.  Any output pointer may be
- * NULL. */
+ * dc_plan_set_tile_class / dc_plan_set_two_level; with NK1 cluster levels
+ * (dc_plan_set_nk1_cluster) `tile` is the cluster's fused run width.  Any
+ * output pointer may be NULL. */
 dc_status dc_plan_schedule(dc_plan_t plan, dc_key_type key_type, int32_t with_vals,
                            int32_t *tile, int32_t *fused_levels, int32_t *global_passes,
                            int32_t *hbm_passes);
@@ -118,6 +119,18 @@ dc_status dc_plan_set_two_level(dc_plan_t plan, int32_t enable);
 /* Force the NK1 tile class (1 quarter-size tiles of 128-thread CTAs, 2 full
  * tiles) or leave it to the planner (0, default).  Results are identical. */
 dc_status dc_plan_set_tile_class(dc_plan_t plan, int32_t tile_class);
+
+/* NK1 cluster levels for keys-only u32/i32 sorts: a cluster of cs
+ * CTAs (cs = 2, 4, 8 or 16; a thread-block cluster, distributed shared
+ * memory) sorts cs adjacent tiles and runs log2(cs) more merge levels of Alg 7
+ * on chip -- every CTA gathers the inputs of its output range
+ * from its partners' shared memory, then merges locally -- so the fused runs
+ * are cs tiles wide and log2(cs) global levels fewer remain.  cs = 1 turns it
+ * off, 0 (default) leaves it to the planner's rule (small sorts, where every
+ * global level is a latency-bound launch).  Key-value and
+ * f32 sorts ignore it.  Results are identical.  DC_ERR_INVALID_ARG for any
+ * other cs. */
+dc_status dc_plan_set_nk1_cluster(dc_plan_t plan, int32_t cs);
 
 /* Enable (default) or disable the fused partition of L2-resident sorts (n <
  * 2^23): every one-level merge CTA finds the co-ranks of its own output tile

@@ -65,6 +65,7 @@ _SIGS = {
                           ctypes.POINTER(_I32), ctypes.POINTER(_I32)], ctypes.c_int),
     "dc_plan_set_two_level": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_tile_class": ([_P, _I32], ctypes.c_int),
+    "dc_plan_set_nk1_cluster": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_fused_partition": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_graphs": ([_P, _I32], ctypes.c_int),
     "dc_plan_set_pipeline": ([_P, _I32], ctypes.c_int),
@@ -361,6 +362,12 @@ class Plan:
     def set_tile_class(self, tile_class: int) -> None:
         """NK1 tile class: 1 quarter-size, 2 full, 0 planner (default)."""
         _check(lib().dc_plan_set_tile_class(self._h, tile_class))
+
+    def set_nk1_cluster(self, cs: int) -> None:
+        """NK1 cluster size for keys-only u32/i32 sorts: 2/4/8/16
+        fuse log2(cs) more levels through distributed shared memory, 1 off,
+        0 the planner's rule (default)."""
+        _check(lib().dc_plan_set_nk1_cluster(self._h, int(cs)))
 
     def scratch_bytes(self, with_vals: bool = False) -> int:
         b = ctypes.c_size_t()

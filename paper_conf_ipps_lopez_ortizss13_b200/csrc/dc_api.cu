@@ -386,7 +386,7 @@ dc_status pass4(dc_plan_t p, const dc::Pass4& P, int tiles, dc::Cut4* cuts, uint
 // the output buffer.
 template <class K, bool V, bool SMALL>
 dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_k,
-                     uint32_t* out_v, bool two_level) {
+                     uint32_t* out_v, bool two_level, int cs) {
     const int64_t n = p->n;
     const bool hv = V;
     dc_status st = ensure_scratch(p, hv);
@@ -415,13 +415,11 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     // Levels over HBM: P = ceil(log2(ceil(n/tile))).  Keys-only sorts fold
     // two levels into one pass (4-way groups, sort4_kernels.cuh); with P odd
     // one single-level pass goes first.
-    // f2 prototype (-DDC_NK1_CLUSTER=2, keys-only full tiles): NK1 runs one more
-    // level across each cluster of two CTAs, so the fused runs are 2 tiles wide.
-#ifndef DC_NK1_CLUSTER
-#define DC_NK1_CLUSTER 0
-#endif
-    constexpr bool kCl = DC_NK1_CLUSTER == 2 && !V && !K::kNeedStable && !SMALL;
-    const int64_t ftile = kCl ? 2 * (int64_t)C.tile() : (int64_t)C.tile();
+    // f2: NK1 cluster levels (keys-only u32/i32): the fused runs are cs tiles wide.
+    constexpr bool kClCapable = !V && !K::kNeedStable;
+    if (!kClCapable) cs = 1;
+    const bool kCl = cs > 1;
+    const int64_t ftile = (int64_t)C.tile() * cs;
     const int P = global_passes(n, ftile);
     constexpr bool kTwoCapable = true;
     const bool two = two_level && P >= 2;
@@ -519,16 +517,30 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
     } else {
         // NK1: base cases + fused bottom levels (reads the caller's buffer).
         TimedScope ts(p, DC_KERNEL_NK1_BLOCKSORT);
-        if constexpr (kCl) {
-            auto* kc = dc::nk1_blocksort_cl2<C.nt1, C.it1, K>;
-            const int smem = dc::tile_words(C.tile(), C.it1 + 4) * 4;
-            static PerDevice cl_attr;
-            if (!cl_attr.get()) {
-                DC_CUDA(p, cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-                cl_attr.set(1);
+        if (kCl) {
+            if constexpr (kClCapable) {
+                auto* kc = dc::nk1_blocksort_cl<C.nt1, C.it1, K>;
+                const int smem = dc::tile_words(C.tile(), C.it1 + 4) * 4;
+                static PerDevice cl_attr;
+                if (!cl_attr.get()) {
+                    DC_CUDA(p, cudaFuncSetAttribute(kc, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+                    DC_CUDA(p, cudaFuncSetAttribute(kc, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
+                    cl_attr.set(1);
+                }
+                cudaLaunchConfig_t cfg = {};
+                cfg.gridDim = dim3((unsigned)(num_tiles(n, ftile) * cs));
+                cfg.blockDim = dim3(C.nt1);
+                cfg.dynamicSmemBytes = (size_t)smem;
+                cfg.stream = p->stream;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = (unsigned)cs;
+                at[0].val.clusterDim.y = 1;
+                at[0].val.clusterDim.z = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                DC_CUDA(p, cudaLaunchKernelEx(&cfg, kc, (const uint32_t*)keys, cur_k, (long long)n));
             }
-            const unsigned grid = (unsigned)(num_tiles(n, 2 * (int64_t)C.tile()) * 2);
-            kc<<<grid, C.nt1, smem, p->stream>>>(keys, cur_k, n);
         } else {
             k1<<<(unsigned)num_tiles(n, C.tile()), C.nt1, nk1_smem_bytes(C, hv), p->stream>>>(
                 keys, vals, cur_k, cur_v, n);
@@ -577,21 +589,33 @@ dc_status sort_typed(dc_plan_t p, uint32_t* keys, uint32_t* vals, uint32_t* out_
 // forces one of them.
 struct Decision {
     bool small, two;
+    int cs;   // NK1 cluster size (1: plain NK1)
 };
+// NK1 cluster rule (keys-only u32/i32).  Measured r02b (tools/cluster_sweep.py,
+// profiles/r02b/cluster_sweep.txt: u32, n = 2^16..2^26, cs = 1..16, both tile
+// classes and pass kinds): a cluster level costs about what the global level it
+// removes costs at small n (both latency-bound, ~5-8 us) and more at large n
+// (0.40 vs 0.26 ms per level at 2^28): no size gains more than one ~2 us
+// timer quantum (2^18: cs = 8 57.3 vs 59.4 us), most lose.  The rule keeps
+// them off; dc_plan_set_nk1_cluster forces them.
+int cluster_rule(int64_t, bool) { return 1; }
 Decision decide(dc_plan_t p, dc_key_type kt, bool vals) {
     dc_sort_schedule s{};
     dc_model_sort_schedule(p->n, kt, vals ? 1 : 0, p->tile_class, p->two_force, &s);
-    return {s.tile_class == 1, s.two_level != 0};
+    const bool small = s.tile_class == 1;
+    int cs = 1;
+    if (!vals && kt != DC_KEY_F32) cs = p->nk1_cluster ? p->nk1_cluster : cluster_rule(p->n, small);
+    return {small, s.two_level != 0, cs};
 }
 
 template <class K>
 dc_status sort_kv_dispatch(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals,
                            uint32_t* ok, uint32_t* ov) {
     const Decision d = decide(p, kt, vals != nullptr);
-    if (vals) return d.small ? sort_typed<K, true, true>(p, keys, vals, ok, ov, d.two)
-                             : sort_typed<K, true, false>(p, keys, vals, ok, ov, d.two);
-    return d.small ? sort_typed<K, false, true>(p, keys, nullptr, ok, nullptr, d.two)
-                   : sort_typed<K, false, false>(p, keys, nullptr, ok, nullptr, d.two);
+    if (vals) return d.small ? sort_typed<K, true, true>(p, keys, vals, ok, ov, d.two, 1)
+                             : sort_typed<K, true, false>(p, keys, vals, ok, ov, d.two, 1);
+    return d.small ? sort_typed<K, false, true>(p, keys, nullptr, ok, nullptr, d.two, d.cs)
+                   : sort_typed<K, false, false>(p, keys, nullptr, ok, nullptr, d.two, d.cs);
 }
 
 dc_status sort_direct(dc_plan_t p, dc_key_type kt, uint32_t* keys, uint32_t* vals, uint32_t* ok,
@@ -1094,11 +1118,12 @@ dc_status dc_plan_schedule(dc_plan_t p, dc_key_type kt, int32_t with_vals, int32
         return fail(DC_ERR_INVALID_ARG, "unknown key type");
     const Decision d = decide(p, kt, with_vals != 0);
     const SortCfg c = cfg_for_runtime(kt, with_vals != 0, d.small);
-    if (tile) *tile = c.tile();
-    int f = 0;   // levels of the binary tree inside one tile: ceil(log2(tile))
-    while ((1 << f) < c.tile()) ++f;
+    const int64_t ft = (int64_t)c.tile() * d.cs;   // fused run width
+    if (tile) *tile = (int32_t)ft;
+    int f = 0;   // levels of the binary tree inside one fused run: ceil(log2(run))
+    while (((int64_t)1 << f) < ft) ++f;
     if (fused_levels) *fused_levels = f;
-    const int P = global_passes(p->n, c.tile());
+    const int P = global_passes(p->n, ft);
     if (passes) *passes = P;
     const bool two = d.two && P >= 2;
     if (hbm_passes) *hbm_passes = two ? (P % 2) + (P - P % 2) / 2 : P;
@@ -1117,6 +1142,15 @@ dc_status dc_plan_set_tile_class(dc_plan_t p, int32_t tile_class) {
     if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
     if (tile_class < 0 || tile_class > 2) return fail(DC_ERR_INVALID_ARG, "tile_class must be 0, 1 or 2");
     p->tile_class = tile_class;
+    drop_graphs(p);
+    return DC_OK;
+}
+
+dc_status dc_plan_set_nk1_cluster(dc_plan_t p, int32_t cs) {
+    if (!p) return fail(DC_ERR_INVALID_ARG, "plan is NULL");
+    if (!(cs == 0 || cs == 1 || cs == 2 || cs == 4 || cs == 8 || cs == 16))
+        return fail(DC_ERR_INVALID_ARG, "cs must be 0, 1, 2, 4, 8 or 16");
+    p->nk1_cluster = cs;
     drop_graphs(p);
     return DC_OK;
 }

@@ -75,6 +75,10 @@ struct dc_plan_s {
     int two_force = -1;       // -1 planner; 0 one level per HBM pass; 1 two levels (4-way)
     int tile_class = 0;       // 0 planner; 1 quarter-size tiles; 2 full tiles
     bool fuse_partition = true;   // small sorts: merge CTAs find their own co-ranks
+    // NK1 cluster size for keys-only u32/i32 sorts (f2: log2(CS) more levels on
+    // chip through distributed shared memory): 0 the planner's rule, 1 off,
+    // 2/4/8/16 forced
+    int nk1_cluster = 0;
     // D&C sum (f4): per-CTA parts + ticket + result
     long long* sum_state = nullptr;
     int sum_grid = 0;

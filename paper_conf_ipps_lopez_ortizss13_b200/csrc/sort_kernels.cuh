@@ -441,20 +441,30 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     if (V) store_tile(out_v + base, si, 0, count);
 }
 
-// ------------------------------------------- NK1 + one cluster level (f2)
-// Prototype of SURVEY f2's cluster/DSMEM levels (keys-only u32/i32): a
-// cluster of two CTAs sorts two adjacent tiles exactly like nk1_blocksort,
-// then runs ONE more merge level across the pair on chip: CTA r produces
-// outputs [r*TILE, (r+1)*TILE) of merge(tile 0, tile 1), reading the partner's
-// sorted tile straight out of its shared memory through the cluster window
-// (ld.shared::cluster, distributed shared memory; DC_NK1_CL_SWAP = 1: the two
-// CTAs first exchange the pieces each needs by coalesced DSMEM loads, then merge
-// locally).  The fused run width doubles
-// (2*TILE), so one global level fewer is left for the HBM passes.  Built with
-// -DDC_NK1_CLUSTER=2 (off by default: measured in DESIGN.md Sec. 5).
-#ifndef DC_NK1_CL_SWAP
-#define DC_NK1_CL_SWAP 1
-#endif
+// ------------------------------------------ NK1 + cluster levels (f2)
+// SURVEY f2's cluster / distributed-shared-memory levels (keys-only u32/i32):
+// a cluster of CS CTAs (CS = 2, 4, 8 or 16, a launch attribute) sorts CS
+// adjacent tiles exactly like nk1_blocksort, then runs log2(CS) more merge
+// levels on chip.  At cluster level g (runs of g tiles -> 2g tiles), CTA r of
+// a group pair [p0, p0 + 2g) produces the outputs [(r - p0)*TILE, +TILE) of
+// merge(A, B), A = tiles p0 .. p0+g-1, B = the next g tiles, each tile sorted
+// in its own CTA's shared memory:
+//   1. two warps find the co-ranks c(d0), c(d0 + TILE) of its output range by
+//      33-ary warp searches through the cluster window (ld.shared::cluster);
+//   2. every thread gathers its share of the TILE inputs A[c0, c1) and
+//      B[d0 - c0, d0 + TILE - c1) from the owning CTAs (coalesced DSMEM loads
+//      into registers);
+//   3. a cluster barrier (every read of every tile done), the inputs go to the
+//      CTA's own shared memory as two sorted runs, and one local merge-path
+//      level (co-rank + serial merge) produces the CTA's TILE outputs.
+// The fused runs are CS tiles wide, so log2(CS) global levels fewer remain.
+// Every level is the stable merge of adjacent runs (A wins ties), i.e. Alg 7's
+// combine; for keys-only sorts the result is the sorted multiset.
+// Measured: a cluster level costs more than a global level
+// at 2^28 but far less than one at small n, where every global level is a
+// latency-bound launch; the planner's cluster rule (dc_api.cu) picks CS.
+// (A first prototype merged straight out of the partner's shared memory --
+// every serial-merge step a DSMEM load -- and cost 0.98 ms per 2^28 level.)
 __device__ __forceinline__ uint32_t ldcl(uint32_t addr) {   // shared::cluster address
     uint32_t v;
     asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr));
@@ -470,23 +480,59 @@ __device__ __forceinline__ uint32_t cluster_rank() {
     asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
     return r;
 }
+__device__ __forceinline__ uint32_t cluster_size() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r));
+    return r;
+}
 __device__ __forceinline__ void cluster_sync_all() {
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// Element i of a run of g tiles starting at cluster rank `first` (tile t of
+// the run lives in CTA first + t, word i mod TILE of its tile buffer SK).
+template <int TILE>
+__device__ __forceinline__ uint32_t run_at(uint32_t SK, uint32_t first, int i) {
+    const int t = i / TILE;
+    return ldcl(cluster_map(SK + 4u * (uint32_t)(i - t * TILE), first + (uint32_t)t));
+}
+
+// c(d) = #A among the first d outputs of merge(A, B), both runs of width W
+// (A wins ties), by a 33-ary search of one warp through the cluster window:
+// P(q) = "q <= c" = A[q - 1] <= B[d - q] is monotone, probes that hold are a
+// prefix.  Returns c in every lane.
+template <class K, int TILE>
+__device__ __forceinline__ int cluster_corank(uint32_t SK, uint32_t fa, uint32_t fb, int W, int d) {
+    const int lane = threadIdx.x & 31;
+    int lo = max(0, d - W), hi = min(d, W);
+    while (hi > lo) {
+        const int step = (hi - lo + 31) >> 5;       // probes lo + (l + 1) * step reach hi
+        const int q = lo + (lane + 1) * step;
+        bool ok = false;
+        if (q <= hi) ok = !K::lt(run_at<TILE>(SK, fb, d - q), run_at<TILE>(SK, fa, q - 1));
+        const int nt = __popc(__ballot_sync(0xffffffffu, ok));
+        const int nlo = lo + nt * step;
+        hi = min(hi, lo + (nt + 1) * step - 1);
+        lo = nlo;
+    }
+    return lo;
+}
+
 template <int NT, int IT, class K>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NT)
-nk1_blocksort_cl2(const uint32_t* __restrict__ in_k, uint32_t* __restrict__ out_k, long long n) {
+__global__ void __launch_bounds__(NT)
+nk1_blocksort_cl(const uint32_t* __restrict__ in_k, uint32_t* __restrict__ out_k, long long n) {
     static_assert(IT % 2 == 1, "odd items per thread keep the blocked layout conflict-free");
-    static_assert(!K::kNeedStable, "keys-only (pad-safe merges)");
+    static_assert(!K::kNeedStable, "keys-only");
+    static_assert(NT >= 64, "two warps search the co-ranks");
     constexpr int TILE = NT * IT;
     extern __shared__ __align__(16) uint32_t smem[];
-    uint32_t* sk = smem;              // [TILE + IT pads]
+    uint32_t* sk = smem;              // [TILE + slack]
     __shared__ __align__(8) uint64_t bar;
+    __shared__ int s_c[2];
     const uint32_t SK = smem_addr(sk);
     const uint32_t BAR = smem_addr(&bar);
     const int tid = threadIdx.x;
-    const uint32_t rank = cluster_rank();
+    const uint32_t rank = cluster_rank(), CS = cluster_size();
     const long long base = (long long)blockIdx.x * TILE;
     const int count = (int)max(0LL, min((long long)TILE, n - base));
     const int body = count & ~3;
@@ -506,96 +552,48 @@ nk1_blocksort_cl2(const uint32_t* __restrict__ in_k, uint32_t* __restrict__ out_
     thread_sort<K, IT, false>(k, ix);
     merge_levels_bitonic<NT, IT, K>(k, sk);      // this tile sorted, in registers
 
-    // ---- the cluster level: tile 0 (A) and tile 1 (B) -> runs of 2*TILE
-    __syncthreads();
+#pragma unroll 1
+    for (uint32_t g = 1; g < CS; g <<= 1) {
+        __syncthreads();
 #pragma unroll
-    for (int j = 0; j < IT; ++j) sk[tid * IT + j] = k[j];
-    cluster_sync_all();                          // both sorted tiles visible in the cluster
-    const uint32_t A = cluster_map(SK, 0), B = cluster_map(SK, 1);
-#if DC_NK1_CL_SWAP
-    // Exchange, then merge locally.  c = #A among the first TILE outputs; CTA 0
-    // keeps A[0, c) and needs B[0, m), CTA 1 keeps B[m, TILE) and needs A[c, TILE)
-    // (m = TILE - c on both sides).  c by a 33-ary warp search over the
-    // cluster window (every CTA finds the same c), the partner's piece copied
-    // in coalesced DSMEM loads, a cluster barrier, then one local merge level.
-    __shared__ int s_c;
-    if (tid < 32) {
-        int lo = 0, hi = TILE;                   // c in [lo, hi]
-        while (hi > lo) {
-            const int step = (hi - lo + 31) / 32;   // probes lo + (l + 1) * step reach hi
-            const int q = lo + (tid + 1) * step;
-            // predicate(q): q <= c  <=>  A[q - 1] <= B[TILE - q] (A wins ties);
-            // monotone, so the probes that hold are a prefix
-            bool ok = false;
-            if (q <= hi) ok = !K::lt(ldcl(B + 4u * (TILE - q)), ldcl(A + 4u * (q - 1)));
-            const int nt = __popc(__ballot_sync(0xffffffffu, ok));
-            const int nlo = lo + nt * step;
-            hi = min(hi, lo + (nt + 1) * step - 1);
-            lo = nlo;
+        for (int j = 0; j < IT; ++j) sk[tid * IT + j] = k[j];
+        cluster_sync_all();                      // every CTA's run piece visible
+        const uint32_t p0 = rank & ~(2 * g - 1);
+        const int W = (int)g * TILE;
+        const int d0 = (int)(rank - p0) * TILE;
+        if (tid < 64) {
+            const int c = cluster_corank<K, TILE>(SK, p0, p0 + g, W, d0 + (tid >> 5) * TILE);
+            if ((tid & 31) == 0) s_c[tid >> 5] = c;
         }
-        if (tid == 0) s_c = lo;
-    }
-    __syncthreads();
-    const int c = s_c, m = TILE - c;
-    // CTA 0: [0, c) own A, [c, TILE) <- B[0, m);  CTA 1: [0, m) <- A[c, TILE), [m, TILE) own B
-    const uint32_t src = rank == 0 ? B : A + 4u * c;
-    const int dst0 = rank == 0 ? c : 0;
-#pragma unroll
-    for (int j = 0; j < IT; ++j) {
-        const int e = j * NT + tid;
-        if (e < m) k[j] = ldcl(src + 4u * e);
-    }
-    cluster_sync_all();                          // every read of the partner's tile done
-#pragma unroll
-    for (int j = 0; j < IT; ++j) {
-        const int e = j * NT + tid;
-        if (e < m) sk[dst0 + e] = k[j];
-    }
-    __syncthreads();
-    {
-        const int l1 = rank == 0 ? c : m;        // first run [0, l1), second [l1, TILE)
-        const int d = tid * IT;
-        const int i1 = corank_smem<K>(SK, l1, SK + 4u * l1, TILE - l1, d);
-        uint32_t srcs[IT];
-        serial_merge<K, IT, false>(SK + 4u * i1, SK + 4u * l1, SK + 4u * (l1 + d - i1),
-                                   SK + 4u * TILE, k, srcs);
-    }
-#else
-    for (int e = tid; e < IT + 1; e += NT) sk[TILE + e] = K::kPad;   // pads behind the run
-    cluster_sync_all();
-    const int d = (int)rank * TILE + tid * IT;
-    int lo = max(0, d - TILE), hi = min(d, TILE);
-    while (lo < hi) {
-        const int m = (lo + hi) >> 1;
-        if (!K::lt(ldcl(B + 4u * (d - 1 - m)), ldcl(A + 4u * m))) lo = m + 1;
-        else hi = m;
-    }
-    {   // pad-safe serial merge (merge_pad) over the cluster window
-        uint32_t ai = A + 4u * lo, bi = B + 4u * (d - lo);
-        uint32_t a = ldcl(ai), b = ldcl(bi);
-        const uint32_t c0 = ai + bi;
+        __syncthreads();
+        const int c0 = s_c[0], c1 = s_c[1];
+        const int a = c1 - c0;                   // A elements of this CTA's outputs
+        const int b0 = d0 - c0;                  // first B element
 #pragma unroll
         for (int j = 0; j < IT; ++j) {
-            const bool p = K::lt(b, a);
-            k[j] = p ? b : a;
-            if (!p) ai += 4u;
-            bi = c0 + 4u * (j + 1) - ai;
-            const uint32_t v = ldcl(p ? bi : ai);
-            if (p) b = v; else a = v;
+            const int e = j * NT + tid;          // input e of TILE: A part, then B part
+            k[j] = e < a ? run_at<TILE>(SK, p0, c0 + e) : run_at<TILE>(SK, p0 + g, b0 + e - a);
         }
+        cluster_sync_all();                      // every read of every tile done
+#pragma unroll
+        for (int j = 0; j < IT; ++j) sk[j * NT + tid] = k[j];
+        __syncthreads();
+        const int d = tid * IT;
+        const int i1 = corank_smem<K>(SK, a, SK + 4u * a, TILE - a, d);
+        uint32_t srcs[IT];
+        serial_merge<K, IT, false>(SK + 4u * i1, SK + 4u * a, SK + 4u * (a + d - i1),
+                                   SK + 4u * TILE, k, srcs);
     }
-    cluster_sync_all();                          // the partner is done reading this tile
-#endif
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < IT; ++j) sk[tid * IT + j] = k[j];
     fence_proxy_async_smem();
     __syncthreads();
-    // the pair's real keys come first (pads are maximum keys)
+    // the cluster's real keys come first (pads are maximum keys)
     const long long cbase = base - (long long)rank * TILE;
-    const long long tot = max(0LL, min(2LL * TILE, n - cbase));
+    const long long tot = max(0LL, min((long long)CS * TILE, n - cbase));
     const int cnt = (int)max(0LL, min((long long)TILE, tot - (long long)rank * TILE));
-    if (cnt > 0) store_tile(out_k + cbase + (long long)rank * TILE, sk, 0, cnt);
+    if (cnt > 0) store_tile(out_k + base, sk, 0, cnt);
 }
 
 // ------------------------------------------------------------------ NK2

@@ -606,3 +606,47 @@ def test_launch_counts(dc, n, fused):
     single = P - 2 * (P - H)          # one-level passes; the rest are two-level passes
     per_single = 1 if (fused and s["tile"] == 128 * 49) else 2   # quarter tiles: fused partition
     assert p.launch_count() == 1 + per_single * single + 2 * (H - single)
+
+
+# ---------------------------------------------------------------- f2 clusters
+@pytest.mark.parametrize("cs", [2, 4, 8, 16])
+@pytest.mark.parametrize("tile_class", [1, 2])
+@pytest.mark.parametrize("key_type", ["u32", "i32"])
+def test_sort_nk1_cluster_levels(dc, oracle_mod, cs, tile_class, key_type):
+    """NK1 with log2(cs) cluster levels (distributed shared memory,
+    nk1_blocksort_cl): bit-exact against the oracle for a partial last
+    cluster, a ragged tail, a single tile, both pass kinds."""
+    tile = 6272 if tile_class == 1 else 25088
+    for n, dist in [(1, "uniform"), (tile - 3, "few"), (cs * tile + 1, "uniform"),
+                    (3 * cs * tile + 4099, "uniform"), (5 * cs * tile // 2 + 17, "reverse"),
+                    (1 << 20, "sorted")]:
+        keys = dcgen.sort_keys(n, dist, seed=47, key_type=key_type, device="cuda")
+        ka = keys.cpu().numpy()
+        ka = ka.view(np.uint32) if key_type == "u32" else ka.view(np.int32)
+        ek = oracle_mod.mergesort(ka, key_type=key_type)
+        for two in (False, True):
+            k = keys.clone()
+            plan = dc.Plan(n)
+            plan.set_tile_class(tile_class)
+            plan.set_two_level(two)
+            plan.set_nk1_cluster(cs)
+            assert plan.schedule(key_type)["tile"] == tile * cs
+            plan.sort_(k, None, key_type=key_type)
+            torch.cuda.synchronize()
+            assert np.array_equal(k.cpu().numpy().view(ek.dtype), ek), (n, dist, two)
+
+
+def test_sort_nk1_cluster_ignored_for_stable_sorts(dc, oracle_mod):
+    """Key-value and f32 sorts run the plain NK1 whatever the cluster setting."""
+    n = 3 * 25088 + 5
+    plan = dc.Plan(n)
+    plan.set_nk1_cluster(8)
+    assert plan.schedule("u32", with_vals=True)["tile"] in (8448, 4224)
+    keys = dcgen.sort_keys(n, "few", seed=5, device="cuda")
+    vals = dcgen.sort_vals(n, device="cuda")
+    ek, ev = oracle_mod.mergesort(keys.cpu().numpy().view(np.uint32),
+                                  np.arange(n, dtype=np.uint32))
+    plan.sort_(keys, vals, key_type="u32")
+    torch.cuda.synchronize()
+    assert np.array_equal(keys.cpu().numpy().view(np.uint32), ek)
+    assert np.array_equal(vals.cpu().numpy().view(np.uint32), ev)

@@ -132,49 +132,3 @@ def test_maxsub_rows_kernel(tmp_path):
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     assert "variant ok" in r.stdout
 
-
-CLUSTER_SCRIPT = r"""
-import sys
-import numpy as np
-import torch
-sys.path.insert(0, {root!r})
-import dcgen, oracle
-import paper_conf_ipps_lopez_ortizss13_b200 as dc
-oracle.build()
-T = 25088   # full keys-only tile; the cluster kernel fuses runs of 2T
-cases = [(1, "uniform", "u32"), (T - 3, "uniform", "u32"), (T + 1, "few", "u32"),
-         (2 * T, "uniform", "u32"), (3 * T + 17, "uniform", "u32"), (5 * T, "reverse", "u32"),
-         ((1 << 23) + 12345, "uniform", "u32"), ((1 << 23) + 99, "uniform", "i32"),
-         ((1 << 24) + 7, "few", "u32"), ((1 << 22) + 3, "sorted", "i32")]
-for n, dist, kt in cases:
-    keys = dcgen.sort_keys(n, dist, seed=43, key_type=kt, device="cuda")
-    ka = keys.cpu().numpy()
-    ka = ka.view(np.uint32) if kt == "u32" else ka.view(np.int32)
-    ek = oracle.mergesort(ka, key_type=kt)
-    for two in (False, True):
-        k = keys.clone()
-        plan = dc.Plan(n)
-        plan.set_tile_class(2)
-        plan.set_two_level(two)
-        plan.sort_(k, None, key_type=kt)
-        torch.cuda.synchronize()
-        assert np.array_equal(k.cpu().numpy().view(ek.dtype), ek), (n, dist, kt, two)
-print("variant ok")
-"""
-
-
-def test_nk1_cluster_level(tmp_path):
-    """f2 prototype: NK1 with one more merge level across a cluster of two CTAs
-    through distributed shared memory (-DDC_NK1_CLUSTER=2, nk1_blocksort_cl2):
-    bit-exact against the oracle for partial, odd and ragged tile counts, both
-    pass kinds, u32 and i32 keys."""
-    if not torch.cuda.is_available():
-        pytest.skip("no CUDA device")
-    from paper_conf_ipps_lopez_ortizss13_b200 import build
-
-    lib = build.build(out=str(tmp_path / "libdc_cl2.so"), defines=["DC_NK1_CLUSTER=2"])
-    env = dict(os.environ, DC_LIB=lib)
-    r = subprocess.run([sys.executable, "-c", CLUSTER_SCRIPT.format(root=ROOT)], env=env,
-                       capture_output=True, text=True, timeout=900)
-    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
-    assert "variant ok" in r.stdout
