@@ -631,9 +631,12 @@ def test_sort_nk1_cluster_levels(dc, oracle_mod, cs, tile_class, key_type):
             plan.set_two_level(two)
             plan.set_nk1_cluster(cs)
             assert plan.schedule(key_type)["tile"] == tile * cs
-            plan.sort_(k, None, key_type=key_type)
-            torch.cuda.synchronize()
-            assert np.array_equal(k.cpu().numpy().view(ek.dtype), ek), (n, dist, two)
+            # three runs on the same buffers: eager, graph capture, graph replay
+            for rep in range(3):
+                k.copy_(keys)
+                plan.sort_(k, None, key_type=key_type)
+                torch.cuda.synchronize()
+                assert np.array_equal(k.cpu().numpy().view(ek.dtype), ek), (n, dist, two, rep)
 
 
 def test_sort_nk1_cluster_ignored_for_stable_sorts(dc, oracle_mod):
