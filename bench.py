@@ -89,6 +89,15 @@ class L2Flush:
         torch.sum(self.buf, dim=0, out=self.out)
 
 
+def ncu_entry(kernel: str, workload: str, key: str):
+    """One field of the committed ncu --set full summary (profiles/ncu_summary.json)."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        return json.load(open(path))[workload][kernel][key]
+    except Exception:
+        return None
+
+
 def ncu_traffic(kernel: str, workload: str):
     """dram bytes per launch of `kernel` from the committed ncu --set full summary."""
     path = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -398,6 +407,25 @@ def run_dc(args, wl):
                       "hbm_gbs": achieved, "share_of_step": nk3_ms / args.steps / ms_instr},
     }
 
+    # Shared-memory roofline of the two merge kernels (both bound by shared-memory
+    # wavefronts): LSU wavefronts per launch from the committed
+    # ncu capture of the same workload / live launch time, against one wavefront
+    # per clock per SM at the clock NVML saw during the timed loop.
+    csum = clk.summary()
+    mhz = csum.get("sm_mhz") or csum.get("sm_max_mhz")
+    if mhz:
+        speak = torch.cuda.get_device_properties(local).multi_processor_count * float(mhz) * 1e6
+        smem = {"unit": "wavefronts/s", "peak": speak,
+                "peak_source": "1 wavefront / clock / SM x SMs x NVML SM clock; TMA traffic excluded",
+                "wavefronts_source": "profiles/ncu_summary.json (ncu l1tex shared ld + st wavefronts)"}
+        for name, kern, avg in (("nk1_blocksort", "nk1_blocksort", nk1_avg),
+                                ("nk3_merge", "nk3_merge4" if two else "nk3_merge", nk3_avg)):
+            w = ncu_entry(kern, wl, "smem_wavefronts_per_launch")
+            if w and avg:
+                kernels[name]["smem_roofline"] = dict(smem, wavefronts_per_launch=w,
+                                                      achieved=w / (avg / 1e3),
+                                                      frac=w / (avg / 1e3) / speak)
+
     e2e = None
     if not args.no_e2e:
         e2e = e2e_sort(args, plan, n, kv, pristine_k, pristine_v)
@@ -428,7 +456,7 @@ def run_dc(args, wl):
                    "instrumented_step_ms": ms_instr,
                    "sorted_check": sorted_ok},
         "roofline": roofline, "kernels": kernels, "gpu_launches": launches,
-        "clocks": clk.summary(), "e2e": e2e, "cpu_baseline": cpu,
+        "clocks": csum, "e2e": e2e, "cpu_baseline": cpu,
     }), flush=True)
 
 

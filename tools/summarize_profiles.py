@@ -82,9 +82,15 @@ for cap, (wl, kern) in caps.items():
     json.dump(s, open(os.path.join(out, f"ncu_{wl}_{kern}.json"), "w"), indent=1)
     rd = float(s["dram__bytes_read.sum"].split()[0]) * (1e9 if "Gbyte" in s["dram__bytes_read.sum"] else 1e6 if "Mbyte" in s["dram__bytes_read.sum"] else 1e3)
     wr = float(s["dram__bytes_write.sum"].split()[0]) * (1e9 if "Gbyte" in s["dram__bytes_write.sum"] else 1e6 if "Mbyte" in s["dram__bytes_write.sum"] else 1e3)
-    summary.setdefault(wl, {})[kern] = {"dram_bytes_per_launch": rd + wr,
-                                        "duration": s["gpu__time_duration.sum"],
-                                        "source": f"profiles/{rnd}/ncu_{wl}_{kern}.json"}
+    ent = {"dram_bytes_per_launch": rd + wr, "duration": s["gpu__time_duration.sum"],
+           "source": f"profiles/{rnd}/ncu_{wl}_{kern}.json"}
+    try:   # shared-memory wavefronts of LSU loads + stores (TMA traffic not included)
+        ent["smem_wavefronts_per_launch"] = (
+            float(s["l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum"])
+            + float(s["l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum"]))
+    except (KeyError, ValueError):
+        pass
+    summary.setdefault(wl, {})[kern] = ent
     print(wl, kern, s["gpu__time_duration.sum"], f"dram {(rd + wr) / 1e9:.4f} GB")
 json.dump(summary, open(os.path.join(ROOT, "profiles", "ncu_summary.json"), "w"), indent=1)
 
