@@ -133,7 +133,7 @@ dc_status fail(dc_status s, const std::string& msg) {
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 int nk1_smem_bytes(SortCfg c, bool vals) {
-    return (vals ? 3 : 1) * dc::tile_words(c.tile(), 0) * 4;
+    return (vals ? (DC_NK1_KV_LATE ? 2 : 3) : 1) * dc::tile_words(c.tile(), 0) * 4;
 }
 int nk3_smem_bytes(SortCfg c, bool vals) {
     return (vals ? 2 : 1) * dc::tile_words(c.tout(), c.it + 16) * 4;

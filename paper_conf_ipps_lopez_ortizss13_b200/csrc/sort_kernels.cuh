@@ -351,6 +351,13 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
 //   4. the sorted tile leaves by one TMA bulk store.
 // With values (V): the merges carry the tile-local index of every key; the
 // values wait in shared memory and are gathered by index at the end.
+// Key-value NK1: the values are loaded after the last merge level, into the
+// index region, so a CTA needs two tile regions instead of three (256 x 33:
+// 67.6 KB, three CTAs per SM instead of two): NK1 3.33 -> 2.87 ms per 2^28
+// key-value sort (r02b).  0 loads them with the keys into a third region.
+#ifndef DC_NK1_KV_LATE
+#define DC_NK1_KV_LATE 1
+#endif
 template <int NT, int IT, class K, bool V>
 __global__ void __launch_bounds__(NT)
 nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in_v,
@@ -362,7 +369,10 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     extern __shared__ __align__(16) uint32_t smem[];
     uint32_t* sk = smem;              // [TW] keys
     uint32_t* si = smem + TW;         // [TW] tile-local indices, then gathered values (V)
-    uint32_t* sv = smem + 2 * TW;     // [TW] values, by original position (V)
+    // [TW] values by original position (V).  DC_NK1_KV_LATE: the values arrive
+    // after the last merge level, into the index region (the indices are in
+    // registers by then), so the CTA needs two regions instead of three.
+    uint32_t* sv = DC_NK1_KV_LATE ? si : smem + 2 * TW;
     __shared__ __align__(8) uint64_t bar;
     const uint32_t SK = smem_addr(sk);
     const uint32_t BAR = smem_addr(&bar);
@@ -374,17 +384,18 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     const int body = count & ~3;       // 16-byte part moved by TMA
 
     // ---- 1. load
+    constexpr bool kEarlyV = V && !DC_NK1_KV_LATE;
     if (tid == 0) {
         mbar_init(BAR, 1);
-        mbar_arrive_expect_tx(BAR, 4u * body * (V ? 2 : 1));
+        mbar_arrive_expect_tx(BAR, 4u * body * (kEarlyV ? 2 : 1));
         if (body > 0) {
             bulk_g2s(SK, in_k + base, 4u * body, BAR);
-            if (V) bulk_g2s(smem_addr(sv), in_v + base, 4u * body, BAR);
+            if (kEarlyV) bulk_g2s(smem_addr(sv), in_v + base, 4u * body, BAR);
         }
     }
     for (int e = body + tid; e < TILE; e += NT) {   // ragged tail + pads
         sk[e] = e < count ? in_k[base + e] : K::kPad;
-        if (V) sv[e] = e < count ? in_v[base + e] : 0u;
+        if (kEarlyV) sv[e] = e < count ? in_v[base + e] : 0u;
     }
     __syncthreads();                  // barrier init + tail visible
     mbar_wait(BAR, 0);
@@ -429,11 +440,31 @@ nk1_blocksort(const uint32_t* __restrict__ in_k, const uint32_t* __restrict__ in
     }
 
     // ---- 4. store: blocked write into shared memory, one bulk store
+    if (V && DC_NK1_KV_LATE) fence_proxy_async_smem();   // index writes before the TMA refill
     __syncthreads();
+    if constexpr (V && DC_NK1_KV_LATE) {
+        // the values by original position into the (now free) index region
+        if (tid == 0) {
+            mbar_arrive_expect_tx(BAR, 4u * body);
+            if (body > 0) bulk_g2s(smem_addr(sv), in_v + base, 4u * body, BAR);
+        }
+        for (int e = body + tid; e < TILE; e += NT) sv[e] = e < count ? in_v[base + e] : 0u;
 #pragma unroll
-    for (int j = 0; j < IT; ++j) {
-        sk[tid * IT + j] = k[j];
-        if (V) si[tid * IT + j] = sv[ix[j]];    // gather the values by index
+        for (int j = 0; j < IT; ++j) sk[tid * IT + j] = k[j];
+        __syncthreads();                  // barrier phase 1 armed, tail written
+        mbar_wait(BAR, 1);
+        uint32_t vv[IT];
+#pragma unroll
+        for (int j = 0; j < IT; ++j) vv[j] = sv[ix[j]];   // gather the values by index
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < IT; ++j) si[tid * IT + j] = vv[j];
+    } else {
+#pragma unroll
+        for (int j = 0; j < IT; ++j) {
+            sk[tid * IT + j] = k[j];
+            if (V) si[tid * IT + j] = sv[ix[j]];    // gather the values by index
+        }
     }
     fence_proxy_async_smem();
     __syncthreads();
