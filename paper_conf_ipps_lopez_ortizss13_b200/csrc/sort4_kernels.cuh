@@ -269,6 +269,9 @@ __device__ __forceinline__ Cut4 select4_warp(const Pass4& P, int j, bool valid =
     bool more = true;
     for (; more && round < DC_SEL4_EXACT_FROM; ++round) more = round_step(std::false_type{});
     for (; more; ++round) more = round_step(std::true_type{});
+#ifdef DC_SEL4_ROUNDS_OUT   // measurement hook (tools/select4_rounds.cu): rounds per boundary
+    if (valid && ll == 0) DC_SEL4_ROUNDS_OUT[j] = round;
+#endif
     Cut4 c;
 #pragma unroll
     for (int r = 0; r < 4; ++r) c.c[r] = lo[r];
