@@ -349,8 +349,8 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
 //   3. levels with runs IT .. TILE/2: merge-path in shared memory, each
 //      thread merging IT outputs serially;
 //   4. the sorted tile leaves by one TMA bulk store.
-// With values (V): the merges carry the tile-local index of every key; the
-// values wait in shared memory and are gathered by index at the end.
+// With values (V): the merges carry the tile-local index of every key, and
+// the values are gathered by index at the end.
 // Key-value NK1: the values are loaded after the last merge level, into the
 // index region, so a CTA needs two tile regions instead of three (256 x 33:
 // 67.6 KB, three CTAs per SM instead of two): NK1 3.33 -> 2.87 ms per 2^28
