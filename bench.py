@@ -413,7 +413,7 @@ def run_dc(args, wl):
     # per clock per SM at the clock NVML saw during the timed loop.
     csum = clk.summary()
     mhz = csum.get("sm_mhz") or csum.get("sm_max_mhz")
-    if mhz:
+    if mhz and args.dist == "uniform":   # (the ncu capture is of the uniform workload)
         speak = torch.cuda.get_device_properties(local).multi_processor_count * float(mhz) * 1e6
         smem = {"unit": "wavefronts/s", "peak": speak,
                 "peak_source": "1 wavefront / clock / SM x SMs x NVML SM clock; TMA traffic excluded",
