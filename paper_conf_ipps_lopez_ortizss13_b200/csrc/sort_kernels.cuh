@@ -270,6 +270,92 @@ __device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uin
     if (t < count - tail0) dst[tail0 + t] = s[h + tail0 + t];
 }
 
+// ------------------------------------- first merge level by warp shuffles
+// Keys-only: after the in-register network every thread holds one sorted run
+// of IT keys; threads 2t and 2t+1 (lanes of one warp) merge theirs without
+// shared memory.  The bitonic split min(A[j], B[IT-1-j]) / max(...) gives the
+// lower / upper IT keys as bitonic sequences; the odd lane works on bit
+// complements (~x reverses the order), so both lanes run the same
+// instructions: exchange by one shuffle per key, take the minimum, sort the
+// resulting ascending-then-descending sequence with a bitonic merge network
+// (padded to a power of two with virtual minima that never cost an
+// instruction, generated at compile time), and the odd lane un-complements and
+// reverses.  Replaces one shared-memory level (~5 wavefronts per 32 keys:
+// store, co-rank and conflicted merge loads) by one shuffle per key plus ALU.
+template <int N>
+struct BitonicPadNet {
+    static constexpr int P2 = (N <= 1) ? 1 : (N <= 2) ? 2 : (N <= 4) ? 4 : (N <= 8) ? 8
+                            : (N <= 16) ? 16 : (N <= 32) ? 32 : (N <= 64) ? 64 : 128;
+    struct Arr {
+        int cnt;
+        short a[1024];
+        short b[1024];
+        short fin[128];   // fin[k]: register holding the k-th smallest after the network
+    };
+    static constexpr Arr make() {
+        Arr r{};
+        int map[P2] = {};
+        bool pad[P2] = {};
+        for (int p = 0; p < P2; ++p) { map[p] = p < N ? p : -1; pad[p] = p >= N; }
+        r.cnt = 0;
+        for (int d = P2 / 2; d >= 1; d /= 2)
+            for (int i = 0; i < P2; ++i) {
+                if (i & d) continue;
+                const int j = i + d;
+                if (pad[i] && pad[j]) continue;
+                if (pad[j]) {          // j holds a virtual minimum: it moves to i for free
+                    map[j] = map[i]; map[i] = -1; pad[i] = true; pad[j] = false;
+                    continue;
+                }
+                if (pad[i]) continue;  // i already holds the minimum
+                r.a[r.cnt] = (short)map[i];
+                r.b[r.cnt] = (short)map[j];
+                ++r.cnt;
+            }
+        for (int k = 0; k < N; ++k) r.fin[k] = (short)map[P2 - N + k];
+        return r;
+    }
+    static constexpr Arr net = make();
+};
+
+template <int N, class F, int... C>
+__device__ __forceinline__ void bitonic_pad_apply(F& f, std::integer_sequence<int, C...>) {
+    (f(std::integral_constant<int, BitonicPadNet<N>::net.a[C]>{},
+       std::integral_constant<int, BitonicPadNet<N>::net.b[C]>{}),
+     ...);
+}
+
+template <int N, int... J>
+__device__ __forceinline__ void bitonic_pad_final(uint32_t (&s)[N], const uint32_t (&u)[N],
+                                                  std::integer_sequence<int, J...>) {
+    ((s[J] = u[BitonicPadNet<N>::net.fin[J]]), ...);
+}
+
+template <int IT, class K>
+__device__ __forceinline__ void merge_level_shfl(uint32_t (&k)[IT]) {
+    const uint32_t m = (threadIdx.x & 1) ? 0xFFFFFFFFu : 0u;
+    const bool odd = threadIdx.x & 1;
+    uint32_t u[IT];
+#pragma unroll
+    for (int j = 0; j < IT; ++j) u[j] = (odd ? k[IT - 1 - j] : k[j]) ^ m;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+        const uint32_t r = __shfl_xor_sync(0xffffffffu, u[j], 1) ^ 0xFFFFFFFFu;
+        u[j] = K::mn(u[j], r);
+    }
+    auto cas = [&](auto a, auto b) {
+        constexpr int A = decltype(a)::value, B = decltype(b)::value;
+        const uint32_t lo = K::mn(u[A], u[B]), hi = K::mx(u[A], u[B]);
+        u[A] = lo;
+        u[B] = hi;
+    };
+    bitonic_pad_apply<IT>(cas, std::make_integer_sequence<int, BitonicPadNet<IT>::net.cnt>{});
+    uint32_t s[IT];
+    bitonic_pad_final<IT>(s, u, std::make_integer_sequence<int, IT>{});
+#pragma unroll
+    for (int j = 0; j < IT; ++j) k[j] = (odd ? s[IT - 1 - j] : s[j]) ^ m;
+}
+
 // ------------------------------------------- keys-only bitonic merge levels
 // Keys-only u32/i32 (equal keys are identical bit patterns, so which copy of
 // an equal key is emitted first is unobservable): every B run is stored
@@ -279,6 +365,11 @@ __device__ __forceinline__ void store_tile(uint32_t* __restrict__ dst, const uin
 // into the other run from that run's LARGEST end, so the value it reads is
 // >= every element still pending and the plain comparison "b < a" keeps
 // selecting the right side: no bounds checks, one tracked pointer.
+// r02b: NK1 1.866 -> 1.814 ms per 2^28 u32 sort (5.90 -> 5.85 ms per step);
+// 0 runs level 0 in shared memory like the others.
+#ifndef DC_NK1_SHFL_L0
+#define DC_NK1_SHFL_L0 1
+#endif
 template <int NT, int IT, class K>
 __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t* sk) {
     constexpr int TILE = NT * IT;
@@ -291,8 +382,16 @@ __device__ __forceinline__ void merge_levels_bitonic(uint32_t (&k)[IT], uint32_t
     // and the diagonal are shifts and masks (runtime divisions by w compiled
     // to ~20-instruction float sequences, ~4 % of NK1's issue slots in r01)
     int lg = 0;
+    int w0 = IT;
+#if DC_NK1_SHFL_L0
+    if (TILE >= 2 * IT) {            // level 0 (runs of IT -> 2 IT) without shared memory
+        merge_level_shfl<IT, K>(k);
+        w0 = 2 * IT;
+        lg = 1;
+    }
+#endif
 #pragma unroll 1
-    for (int w = IT; w < TILE && w < DC_NK1_STOPW; w *= 2, ++lg) {
+    for (int w = w0; w < TILE && w < DC_NK1_STOPW; w *= 2, ++lg) {
         // Levels whose pairs fit in one warp (2w <= 32*IT) only touch that
         // warp's own region: a warp barrier suffices and warps drift apart
         // (search / merge / write phases overlap across warps).
