@@ -220,11 +220,12 @@ __device__ __forceinline__ Cut4 select4_warp(const Pass4& P, int j, bool valid =
             const bool other = r != q;
             dt |= other & (lo[r] > 0) & !precedes<K>(elo[r], r, v, q);      // E before a taken edge
             du |= other & (hi[r] < g.l[r]) & precedes<K>(ehi[r], r, v, q);  // untaken edge before E
-            int Lp = lo[r], Up = hi[r];
-            if (W[r] > 0) {
-                if (a > 0) Lp = sel4_pivot<PV>(lo[r], W[r], st[r], a - 1) + 1;
-                if (a < PV) Up = sel4_pivot<PV>(lo[r], W[r], st[r], a);
-            }
+            // (branch-free: the positions of pivots a-1 and a of run r)
+            const bool big = W[r] >= PV + 1;
+            const int pa1 = lo[r] + (big ? a * st[r] : min(a - 1, W[r] - 1));
+            const int pa = lo[r] + (big ? (a + 1) * st[r] : min(a, W[r] - 1));
+            int Lp = (W[r] > 0) & (a > 0) ? pa1 + 1 : lo[r];
+            int Up = (W[r] > 0) & (a < PV) ? pa : hi[r];
             if constexpr (exact) {
                 if (other && !(dt | du) && active) {
                     int x0 = Lp, x1 = Up;                // first position not preceding E
@@ -254,14 +255,12 @@ __device__ __forceinline__ Cut4 select4_warp(const Pass4& P, int j, bool valid =
             const uint32_t vt = __shfl_sync(0xffffffffu, v, base + PV * r + tt);
             const uint32_t vu = __shfl_sync(0xffffffffu, v, base + PV * r + tu);
             const int lo0 = lo[r];                          // this round's pivot base
-            if (gt) {
-                elo[r] = vt;
-                lo[r] = sel4_pivot<PV>(lo0, W[r], st[r], tt) + 1;
-            }
-            if (gu) {
-                ehi[r] = vu;
-                hi[r] = sel4_pivot<PV>(lo0, W[r], st[r], tu);
-            }
+            const int nlo = sel4_pivot<PV>(lo0, W[r], st[r], tt) + 1;
+            const int nhi = sel4_pivot<PV>(lo0, W[r], st[r], tu);
+            elo[r] = gt ? vt : elo[r];                      // (branch-free updates)
+            lo[r] = gt ? nlo : lo[r];
+            ehi[r] = gu ? vu : ehi[r];
+            hi[r] = gu ? nhi : hi[r];
         }
         return true;
     };
