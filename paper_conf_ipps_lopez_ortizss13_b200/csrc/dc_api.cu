@@ -370,7 +370,10 @@ dc_status pass4(dc_plan_t p, const dc::Pass4& P, int tiles, dc::Cut4* cuts, uint
 #ifndef DC_SEL4_PV_KV
 #define DC_SEL4_PV_KV 2   // r02b: 0.689 -> 0.652 ms per 2^28 key-value sort (PV 4 before the branch-free rounds)
 #endif
-        constexpr int PV = V ? DC_SEL4_PV_KV : 2;   // pivots per run (sort4_kernels.cuh)
+#ifndef DC_SEL4_PV_KEYS
+#define DC_SEL4_PV_KEYS 2
+#endif
+        constexpr int PV = V ? DC_SEL4_PV_KV : DC_SEL4_PV_KEYS;   // pivots per run (sort4_kernels.cuh)
         constexpr int bpw = dc::sel4_bpw<PV>();
         const int sel_warps = (tiles + bpw - 1) / bpw;
         dc::nk2_select4<K, PV><<<(sel_warps + 3) / 4, 128, 0, st>>>(P, tiles, cuts);
