@@ -136,6 +136,42 @@ def test_schedule(n, kt, vals):
         assert s["fused_levels"] + s["global_passes"] >= math.ceil(math.log2(n))
 
 
+@pytest.mark.parametrize("cs", [2, 4, 8, 16])
+@pytest.mark.parametrize("n", [100, 25088 * 3 + 1, 1 << 20, 1 << 28])
+def test_nk1_cluster_schedule(cs, n):
+    """f2 cluster levels (dc_plan_set_nk1_cluster): keys-only u32/i32 sorts fuse
+    cs tiles per run (log2 cs more levels on chip, as many fewer above); key-value
+    and f32 sorts ignore the setting; the planner's rule leaves it off (cs = 1);
+    any size other than 0/1/2/4/8/16 is rejected."""
+    for kt in ("u32", "i32"):
+        p0 = dc.Plan(n)
+        base = p0.schedule(kt)
+        assert p0.schedule(kt) == base
+        p = dc.Plan(n)
+        p.set_nk1_cluster(cs)
+        s = p.schedule(kt)
+        assert s["tile"] == base["tile"] * cs
+        assert s["fused_levels"] == math.ceil(math.log2(s["tile"]))
+        assert s["global_passes"] == max(0, math.ceil(math.log2(math.ceil(n / s["tile"]))))
+        p.set_nk1_cluster(1)
+        assert p.schedule(kt) == base
+        p.set_nk1_cluster(0)
+        assert p.schedule(kt) == base                 # the planner's rule: no cluster levels
+    for kt, vals in (("u32", True), ("f32", False)):
+        p = dc.Plan(n)
+        ref = p.schedule(kt, vals)
+        p.set_nk1_cluster(cs)
+        assert p.schedule(kt, vals) == ref
+
+
+@pytest.mark.parametrize("cs", [-1, 3, 5, 32])
+def test_nk1_cluster_rejects_other_sizes(cs):
+    p = dc.Plan(1 << 20)
+    with pytest.raises(Exception):
+        p.set_nk1_cluster(cs)
+    assert dc.lib().dc_plan_set_nk1_cluster(p._h, cs) == 1   # DC_ERR_INVALID_ARG
+
+
 def test_scratch_is_the_papers_2n_working_space():
     # P:L1182-1183: "working space of 2n*sizeof(int)" -> input + one n-int temp
     golden = json.load(open(os.path.join(ROOT, "tests", "golden", "paper_numbers.json")))
