@@ -1,13 +1,16 @@
 """Reading R21: chunk-label index recovery for max-subarray.
 
-The values-only NK4 variant (-DDC_MS_VONLY=1) folds each chunk of L elements
+The values-only NK4 (the default since r02b; -DDC_MS_VONLY=0 is the indexed
+variant) folds each chunk of L elements
 without indices, labels the chunk leaf by its start, combines the leaves with
 the ordered tie rules of the D&C combine (R10), and then
 re-scans at most four chunks for the exact (pe, ss, bs, be).  This test checks
 that claim in plain Python against the oracle (lexicographically smallest
 optimal (start, end), R10) and against numpy's first argmax of the prefix and
 suffix sums, on tie-heavy arrays and every chunk size 1..9.  It pins the
-reading only; the CUDA variant is checked by tests/test_gpu_variants.py.
+reading only; the CUDA kernel is checked against the oracle by the maxsub tests
+of tests/test_gpu_parity.py (tie-heavy, degenerate, tuple) and the indexed
+variant by tests/test_gpu_variants.py.
 """
 import numpy as np
 
@@ -88,3 +91,39 @@ def test_chunk_label_recovery_matches_oracle():
         a = x.astype(np.int64)
         assert pe == int(np.argmax(np.cumsum(a))), (x.tolist(), L)
         assert ss == int(np.argmax(np.cumsum(a[::-1])[::-1])), (x.tolist(), L)
+
+
+def _in_chunk_prefix_rule(xs):
+    """r02b's warp-parallel in-chunk recovery (maxsub_tma.cuh ms_par_kadane):
+    s_e = first argmin of Q_q = P_{q-1} over q in [0, e] (P_{-1} = 0),
+    e* = first argmax of P_e - Q_{s_e}; returns (value, s_{e*}, e*)."""
+    best, bs, be = None, 0, 0
+    P, qmin, qarg = 0, None, 0
+    for e, v in enumerate(xs):
+        Q = P                          # P_{e-1}
+        if qmin is None or Q < qmin:   # strict: the first minimum
+            qmin, qarg = Q, e
+        P += v
+        val = P - qmin
+        if best is None or val > best:   # strict: the first maximum
+            best, bs, be = val, qarg, e
+    return best, bs, be
+
+
+def test_in_chunk_prefix_rule_is_the_lexicographic_minimum():
+    """Pins the in-chunk rule of the warp-parallel recovery against brute force
+    (the lexicographically smallest optimal (start, end), reading R10) on
+    tie-heavy and random chunks: every optimal (s, e) has s_e <= s with (s_e, e)
+    optimal, and s_e does not decrease with e, so the first optimal e gives the
+    lexicographic minimum (R21)."""
+    rng = np.random.default_rng(2102)
+    for it in range(4000):
+        n = int(rng.integers(1, 30))
+        if it % 3 == 0:
+            xs = [int(v) for v in rng.integers(-1, 2, n)]
+        elif it % 3 == 1:
+            xs = [int(v) for v in rng.integers(-3, 3, n)]
+        else:
+            xs = [int(v) for v in rng.integers(-(1 << 31), 1 << 31, n, dtype=np.int64)]
+        brute = max((sum(xs[s:e + 1]), -s, -e) for s in range(n) for e in range(s, n))
+        assert _in_chunk_prefix_rule(xs) == (brute[0], -brute[1], -brute[2]), xs
